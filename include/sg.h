@@ -1,0 +1,181 @@
+/*
+ * sg.h — C ABI of libsg, the B200 (sm_100a) sampled-threshold Gustavson SpGEMM.
+ *
+ * The operation is C = A·B on CSR inputs, "A with n rows and m columns, B with m rows and k
+ * columns ... Resultant Matrix C with n rows and k columns" (Alg. 2), computed
+ * row by row (Gustavson; Alg. 2 l.5-6, L222-L223). Rows are routed between a light
+ * and a heavy kernel path by a threshold t on the per-row work volume w_i = L_AB[i],
+ * heavy iff w_i > t, and t is chosen by the paper's Sample -> Identify ->
+ * Extrapolate procedure (Fig. 2). Row ranges for several GPUs are cut on the work
+ * prefix (Alg. 2 l.1-4, L215-L218; threshold vector, L106). "PAPER Lnnn" is line nnn of the paper
+ * text; DESIGN.md lists every reading taken where it is ambiguous.
+ *
+ * Conventions shared by every entry point
+ *  - Matrices are canonical CSR: row_ptr int64[nrows+1] (row_ptr[0] == 0), col_idx int32[nnz]
+ *    strictly ascending within each row, values fp64 or fp32[nnz]. A and B must have the same
+ *    value dtype; C gets that dtype. Inputs are BORROWED device pointers, never freed by sg.
+ *  - Pointers are DEVICE pointers unless marked (host). Scalars marked (host) are written by the
+ *    call before it returns (the call synchronises the stream for them).
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream). Work is
+ *    stream-ordered; the only host synchronisations are the documented host outputs.
+ *  - Every call returns a status and never throws across the ABI. On error, caller-owned outputs
+ *    are left untouched where possible and a plan involved in the failure is poisoned (every later
+ *    call with it returns SG_ERR_CUDA); destroy it with sg_plan_destroy.
+ *  - Structural semantics: C has an entry wherever some product a_ik*b_kj exists, even if the
+ *    values cancel to zero (reading R9). Columns of each C row are ascending.
+ */
+#ifndef SG_H
+#define SG_H
+
+#include <stdint.h>
+#include <stddef.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    SG_OK = 0,
+    SG_ERR_INVALID_ARG = 1,   /* null pointer, sample_frac outside (0,1], thr outside [0,cap_L], bad row range */
+    SG_ERR_SHAPE = 2,         /* A.ncols != B.nrows, or a buffer shape mismatch */
+    SG_ERR_DTYPE = 3,         /* A and B value dtypes differ, or unknown dtype */
+    SG_ERR_NOT_CANONICAL = 4, /* only with SG_VALIDATE=1 in the environment: unsorted/duplicate/out-of-range columns */
+    SG_ERR_EMPTY_SAMPLE = 5,  /* the sample holds no non-empty row */
+    SG_ERR_OOM = 6,           /* device workspace allocation failed */
+    SG_ERR_CUDA = 7,          /* a CUDA runtime error (or a poisoned plan) */
+    SG_ERR_NCCL = 8,          /* an NCCL error in sg_gather */
+    SG_ERR_OVERFLOW = 9       /* a dimension exceeds INT32_MAX columns, or a cost sum could overflow int64 */
+} sg_status;
+
+typedef enum { SG_F64 = 0, SG_F32 = 1 } sg_dtype;
+
+/* A borrowed view of a device CSR matrix. */
+typedef struct {
+    int64_t nrows, ncols, nnz;
+    const int64_t* row_ptr;   /* device, nrows+1 */
+    const int32_t* col_idx;   /* device, nnz */
+    const void* val;          /* device, nnz of dtype */
+    sg_dtype dtype;
+} sg_csr_view;
+
+/* Per-row path costs in integer picoseconds (the "offline relation" of PAPER L94):
+ *   c_L(i) = kappa_L + lambda_L*w_i + sigma_L*u_i*ceil(log2 max(u_i,2)) + rho_L*u_i
+ *   c_H(i) = kappa_H + lambda_H*w_i + tau_H*a_i*R(u_i) + mu_H*u_i
+ *   R(u)   = tiles_fixed if capu == 0, else max(1, ceil(u/capu))
+ * with a_i = nnz(A_i), w_i = L_AB[i], u_i = nnz(C_i). cap_L is the largest admissible
+ * threshold (the light path's table capacity); it must be <= SG_CAP_L_MAX. */
+typedef struct {
+    int64_t kappa_L, lambda_L, sigma_L, rho_L;
+    int64_t kappa_H, lambda_H, tau_H, mu_H;
+    int64_t tiles_fixed, capu, cap_L;
+} sg_cost_model;
+
+#define SG_CAP_L_MAX 4096
+
+/* What sg_sample_threshold saw (host struct). */
+typedef struct {
+    int64_t sample_rows;      /* |S| (Binomial(n, f)) */
+    int64_t sample_nonempty;  /* rows of S with w > 0 */
+    int64_t thr;              /* the returned threshold */
+    int64_t W_est_L, W_est_H; /* sum of w over sampled light / heavy rows at thr */
+    int64_t J_min;            /* min_t J(t; S) in ps (unscaled: the n/|S| factor cancels in the argmin) */
+} sg_sample_report;
+
+/* Per-class counts of a plan (host struct). */
+typedef struct {
+    int64_t row_begin, row_end, thr;
+    int64_t n_empty, n_light, n_heavy;
+    int64_t nnz_c;            /* sum of u_i over the plan's rows */
+    int64_t flops;            /* W = sum of w_i over the plan's rows (multiply-adds) */
+    int64_t n_ranges;         /* heavy column ranges (numeric work items of the heavy path) */
+    int64_t light_bins[13];   /* light rows per bin b: 2^(b-1) < w <= 2^b (b = 0: w == 1) */
+} sg_plan_info;
+
+typedef struct sg_plan sg_plan;   /* opaque; owns only its workspace */
+
+/* Human-readable status name (static storage). */
+const char* sg_status_string(sg_status st);
+/* Library version string, e.g. "sg 0.1.0 sm_100a". */
+const char* sg_version(void);
+/* The calibrated default cost model. */
+void sg_default_cost_model(sg_cost_model* out /*host*/);
+
+/* Row work volume w_i = sum_{k in A_i} nnz(B_k) = L_AB[i] (Alg. 2 l.1 L215) for rows
+ * [row_begin, row_end) into w_out[0 .. row_end-row_begin) (device, caller-owned). If total_out is
+ * non-NULL the sum W is written there (host; synchronises). */
+sg_status sg_row_work(const sg_csr_view* A, const sg_csr_view* B, int64_t row_begin, int64_t row_end,
+                      int64_t* w_out, int64_t* total_out /*host, nullable*/, void* stream);
+
+/* Sample -> Identify -> Extrapolate: draws the Bernoulli(sample_frac) row sample
+ * S = { i : h(seed, SAMPLE, i) < floor(sample_frac*2^64) } (uniform sampling, L92; R4),
+ * computes (w_i, a_i, u_i) for i in S on the device (u_i by an exact sample-symbolic pass), and
+ * returns thr = the smallest minimiser of J(t;S) = sum_{i in S, 0<w_i<=t} c_L(i) + sum_{i in S,
+ * w_i>t} c_H(i) over t in {0} u {w_i : i in S, 0 < w_i <= cap_L} (Identify, L87-L89). Extrapolation
+ * is the identity (r = r', L236). cm == NULL uses sg_default_cost_model. Synchronises.
+ * Errors: INVALID_ARG (sample_frac outside (0,1]), EMPTY_SAMPLE, SHAPE, DTYPE. */
+sg_status sg_sample_threshold(const sg_csr_view* A, const sg_csr_view* B, double sample_frac, uint64_t seed,
+                              const sg_cost_model* cm, int64_t* thr_out /*host*/,
+                              sg_sample_report* rep /*host, nullable*/, void* stream);
+
+/* The exhaustive threshold thr* = thr over ALL rows (needs u_i for every row, i.e. a full
+ * symbolic pass — what the paper calls "not practical", L198, L246). Used for the gap report. */
+sg_status sg_exhaustive_threshold(const sg_csr_view* A, const sg_csr_view* B, const sg_cost_model* cm,
+                                  int64_t* thr_out /*host*/, int64_t* J_min_out /*host, nullable*/, void* stream);
+
+/* J(t; all rows) for an explicit list of thresholds (host arrays of length nt), for the gap report.
+ * Needs a full symbolic pass, like sg_exhaustive_threshold. Synchronises. */
+sg_status sg_cost_curve(const sg_csr_view* A, const sg_csr_view* B, const sg_cost_model* cm,
+                        int64_t nt, const int64_t* t_host, int64_t* J_host /*host, nt*/, void* stream);
+
+/* Work-balanced contiguous row blocks for nparts GPUs (Alg. 2 l.2-4, L216-L218, as a vector L106):
+ * cuts_out[0] = 0, cuts_out[nparts] = A.nrows, and cuts_out[g] (0<g<nparts) is the boundary j whose
+ * work prefix P[j] = sum_{i<j} w_i is closest to floor(g*W/nparts), ties to the smaller j, made
+ * monotone. Part g owns rows [cuts_out[g], cuts_out[g+1]). flops_out = W. Synchronises. */
+sg_status sg_partition(const sg_csr_view* A, const sg_csr_view* B, int nparts,
+                       int64_t* cuts_out /*host, nparts+1*/, int64_t* flops_out /*host, nullable*/, void* stream);
+
+/* Symbolic phase for rows [row_begin, row_end) at threshold thr (0 <= thr <= SG_CAP_L_MAX):
+ * classifies rows (EMPTY w=0, LIGHT 0<w<=thr, HEAVY w>thr; L272-L274), computes u_i = nnz(C_i)
+ * exactly and writes the local exclusive prefix C_row_ptr[0..row_end-row_begin] (device,
+ * caller-owned; C_row_ptr[0] = 0). nnz_c_out (host) = C_row_ptr[last]; synchronises so the caller
+ * can allocate C. *plan_out receives a plan owning the routing workspace for sg_numeric. */
+sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, int64_t row_begin, int64_t row_end,
+                      int64_t* C_row_ptr, int64_t* nnz_c_out /*host*/, sg_plan** plan_out /*host*/, void* stream);
+
+/* Numeric phase: writes C_col (int32[nnz_c]) and C_val (dtype[nnz_c]) for the plan's rows, each
+ * row at [C_row_ptr[i], C_row_ptr[i+1]) with ascending columns; c_ij = sum_k a_ik*b_kj accumulated
+ * in fp64 (stored in the input dtype). A and B must be the views given to sg_symbolic. */
+sg_status sg_numeric(sg_plan* plan, const sg_csr_view* A, const sg_csr_view* B,
+                     int32_t* C_col, void* C_val, void* stream);
+
+/* Assembly of the row-distributed C (Alg. 2 l.7, L224) over NCCL: rank r of the communicator owns
+ * the plan rows [row_begin_r, row_end_r) (contiguous, in rank order, covering [0, n)). Gathers the
+ * per-rank nnz (allgather), writes the GLOBAL row_ptr (n+1, device) on every rank (allgatherv of
+ * the local prefixes + offset fix-up) and, if gather_values != 0, the full C_col / C_val (nnz_total,
+ * device) on every rank. nccl_comm is an ncclComm_t (e.g. ProcessGroupNCCL._comm_ptr()).
+ * local_row_ptr / local_col / local_val are this rank's sg_symbolic / sg_numeric outputs.
+ * nnz_total_out (host). Synchronises. Errors: NCCL, SHAPE (ranges not contiguous). */
+sg_status sg_gather(sg_plan* plan, void* nccl_comm, int gather_values,
+                    const int64_t* local_row_ptr, const int32_t* local_col, const void* local_val,
+                    int64_t* C_row_ptr_global, int32_t* C_col_global /*nullable*/, void* C_val_global /*nullable*/,
+                    int64_t* nnz_total_out /*host*/, void* stream);
+
+/* Plan introspection for tests and reports. */
+sg_status sg_plan_get_info(const sg_plan* plan, sg_plan_info* out /*host*/);
+/* Row classes of the plan's rows: 0 EMPTY, 1 LIGHT, 2 HEAVY (device int8, row_end-row_begin). */
+sg_status sg_plan_get_classes(const sg_plan* plan, int8_t* cls_out, void* stream);
+/* The plan's w_i (device int64, row_end-row_begin). */
+sg_status sg_plan_get_work(const sg_plan* plan, int64_t* w_out, void* stream);
+
+/* Destroys a plan (NULL is allowed). Frees its workspace stream-ordered on the plan's stream. */
+void sg_plan_destroy(sg_plan* plan);
+
+/* The sample set S itself (device int64 row ids in ascending order, capacity rows_cap) and its
+ * size (host), for parity tests of the sampler. Rows in [row_begin, row_end). */
+sg_status sg_sample_rows(int64_t row_begin, int64_t row_end, double sample_frac, uint64_t seed,
+                         int64_t* rows_out, int64_t rows_cap, int64_t* count_out /*host*/, void* stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SG_H */

@@ -1,0 +1,350 @@
+"""paper_conf_icpp_hardhikbrks17_b200 — B200-native sampled-threshold Gustavson SpGEMM.
+
+A thin ctypes binding over the C ABI of ``libsg.so`` (declared in ``include/sg.h``). Every step of
+the path runs in the library's sm_100a kernels; this module only marshals arguments. PyTorch is
+used for device memory, streams and ``torch.distributed`` process groups. There is no CPU
+fallback: importing works anywhere the library builds, but every call needs a CUDA device and the
+compiled ``libsg.so``; without them it raises.
+
+Entry points keep the C names (``sg_sample_threshold``, ``sg_partition``, ``sg_symbolic``,
+``sg_numeric``, ``sg_gather``, ...) plus ``spgemm()``, the one-call user API:
+Sample -> Identify -> Extrapolate picks the routing threshold, then the
+two-phase Gustavson product (Alg. 2 l.5-6 L222-L223) runs on the device.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+
+import torch
+
+from . import _build
+
+__all__ = [
+    "DeviceCSR", "CostModel", "SampleReport", "PlanInfo", "SgError", "Plan", "lib", "load",
+    "sg_row_work", "sg_sample_rows", "sg_sample_threshold", "sg_exhaustive_threshold", "sg_cost_curve",
+    "sg_partition", "sg_symbolic", "sg_numeric", "sg_gather", "sg_default_cost_model", "spgemm",
+    "SG_CAP_L_MAX",
+]
+
+SG_CAP_L_MAX = 4096
+_STATUS = ["SG_OK", "SG_ERR_INVALID_ARG", "SG_ERR_SHAPE", "SG_ERR_DTYPE", "SG_ERR_NOT_CANONICAL",
+           "SG_ERR_EMPTY_SAMPLE", "SG_ERR_OOM", "SG_ERR_CUDA", "SG_ERR_NCCL", "SG_ERR_OVERFLOW"]
+
+# every symbol include/sg.h declares (checked by tests/test_abi.py)
+EXPORTS = ["sg_status_string", "sg_version", "sg_default_cost_model", "sg_row_work", "sg_sample_threshold",
+           "sg_exhaustive_threshold", "sg_cost_curve", "sg_partition", "sg_symbolic", "sg_numeric", "sg_gather",
+           "sg_plan_get_info", "sg_plan_get_classes", "sg_plan_get_work", "sg_plan_destroy", "sg_sample_rows"]
+
+
+class SgError(RuntimeError):
+    def __init__(self, code: int, where: str):
+        self.code = code
+        name = _STATUS[code] if 0 <= code < len(_STATUS) else f"status {code}"
+        super().__init__(f"{where}: {name}")
+
+
+class CsrView(ctypes.Structure):
+    _fields_ = [("nrows", ctypes.c_int64), ("ncols", ctypes.c_int64), ("nnz", ctypes.c_int64),
+                ("row_ptr", ctypes.c_void_p), ("col_idx", ctypes.c_void_p), ("val", ctypes.c_void_p),
+                ("dtype", ctypes.c_int)]
+
+
+class CostModel(ctypes.Structure):
+    """sg_cost_model (integer picoseconds)."""
+    _fields_ = [(n, ctypes.c_int64) for n in (
+        "kappa_L", "lambda_L", "sigma_L", "rho_L", "kappa_H", "lambda_H", "tau_H", "mu_H",
+        "tiles_fixed", "capu", "cap_L")]
+
+    def as_dict(self):
+        return {n: int(getattr(self, n)) for n, _ in self._fields_}
+
+
+class SampleReport(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int64) for n in (
+        "sample_rows", "sample_nonempty", "thr", "W_est_L", "W_est_H", "J_min")]
+
+    def as_dict(self):
+        return {n: int(getattr(self, n)) for n, _ in self._fields_}
+
+
+class PlanInfo(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int64) for n in (
+        "row_begin", "row_end", "thr", "n_empty", "n_light", "n_heavy", "nnz_c", "flops", "n_ranges")] + [
+        ("light_bins", ctypes.c_int64 * 13)]
+
+    def as_dict(self):
+        d = {n: int(getattr(self, n)) for n, _ in self._fields_ if n != "light_bins"}
+        d["light_bins"] = [int(x) for x in self.light_bins]
+        return d
+
+
+_lib = None
+
+
+def load(build_if_missing: bool = True):
+    """Loads libsg.so (building it with nvcc if missing). Raises if it cannot."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    so = _build.SO
+    if not os.path.exists(so):
+        if not build_if_missing:
+            raise ImportError(f"{so} is missing; run __graft_entry__.build()")
+        _build.build()
+    L = ctypes.CDLL(so)
+    P, i64, u64, st = ctypes.c_void_p, ctypes.c_int64, ctypes.c_uint64, ctypes.c_int
+    V = ctypes.POINTER(CsrView)
+    CM = ctypes.POINTER(CostModel)
+    pi64 = ctypes.POINTER(ctypes.c_int64)
+    sigs = {
+        "sg_status_string": (ctypes.c_char_p, [st]),
+        "sg_version": (ctypes.c_char_p, []),
+        "sg_default_cost_model": (None, [CM]),
+        "sg_row_work": (st, [V, V, i64, i64, P, pi64, P]),
+        "sg_sample_rows": (st, [i64, i64, ctypes.c_double, u64, P, i64, pi64, P]),
+        "sg_sample_threshold": (st, [V, V, ctypes.c_double, u64, CM, pi64, ctypes.POINTER(SampleReport), P]),
+        "sg_exhaustive_threshold": (st, [V, V, CM, pi64, pi64, P]),
+        "sg_cost_curve": (st, [V, V, CM, i64, P, P, P]),
+        "sg_partition": (st, [V, V, ctypes.c_int, P, pi64, P]),
+        "sg_symbolic": (st, [V, V, i64, i64, i64, P, pi64, ctypes.POINTER(ctypes.c_void_p), P]),
+        "sg_numeric": (st, [P, V, V, P, P, P]),
+        "sg_gather": (st, [P, P, ctypes.c_int, P, P, P, P, P, P, pi64, P]),
+        "sg_plan_get_info": (st, [P, ctypes.POINTER(PlanInfo)]),
+        "sg_plan_get_classes": (st, [P, P, P]),
+        "sg_plan_get_work": (st, [P, P, P]),
+        "sg_plan_destroy": (None, [P]),
+    }
+    for name, (res, args) in sigs.items():
+        f = getattr(L, name)
+        f.restype = res
+        f.argtypes = args
+    _lib = L
+    return L
+
+
+def lib():
+    return load()
+
+
+def _check(code: int, where: str):
+    if code != 0:
+        raise SgError(code, where)
+
+
+def _stream():
+    return ctypes.c_void_p(torch.cuda.current_stream().cuda_stream)
+
+
+def _ptr(t: torch.Tensor | None):
+    return ctypes.c_void_p(t.data_ptr() if t is not None and t.numel() > 0 else 0)
+
+
+def _require_cuda():
+    if not torch.cuda.is_available():
+        raise RuntimeError("paper_conf_icpp_hardhikbrks17_b200 needs a CUDA device (no CPU fallback)")
+
+
+@dataclass
+class DeviceCSR:
+    """CSR resident in device memory (torch tensors): row_ptr int64, col int32, val f64|f32."""
+    nrows: int
+    ncols: int
+    row_ptr: torch.Tensor
+    col: torch.Tensor
+    val: torch.Tensor
+
+    @property
+    def nnz(self) -> int:
+        return int(self.col.numel())
+
+    @property
+    def dtype_code(self) -> int:
+        return 1 if self.val.dtype == torch.float32 else 0
+
+    def view(self) -> CsrView:
+        return CsrView(self.nrows, self.ncols, self.nnz, _ptr(self.row_ptr), _ptr(self.col), _ptr(self.val),
+                       self.dtype_code)
+
+    @staticmethod
+    def from_host(H, device="cuda", pin: bool = False, non_blocking: bool = False) -> "DeviceCSR":
+        """From any object with nrows, ncols, row_ptr, col, val (numpy arrays)."""
+        def t(x):
+            x = torch.from_numpy(x)
+            if pin:
+                x = x.pin_memory()
+            return x.to(device, non_blocking=non_blocking)
+        return DeviceCSR(int(H.nrows), int(H.ncols), t(H.row_ptr), t(H.col), t(H.val))
+
+    def to_host(self):
+        return (self.row_ptr.cpu().numpy(), self.col.cpu().numpy(), self.val.cpu().numpy())
+
+
+def sg_default_cost_model() -> CostModel:
+    cm = CostModel()
+    lib().sg_default_cost_model(ctypes.byref(cm))
+    return cm
+
+
+def _cmref(cm):
+    return ctypes.byref(cm) if cm is not None else None
+
+
+def sg_row_work(A: DeviceCSR, B: DeviceCSR, row_begin: int = 0, row_end: int | None = None,
+                with_total: bool = False):
+    _require_cuda()
+    row_end = A.nrows if row_end is None else row_end
+    w = torch.empty(max(row_end - row_begin, 0), dtype=torch.int64, device=A.row_ptr.device)
+    tot = ctypes.c_int64(0)
+    _check(lib().sg_row_work(ctypes.byref(A.view()), ctypes.byref(B.view()), row_begin, row_end, _ptr(w),
+                             ctypes.byref(tot) if with_total else None, _stream()), "sg_row_work")
+    return (w, int(tot.value)) if with_total else w
+
+
+def sg_sample_rows(n: int, sample_frac: float, seed: int, row_begin: int = 0, row_end: int | None = None,
+                   device="cuda") -> torch.Tensor:
+    _require_cuda()
+    row_end = n if row_end is None else row_end
+    out = torch.empty(max(row_end - row_begin, 1), dtype=torch.int64, device=device)
+    c = ctypes.c_int64(0)
+    _check(lib().sg_sample_rows(row_begin, row_end, sample_frac, seed, _ptr(out), out.numel(), ctypes.byref(c),
+                                _stream()), "sg_sample_rows")
+    return out[: c.value]
+
+
+def sg_sample_threshold(A: DeviceCSR, B: DeviceCSR, sample_frac: float, seed: int, cm: CostModel | None = None):
+    """Sample -> Identify -> Extrapolate. Returns (thr, SampleReport dict)."""
+    _require_cuda()
+    thr = ctypes.c_int64(0)
+    rep = SampleReport()
+    _check(lib().sg_sample_threshold(ctypes.byref(A.view()), ctypes.byref(B.view()), sample_frac, seed, _cmref(cm),
+                                     ctypes.byref(thr), ctypes.byref(rep), _stream()), "sg_sample_threshold")
+    return int(thr.value), rep.as_dict()
+
+
+def sg_exhaustive_threshold(A: DeviceCSR, B: DeviceCSR, cm: CostModel | None = None):
+    _require_cuda()
+    thr, J = ctypes.c_int64(0), ctypes.c_int64(0)
+    _check(lib().sg_exhaustive_threshold(ctypes.byref(A.view()), ctypes.byref(B.view()), _cmref(cm),
+                                         ctypes.byref(thr), ctypes.byref(J), _stream()), "sg_exhaustive_threshold")
+    return int(thr.value), int(J.value)
+
+
+def sg_cost_curve(A: DeviceCSR, B: DeviceCSR, ts, cm: CostModel | None = None) -> list[int]:
+    import numpy as np
+    _require_cuda()
+    t = np.ascontiguousarray(ts, dtype=np.int64)
+    J = np.zeros(t.shape[0], dtype=np.int64)
+    _check(lib().sg_cost_curve(ctypes.byref(A.view()), ctypes.byref(B.view()), _cmref(cm), t.shape[0],
+                               t.ctypes.data_as(ctypes.c_void_p), J.ctypes.data_as(ctypes.c_void_p), _stream()),
+           "sg_cost_curve")
+    return [int(x) for x in J]
+
+
+def sg_partition(A: DeviceCSR, B: DeviceCSR, nparts: int):
+    """Returns (cuts list of nparts+1, W)."""
+    import numpy as np
+    _require_cuda()
+    cuts = np.zeros(nparts + 1, dtype=np.int64)
+    W = ctypes.c_int64(0)
+    _check(lib().sg_partition(ctypes.byref(A.view()), ctypes.byref(B.view()), nparts,
+                              cuts.ctypes.data_as(ctypes.c_void_p), ctypes.byref(W), _stream()), "sg_partition")
+    return [int(x) for x in cuts], int(W.value)
+
+
+class Plan:
+    """Owns an sg_plan* and the C.row_ptr it was built with."""
+
+    def __init__(self, handle: ctypes.c_void_p, row_ptr: torch.Tensor, nnz: int, dtype: torch.dtype,
+                 row_begin: int, row_end: int):
+        self.handle = handle
+        self.row_ptr = row_ptr
+        self.nnz = nnz
+        self.dtype = dtype
+        self.row_begin, self.row_end = row_begin, row_end
+
+    def info(self) -> dict:
+        pi = PlanInfo()
+        _check(lib().sg_plan_get_info(self.handle, ctypes.byref(pi)), "sg_plan_get_info")
+        return pi.as_dict()
+
+    def classes(self) -> torch.Tensor:
+        out = torch.empty(self.row_end - self.row_begin, dtype=torch.int8, device=self.row_ptr.device)
+        _check(lib().sg_plan_get_classes(self.handle, _ptr(out), _stream()), "sg_plan_get_classes")
+        return out
+
+    def work(self) -> torch.Tensor:
+        out = torch.empty(self.row_end - self.row_begin, dtype=torch.int64, device=self.row_ptr.device)
+        _check(lib().sg_plan_get_work(self.handle, _ptr(out), _stream()), "sg_plan_get_work")
+        return out
+
+    def destroy(self):
+        if self.handle:
+            lib().sg_plan_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.destroy()
+        except Exception:
+            pass
+
+
+def sg_symbolic(A: DeviceCSR, B: DeviceCSR, thr: int, row_begin: int = 0, row_end: int | None = None) -> Plan:
+    _require_cuda()
+    row_end = A.nrows if row_end is None else row_end
+    rp = torch.empty(row_end - row_begin + 1, dtype=torch.int64, device=A.row_ptr.device)
+    nnz = ctypes.c_int64(0)
+    h = ctypes.c_void_p(0)
+    _check(lib().sg_symbolic(ctypes.byref(A.view()), ctypes.byref(B.view()), thr, row_begin, row_end, _ptr(rp),
+                             ctypes.byref(nnz), ctypes.byref(h), _stream()), "sg_symbolic")
+    return Plan(h, rp, int(nnz.value), A.val.dtype, row_begin, row_end)
+
+
+def sg_numeric(plan: Plan, A: DeviceCSR, B: DeviceCSR, out=None):
+    """Returns (C_col int32[nnz], C_val[nnz]); `out` may pass preallocated (col, val)."""
+    _require_cuda()
+    if out is None:
+        col = torch.empty(plan.nnz, dtype=torch.int32, device=A.row_ptr.device)
+        val = torch.empty(plan.nnz, dtype=plan.dtype, device=A.row_ptr.device)
+    else:
+        col, val = out
+    _check(lib().sg_numeric(plan.handle, ctypes.byref(A.view()), ctypes.byref(B.view()), _ptr(col), _ptr(val),
+                            _stream()), "sg_numeric")
+    return col, val
+
+
+def sg_gather(plan: Plan, comm_ptr: int, local_col=None, local_val=None, gather_values: bool = False,
+              n_global: int | None = None, nnz_global: int | None = None):
+    """Assembles the row-distributed C over NCCL (comm_ptr: ncclComm_t as int, e.g.
+    ProcessGroupNCCL._comm_ptr()). Returns (row_ptr_global, col_global|None, val_global|None, nnz_total)."""
+    _require_cuda()
+    dev = plan.row_ptr.device
+    n = n_global if n_global is not None else plan.row_end  # caller passes n when not the last rank
+    rp = torch.empty(n + 1, dtype=torch.int64, device=dev)
+    col = val = None
+    if gather_values:
+        assert nnz_global is not None, "gather_values needs nnz_global (allocate once, e.g. from a prior gather)"
+        col = torch.empty(nnz_global, dtype=torch.int32, device=dev)
+        val = torch.empty(nnz_global, dtype=plan.dtype, device=dev)
+    tot = ctypes.c_int64(0)
+    _check(lib().sg_gather(plan.handle, ctypes.c_void_p(comm_ptr), int(gather_values), _ptr(plan.row_ptr),
+                           _ptr(local_col), _ptr(local_val), _ptr(rp), _ptr(col), _ptr(val), ctypes.byref(tot),
+                           _stream()), "sg_gather")
+    return rp, col, val, int(tot.value)
+
+
+def spgemm(A: DeviceCSR, B: DeviceCSR, sample_frac: float = 0.01, seed: int = 1, cm: CostModel | None = None,
+           thr: int | None = None):
+    """The one-call API: sampled threshold (unless thr is given), symbolic, numeric.
+    Returns (C as DeviceCSR, info dict)."""
+    rep = None
+    if thr is None:
+        thr, rep = sg_sample_threshold(A, B, sample_frac, seed, cm)
+    plan = sg_symbolic(A, B, thr)
+    col, val = sg_numeric(plan, A, B)
+    C = DeviceCSR(A.nrows, B.ncols, plan.row_ptr, col, val)
+    info = {"thr": thr, "sample": rep, "nnz": plan.nnz}
+    plan.destroy()
+    return C, info

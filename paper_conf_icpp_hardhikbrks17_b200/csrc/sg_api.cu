@@ -1,0 +1,564 @@
+// sg_api.cu — the C ABI (include/sg.h): validation, plans/workspace, orchestration of the kernels.
+#include "sg_internal.cuh"
+#include <cstdlib>
+#include <cstring>
+#include <cmath>
+#include <vector>
+#include <mutex>
+
+using namespace sg;
+
+struct sg_plan {
+    cudaStream_t s = nullptr;
+    bool poisoned = false;
+    int64_t rb = 0, re = 0, nr = 0, thr = 0, p = 0, m = 0;
+    int dt = 0;
+    int64_t* w = nullptr;
+    int8_t* cls = nullptr;
+    int32_t* lists = nullptr;
+    int64_t* u = nullptr;
+    int64_t* dbin = nullptr;  // [0..NBINS) counts, [NBINS] nlong, [NBINS+1 .. 2NBINS+1) cursors
+    int64_t bin_cnt[NBINS] = {0};
+    int64_t bin_off[NBINS + 1] = {0};
+    int64_t nheavy = 0;
+    int64_t* range_bounds = nullptr;
+    int64_t* range_off = nullptr;
+    RangeRec* ranges = nullptr;
+    int64_t nslots = 0;
+    int32_t* long_id = nullptr;
+    uint32_t* tp = nullptr;
+    int64_t nlong = 0;
+    int T = 0;
+    unsigned long long* counter = nullptr;
+    const int64_t* C_rp = nullptr;
+    int64_t nnz_c = 0;
+    std::vector<void*> allocs;
+};
+
+namespace {
+
+std::once_flag g_pool_once;
+
+void init_pool() {
+    std::call_once(g_pool_once, [] {
+        int dev = 0;
+        if (cudaGetDevice(&dev) != cudaSuccess) return;
+        cudaMemPool_t pool;
+        if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+            uint64_t thr = UINT64_MAX;
+            cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+        }
+    });
+}
+
+// stream-ordered scratch owned by a scope (non-plan calls)
+struct Scratch {
+    cudaStream_t s;
+    std::vector<void*> ptrs;
+    explicit Scratch(cudaStream_t st) : s(st) {}
+    void* get(size_t bytes) {
+        void* p = nullptr;
+        if (bytes == 0) bytes = 16;
+        if (cudaMallocAsync(&p, bytes, s) != cudaSuccess) return nullptr;
+        ptrs.push_back(p);
+        return p;
+    }
+    ~Scratch() { for (void* p : ptrs) cudaFreeAsync(p, s); }
+};
+
+void* palloc(sg_plan* pl, size_t bytes) {
+    void* p = nullptr;
+    if (bytes == 0) bytes = 16;
+    if (cudaMallocAsync(&p, bytes, pl->s) != cudaSuccess) return nullptr;
+    pl->allocs.push_back(p);
+    return p;
+}
+
+#define CK(x) do { cudaError_t _e = (x); if (_e != cudaSuccess) { cudaGetLastError(); return SG_ERR_CUDA; } } while (0)
+#define CKP(pl, x) do { cudaError_t _e = (x); if (_e != cudaSuccess) { cudaGetLastError(); (pl)->poisoned = true; return SG_ERR_CUDA; } } while (0)
+
+Mat mat_of(const sg_csr_view* v) {
+    Mat m;
+    m.nrows = v->nrows; m.ncols = v->ncols; m.nnz = v->nnz;
+    m.rp = v->row_ptr; m.col = v->col_idx; m.val = v->val; m.dt = (int)v->dtype;
+    return m;
+}
+
+bool env_validate() {
+    const char* e = getenv("SG_VALIDATE");
+    return e && e[0] == '1';
+}
+
+__global__ void k_validate(Mat M, int* bad) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M.nrows; i += (int64_t)gridDim.x * blockDim.x) {
+        int64_t s = M.rp[i], e = M.rp[i + 1];
+        if (e < s) { atomicOr(bad, 1); continue; }
+        for (int64_t q = s; q < e; ++q) {
+            int c = M.col[q];
+            if (c < 0 || c >= M.ncols || (q > s && M.col[q - 1] >= c)) { atomicOr(bad, 1); break; }
+        }
+    }
+}
+
+sg_status validate_one(const sg_csr_view* v, cudaStream_t s) {
+    if (!v) return SG_ERR_INVALID_ARG;
+    if (v->nrows < 0 || v->ncols < 0 || v->nnz < 0) return SG_ERR_INVALID_ARG;
+    if (v->ncols > INT32_MAX || v->nrows > INT32_MAX) return SG_ERR_OVERFLOW;
+    if (v->dtype != SG_F64 && v->dtype != SG_F32) return SG_ERR_DTYPE;
+    if (!v->row_ptr) return SG_ERR_INVALID_ARG;
+    if (v->nnz > 0 && (!v->col_idx || !v->val)) return SG_ERR_INVALID_ARG;
+    if (env_validate()) {
+        Scratch sc(s);
+        int* bad = (int*)sc.get(sizeof(int));
+        if (!bad) return SG_ERR_OOM;
+        CK(cudaMemsetAsync(bad, 0, sizeof(int), s));
+        Mat m = mat_of(v);
+        if (m.nrows > 0) k_validate<<<(unsigned)((m.nrows + 255) / 256 < 4096 ? (m.nrows + 255) / 256 : 4096), 256, 0, s>>>(m, bad);
+        CK(cudaGetLastError());
+        int h = 0;
+        CK(cudaMemcpyAsync(&h, bad, sizeof(int), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (h) return SG_ERR_NOT_CANONICAL;
+    }
+    return SG_OK;
+}
+
+sg_status validate_pair(const sg_csr_view* A, const sg_csr_view* B, cudaStream_t s) {
+    sg_status st;
+    if ((st = validate_one(A, s)) != SG_OK) return st;
+    if ((st = validate_one(B, s)) != SG_OK) return st;
+    if (A->ncols != B->nrows) return SG_ERR_SHAPE;
+    if (A->dtype != B->dtype) return SG_ERR_DTYPE;
+    return SG_OK;
+}
+
+CostModelD cm_of(const sg_cost_model* c) {
+    CostModelD d;
+    d.kL = c->kappa_L; d.lL = c->lambda_L; d.sL = c->sigma_L; d.rL = c->rho_L;
+    d.kH = c->kappa_H; d.lH = c->lambda_H; d.tH = c->tau_H; d.mH = c->mu_H;
+    d.tiles_fixed = c->tiles_fixed; d.capu = c->capu; d.cap_L = c->cap_L;
+    return d;
+}
+
+// Default model: calibrated from the measured kernels (profiles/).
+const sg_cost_model kDefaultModel = {
+    /*kappa_L*/ 3000, /*lambda_L*/ 120, /*sigma_L*/ 0, /*rho_L*/ 150,
+    /*kappa_H*/ 250000, /*lambda_H*/ 60, /*tau_H*/ 400, /*mu_H*/ 120,
+    /*tiles_fixed*/ 1, /*capu*/ CAPU, /*cap_L*/ SG_CAP_L_MAX};
+
+// Identify over a row list (rows == nullptr: rows [0, nr)). Computes w, a, u of those rows on the
+// device (exact sample-symbolic at routing threshold cap_L), then the cost histogram.
+struct RowStats {
+    int64_t* w = nullptr;
+    int64_t* a = nullptr;
+    int64_t* u = nullptr;
+};
+
+sg_status row_stats(const Mat& A, const Mat& B, const int64_t* rows, int64_t nr, int64_t cap, Scratch& sc,
+                    RowStats& rs, cudaStream_t s) {
+    rs.w = (int64_t*)sc.get(sizeof(int64_t) * (size_t)nr);
+    rs.a = (int64_t*)sc.get(sizeof(int64_t) * (size_t)nr);
+    rs.u = (int64_t*)sc.get(sizeof(int64_t) * (size_t)nr);
+    int32_t* lists = (int32_t*)sc.get(sizeof(int32_t) * (size_t)nr);
+    int64_t* dbin = (int64_t*)sc.get(sizeof(int64_t) * 2 * NBINS);
+    int64_t* all_rows = nullptr;
+    if (!rs.w || !rs.a || !rs.u || !lists || !dbin) return SG_ERR_OOM;
+    if (!rows) {
+        all_rows = (int64_t*)sc.get(sizeof(int64_t) * (size_t)nr);
+        if (!all_rows) return SG_ERR_OOM;
+        // rows [0, nr): use the identity row map through sample-select with f = 1
+        size_t tb = sample_tmp_bytes(nr);
+        void* tmp = sc.get(tb);
+        int64_t* dcount = (int64_t*)sc.get(sizeof(int64_t));
+        if (!tmp || !dcount) return SG_ERR_OOM;
+        CK(launch_sample_select(0, nr, 0, 0, true, all_rows, dcount, tmp, tb, s));
+        rows = all_rows;
+    }
+    CK(launch_row_work_list(A, B, rows, nr, rs.w, rs.a, s));
+    CK(cudaMemsetAsync(rs.u, 0, sizeof(int64_t) * (size_t)nr, s));
+    CK(cudaMemsetAsync(dbin, 0, sizeof(int64_t) * 2 * NBINS, s));
+    CK(launch_bin_count(rs.w, nr, cap, dbin, nullptr, s));
+    int64_t cnt[NBINS];
+    CK(cudaMemcpyAsync(cnt, dbin, sizeof(cnt), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    int64_t off[NBINS + 1];
+    off[0] = 0;
+    for (int b = 0; b < NBINS; ++b) off[b + 1] = off[b] + cnt[b];
+    CK(cudaMemcpyAsync(dbin + NBINS, off, sizeof(int64_t) * NBINS, cudaMemcpyHostToDevice, s));
+    CK(launch_bin_scatter(rs.w, nr, cap, dbin + NBINS, lists, s));
+    for (int b = 0; b < NBIN_LIGHT; ++b)
+        CK(launch_sym_light(b, A, B, lists + off[b], cnt[b], rows, 0, rs.u, s));
+    CK(launch_sym_heavy(A, B, lists + off[BIN_HEAVY], cnt[BIN_HEAVY], rows, 0, rs.w, rs.u, nullptr, nullptr, s));
+    return SG_OK;
+}
+
+sg_status identify(const Mat& A, const Mat& B, const int64_t* rows, int64_t nr, const sg_cost_model* c,
+                   ThrResult* res, cudaStream_t s) {
+    Scratch sc(s);
+    RowStats rs;
+    sg_status st = row_stats(A, B, rows, nr, c->cap_L, sc, rs, s);
+    if (st != SG_OK) return st;
+    CostModelD cm = cm_of(c);
+    size_t hb = sizeof(long long) * (size_t)(c->cap_L + 1);
+    long long* hd = (long long*)sc.get(hb);
+    long long* hc = (long long*)sc.get(hb);
+    long long* hw = (long long*)sc.get(hb);
+    long long* sums = (long long*)sc.get(4 * sizeof(long long));
+    ThrResult* dres = (ThrResult*)sc.get(sizeof(ThrResult));
+    if (!hd || !hc || !hw || !sums || !dres) return SG_ERR_OOM;
+    CK(launch_cost_hist(cm, rs.w, rs.a, rs.u, nr, hd, hc, hw, sums, s));
+    CK(launch_argmin(cm, hd, hc, hw, sums, dres, s));
+    CK(cudaMemcpyAsync(res, dres, sizeof(ThrResult), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    return SG_OK;
+}
+
+sg_status check_model(const sg_cost_model* c) {
+    if (c->cap_L < 0 || c->cap_L > SG_CAP_L_MAX) return SG_ERR_INVALID_ARG;
+    if (c->capu < 0 || c->tiles_fixed < 0) return SG_ERR_INVALID_ARG;
+    return SG_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* sg_status_string(sg_status st) {
+    switch (st) {
+        case SG_OK: return "SG_OK";
+        case SG_ERR_INVALID_ARG: return "SG_ERR_INVALID_ARG";
+        case SG_ERR_SHAPE: return "SG_ERR_SHAPE";
+        case SG_ERR_DTYPE: return "SG_ERR_DTYPE";
+        case SG_ERR_NOT_CANONICAL: return "SG_ERR_NOT_CANONICAL";
+        case SG_ERR_EMPTY_SAMPLE: return "SG_ERR_EMPTY_SAMPLE";
+        case SG_ERR_OOM: return "SG_ERR_OOM";
+        case SG_ERR_CUDA: return "SG_ERR_CUDA";
+        case SG_ERR_NCCL: return "SG_ERR_NCCL";
+        case SG_ERR_OVERFLOW: return "SG_ERR_OVERFLOW";
+    }
+    return "SG_ERR_UNKNOWN";
+}
+
+const char* sg_version(void) { return "sg 0.1.0 sm_100a"; }
+
+void sg_default_cost_model(sg_cost_model* out) {
+    if (out) *out = kDefaultModel;
+}
+
+sg_status sg_row_work(const sg_csr_view* A, const sg_csr_view* B, int64_t row_begin, int64_t row_end, int64_t* w_out,
+                      int64_t* total_out, void* stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    init_pool();
+    sg_status st = validate_pair(A, B, s);
+    if (st != SG_OK) return st;
+    if (row_begin < 0 || row_end < row_begin || row_end > A->nrows) return SG_ERR_INVALID_ARG;
+    if (!w_out && row_end > row_begin) return SG_ERR_INVALID_ARG;
+    Mat a = mat_of(A), b = mat_of(B);
+    CK(launch_row_work(a, b, row_begin, row_end, w_out, s));
+    if (total_out) {
+        Scratch sc(s);
+        int64_t n = row_end - row_begin;
+        int64_t* P = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(n + 1));
+        void* tmp = sc.get(scan_tmp_bytes(n));
+        if (!P || !tmp) return SG_ERR_OOM;
+        CK(scan_exclusive(w_out, P, n, tmp, s));
+        CK(cudaMemcpyAsync(total_out, P + n, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+    }
+    return SG_OK;
+}
+
+sg_status sg_sample_rows(int64_t row_begin, int64_t row_end, double f, uint64_t seed, int64_t* rows_out,
+                         int64_t rows_cap, int64_t* count_out, void* stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    init_pool();
+    if (!(f > 0.0 && f <= 1.0) || row_begin < 0 || row_end < row_begin || !count_out) return SG_ERR_INVALID_ARG;
+    int64_t n = row_end - row_begin;
+    Scratch sc(s);
+    int64_t* rows = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(n > 0 ? n : 1));
+    int64_t* dcount = (int64_t*)sc.get(sizeof(int64_t));
+    size_t tb = sample_tmp_bytes(n);
+    void* tmp = sc.get(tb);
+    if (!rows || !dcount || !tmp) return SG_ERR_OOM;
+    bool all = f >= 1.0;
+    uint64_t Tf = all ? 0 : (uint64_t)std::ldexp(f, 64);
+    CK(launch_sample_select(row_begin, row_end, seed, Tf, all, rows, dcount, tmp, tb, s));
+    int64_t c = 0;
+    CK(cudaMemcpyAsync(&c, dcount, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    *count_out = c;
+    if (rows_out && c > 0) {
+        if (rows_cap < c) return SG_ERR_SHAPE;
+        CK(cudaMemcpyAsync(rows_out, rows, sizeof(int64_t) * (size_t)c, cudaMemcpyDeviceToDevice, s));
+        CK(cudaStreamSynchronize(s));
+    }
+    return SG_OK;
+}
+
+sg_status sg_sample_threshold(const sg_csr_view* A, const sg_csr_view* B, double sample_frac, uint64_t seed,
+                              const sg_cost_model* cm, int64_t* thr_out, sg_sample_report* rep, void* stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    init_pool();
+    if (!thr_out) return SG_ERR_INVALID_ARG;
+    if (!(sample_frac > 0.0 && sample_frac <= 1.0)) return SG_ERR_INVALID_ARG;
+    sg_status st = validate_pair(A, B, s);
+    if (st != SG_OK) return st;
+    const sg_cost_model* c = cm ? cm : &kDefaultModel;
+    if ((st = check_model(c)) != SG_OK) return st;
+    Mat a = mat_of(A), b = mat_of(B);
+    const int64_t n = A->nrows;
+    // Sample: S = { i : h(seed, SAMPLE, i) < floor(f 2^64) }  (R4)
+    Scratch sc(s);
+    int64_t* S = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(n > 0 ? n : 1));
+    int64_t* dcount = (int64_t*)sc.get(sizeof(int64_t));
+    size_t tb = sample_tmp_bytes(n);
+    void* tmp = sc.get(tb);
+    if (!S || !dcount || !tmp) return SG_ERR_OOM;
+    bool all = sample_frac >= 1.0;
+    uint64_t Tf = all ? 0 : (uint64_t)std::ldexp(sample_frac, 64);
+    CK(launch_sample_select(0, n, seed, Tf, all, S, dcount, tmp, tb, s));
+    int64_t ns = 0;
+    CK(cudaMemcpyAsync(&ns, dcount, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if (ns == 0) return SG_ERR_EMPTY_SAMPLE;
+    // Identify on S (exact per-row w, a, u; integer J histogram; smallest argmin)
+    ThrResult r;
+    st = identify(a, b, S, ns, c, &r, s);
+    if (st != SG_OK) return st;
+    if (r.nonempty == 0) return SG_ERR_EMPTY_SAMPLE;
+    // Extrapolate: identity (r = r')
+    *thr_out = r.thr;
+    if (rep) {
+        rep->sample_rows = ns;
+        rep->sample_nonempty = r.nonempty;
+        rep->thr = r.thr;
+        rep->W_est_L = r.W_L;
+        rep->W_est_H = r.W_all - r.W_L;
+        rep->J_min = r.Jmin;
+    }
+    return SG_OK;
+}
+
+sg_status sg_exhaustive_threshold(const sg_csr_view* A, const sg_csr_view* B, const sg_cost_model* cm,
+                                  int64_t* thr_out, int64_t* J_min_out, void* stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    init_pool();
+    if (!thr_out) return SG_ERR_INVALID_ARG;
+    sg_status st = validate_pair(A, B, s);
+    if (st != SG_OK) return st;
+    const sg_cost_model* c = cm ? cm : &kDefaultModel;
+    if ((st = check_model(c)) != SG_OK) return st;
+    ThrResult r;
+    st = identify(mat_of(A), mat_of(B), nullptr, A->nrows, c, &r, s);
+    if (st != SG_OK) return st;
+    *thr_out = r.thr;
+    if (J_min_out) *J_min_out = r.Jmin;
+    return SG_OK;
+}
+
+sg_status sg_cost_curve(const sg_csr_view* A, const sg_csr_view* B, const sg_cost_model* cm, int64_t nt,
+                        const int64_t* t_host, int64_t* J_host, void* stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    init_pool();
+    if (nt < 0 || (nt > 0 && (!t_host || !J_host))) return SG_ERR_INVALID_ARG;
+    sg_status st = validate_pair(A, B, s);
+    if (st != SG_OK) return st;
+    const sg_cost_model* c = cm ? cm : &kDefaultModel;
+    if ((st = check_model(c)) != SG_OK) return st;
+    Scratch sc(s);
+    RowStats rs;
+    Mat a = mat_of(A), b = mat_of(B);
+    st = row_stats(a, b, nullptr, A->nrows, c->cap_L, sc, rs, s);
+    if (st != SG_OK) return st;
+    int64_t* dt = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(nt > 0 ? nt : 1));
+    long long* dJ = (long long*)sc.get(sizeof(long long) * (size_t)(nt > 0 ? nt : 1));
+    if (!dt || !dJ) return SG_ERR_OOM;
+    if (nt > 0) {
+        CK(cudaMemcpyAsync(dt, t_host, sizeof(int64_t) * (size_t)nt, cudaMemcpyHostToDevice, s));
+        CK(launch_cost_curve(cm_of(c), rs.w, rs.a, rs.u, A->nrows, dt, (int)nt, dJ, s));
+        CK(cudaMemcpyAsync(J_host, dJ, sizeof(long long) * (size_t)nt, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+    }
+    return SG_OK;
+}
+
+sg_status sg_partition(const sg_csr_view* A, const sg_csr_view* B, int nparts, int64_t* cuts_out, int64_t* flops_out,
+                       void* stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    init_pool();
+    if (nparts < 1 || !cuts_out) return SG_ERR_INVALID_ARG;
+    sg_status st = validate_pair(A, B, s);
+    if (st != SG_OK) return st;
+    const int64_t n = A->nrows;
+    Scratch sc(s);
+    int64_t* w = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(n > 0 ? n : 1));
+    int64_t* P = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(n + 1));
+    void* tmp = sc.get(scan_tmp_bytes(n));
+    int64_t* dcuts = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(nparts + 1));
+    if (!w || !P || !tmp || !dcuts) return SG_ERR_OOM;
+    Mat a = mat_of(A), b = mat_of(B);
+    CK(launch_row_work(a, b, 0, n, w, s));
+    CK(scan_exclusive(w, P, n, tmp, s));
+    CK(launch_cuts(P, n, nparts, dcuts, s));
+    CK(cudaMemcpyAsync(cuts_out, dcuts, sizeof(int64_t) * (size_t)(nparts + 1), cudaMemcpyDeviceToHost, s));
+    int64_t W = 0;
+    CK(cudaMemcpyAsync(&W, P + n, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if (flops_out) *flops_out = W;
+    return SG_OK;
+}
+
+sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, int64_t row_begin, int64_t row_end,
+                      int64_t* C_row_ptr, int64_t* nnz_c_out, sg_plan** plan_out, void* stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    init_pool();
+    if (!C_row_ptr || !nnz_c_out || !plan_out) return SG_ERR_INVALID_ARG;
+    if (thr < 0 || thr > SG_CAP_L_MAX) return SG_ERR_INVALID_ARG;
+    sg_status st = validate_pair(A, B, s);
+    if (st != SG_OK) return st;
+    if (row_begin < 0 || row_end < row_begin || row_end > A->nrows) return SG_ERR_INVALID_ARG;
+    sg_plan* pl = new sg_plan();
+    pl->s = s;
+    pl->rb = row_begin; pl->re = row_end; pl->nr = row_end - row_begin; pl->thr = thr;
+    pl->p = B->ncols; pl->m = B->nrows; pl->dt = (int)A->dtype;
+    pl->C_rp = C_row_ptr;
+    const int64_t nr = pl->nr;
+    Mat a = mat_of(A), b = mat_of(B);
+    auto fail = [&](sg_status e) { pl->poisoned = true; sg_plan_destroy(pl); return e; };
+    size_t nrb = (size_t)(nr > 0 ? nr : 1);
+    pl->w = (int64_t*)palloc(pl, 8 * nrb);
+    pl->cls = (int8_t*)palloc(pl, nrb);
+    pl->lists = (int32_t*)palloc(pl, 4 * nrb);
+    pl->u = (int64_t*)palloc(pl, 8 * nrb);
+    pl->dbin = (int64_t*)palloc(pl, sizeof(int64_t) * (2 * NBINS + 2));
+    pl->long_id = (int32_t*)palloc(pl, 4 * (size_t)(pl->m > 0 ? pl->m : 1));
+    pl->counter = (unsigned long long*)palloc(pl, sizeof(unsigned long long));
+    void* stmp = palloc(pl, scan_tmp_bytes(nr + 1));
+    if (!pl->w || !pl->cls || !pl->lists || !pl->u || !pl->dbin || !pl->long_id || !pl->counter || !stmp)
+        return fail(SG_ERR_OOM);
+    pl->T = (int)((pl->p + TW - 1) / TW);
+    if (pl->T < 1) pl->T = 1;
+#define CKF(x) do { if ((x) != cudaSuccess) { cudaGetLastError(); return fail(SG_ERR_CUDA); } } while (0)
+    // a1 row work, a5 classes + bin counts, long rows of B
+    CKF(launch_row_work(a, b, row_begin, row_end, pl->w, s));
+    CKF(cudaMemsetAsync(pl->dbin, 0, sizeof(int64_t) * (2 * NBINS + 2), s));
+    CKF(cudaMemsetAsync(pl->u, 0, 8 * nrb, s));
+    CKF(launch_bin_count(pl->w, nr, thr, pl->dbin, pl->cls, s));
+    CKF(launch_long_rows(b, pl->long_id, pl->dbin + NBINS, s));
+    int64_t hc[NBINS + 1];
+    CKF(cudaMemcpyAsync(hc, pl->dbin, sizeof(hc), cudaMemcpyDeviceToHost, s));
+    CKF(cudaStreamSynchronize(s));
+    pl->bin_off[0] = 0;
+    for (int k = 0; k < NBINS; ++k) { pl->bin_cnt[k] = hc[k]; pl->bin_off[k + 1] = pl->bin_off[k] + hc[k]; }
+    pl->nlong = hc[NBINS];
+    CKF(cudaMemcpyAsync(pl->dbin + NBINS + 1, pl->bin_off, sizeof(int64_t) * NBINS, cudaMemcpyHostToDevice, s));
+    CKF(launch_bin_scatter(pl->w, nr, thr, pl->dbin + NBINS + 1, pl->lists, s));
+    // heavy: range-slot bounds -> offsets
+    pl->nheavy = pl->bin_cnt[BIN_HEAVY];
+    const int32_t* heavy = pl->lists + pl->bin_off[BIN_HEAVY];
+    if (pl->nheavy > 0) {
+        pl->range_bounds = (int64_t*)palloc(pl, 8 * (size_t)pl->nheavy);
+        pl->range_off = (int64_t*)palloc(pl, 8 * (size_t)(pl->nheavy + 1));
+        void* t2 = palloc(pl, scan_tmp_bytes(pl->nheavy));
+        if (!pl->range_bounds || !pl->range_off || !t2) return fail(SG_ERR_OOM);
+        CKF(launch_range_bounds(heavy, pl->nheavy, pl->w, pl->p, pl->range_bounds, s));
+        CKF(scan_exclusive(pl->range_bounds, pl->range_off, pl->nheavy, t2, s));
+        CKF(cudaMemcpyAsync(&pl->nslots, pl->range_off + pl->nheavy, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        CKF(cudaStreamSynchronize(s));
+        pl->ranges = (RangeRec*)palloc(pl, sizeof(RangeRec) * (size_t)pl->nslots);
+        if (!pl->ranges) return fail(SG_ERR_OOM);
+        CKF(launch_fill_ranges_unused(pl->ranges, pl->nslots, s));
+        // B tile pointers for long rows (numeric heavy path)
+        pl->tp = (uint32_t*)palloc(pl, 4 * (size_t)(pl->nlong > 0 ? pl->nlong : 1) * (size_t)(pl->T + 1));
+        if (!pl->tp) return fail(SG_ERR_OOM);
+        if (pl->nlong > 0) CKF(launch_build_tp(b, pl->long_id, pl->T, pl->tp, s));
+    }
+    // a6 symbolic
+    for (int k = 0; k < NBIN_LIGHT; ++k)
+        CKF(launch_sym_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], nullptr, row_begin, pl->u, s));
+    CKF(launch_sym_heavy(a, b, heavy, pl->nheavy, nullptr, row_begin, pl->w, pl->u, pl->range_off, pl->ranges, s));
+    CKF(scan_exclusive(pl->u, C_row_ptr, nr, stmp, s));
+    CKF(cudaMemcpyAsync(&pl->nnz_c, C_row_ptr + nr, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    CKF(cudaStreamSynchronize(s));
+#undef CKF
+    *nnz_c_out = pl->nnz_c;
+    *plan_out = pl;
+    return SG_OK;
+}
+
+sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, int32_t* C_col, void* C_val,
+                     void* stream) {
+    if (!pl) return SG_ERR_INVALID_ARG;
+    if (pl->poisoned) return SG_ERR_CUDA;
+    cudaStream_t s = (cudaStream_t)stream;
+    if (!A || !B) return SG_ERR_INVALID_ARG;
+    if (A->nrows < pl->re || B->ncols != pl->p || B->nrows != pl->m) return SG_ERR_SHAPE;
+    if ((int)A->dtype != pl->dt || (int)B->dtype != pl->dt) return SG_ERR_DTYPE;
+    if (pl->nnz_c > 0 && (!C_col || !C_val)) return SG_ERR_INVALID_ARG;
+    if (pl->nnz_c == 0) return SG_OK;
+    Mat a = mat_of(A), b = mat_of(B);
+    for (int k = 0; k < NBIN_LIGHT; ++k)
+        CKP(pl, launch_num_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], pl->rb, pl->C_rp, C_col, C_val, s));
+    if (pl->nheavy > 0)
+        CKP(pl, launch_num_heavy(a, b, pl->ranges, pl->nslots, pl->rb, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
+                                 C_val, pl->counter, s));
+    return SG_OK;
+}
+
+sg_status sg_plan_get_info(const sg_plan* pl, sg_plan_info* out) {
+    if (!pl || !out) return SG_ERR_INVALID_ARG;
+    if (pl->poisoned) return SG_ERR_CUDA;
+    memset(out, 0, sizeof(*out));
+    out->row_begin = pl->rb; out->row_end = pl->re; out->thr = pl->thr;
+    out->n_empty = pl->bin_cnt[BIN_EMPTY];
+    out->n_heavy = pl->bin_cnt[BIN_HEAVY];
+    for (int k = 0; k < NBIN_LIGHT; ++k) { out->light_bins[k] = pl->bin_cnt[k]; out->n_light += pl->bin_cnt[k]; }
+    out->nnz_c = pl->nnz_c;
+    out->n_ranges = pl->nslots;
+    // flops on demand
+    if (pl->nr > 0) {
+        cudaStream_t s = pl->s;
+        Scratch sc(s);
+        int64_t* P = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(pl->nr + 1));
+        void* tmp = sc.get(scan_tmp_bytes(pl->nr));
+        if (!P || !tmp) return SG_ERR_OOM;
+        CK(scan_exclusive(pl->w, P, pl->nr, tmp, s));
+        CK(cudaMemcpyAsync(&out->flops, P + pl->nr, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+    }
+    return SG_OK;
+}
+
+sg_status sg_plan_get_classes(const sg_plan* pl, int8_t* cls_out, void* stream) {
+    if (!pl || (!cls_out && pl->nr > 0)) return SG_ERR_INVALID_ARG;
+    if (pl->poisoned) return SG_ERR_CUDA;
+    if (pl->nr > 0)
+        CK(cudaMemcpyAsync(cls_out, pl->cls, (size_t)pl->nr, cudaMemcpyDeviceToDevice, (cudaStream_t)stream));
+    return SG_OK;
+}
+
+sg_status sg_plan_get_work(const sg_plan* pl, int64_t* w_out, void* stream) {
+    if (!pl || (!w_out && pl->nr > 0)) return SG_ERR_INVALID_ARG;
+    if (pl->poisoned) return SG_ERR_CUDA;
+    if (pl->nr > 0)
+        CK(cudaMemcpyAsync(w_out, pl->w, 8 * (size_t)pl->nr, cudaMemcpyDeviceToDevice, (cudaStream_t)stream));
+    return SG_OK;
+}
+
+void sg_plan_destroy(sg_plan* pl) {
+    if (!pl) return;
+    for (void* p : pl->allocs) cudaFreeAsync(p, pl->s);
+    pl->allocs.clear();
+    delete pl;
+}
+
+// internal accessors for sg_gather.cu
+int64_t sg_internal_plan_rows(const sg_plan* pl, int64_t* rb, int64_t* re) {
+    *rb = pl->rb; *re = pl->re;
+    return pl->nnz_c;
+}
+int sg_internal_plan_dtype(const sg_plan* pl) { return pl->dt; }
+bool sg_internal_plan_poisoned(const sg_plan* pl) { return pl->poisoned; }
+void sg_internal_plan_poison(sg_plan* pl) { pl->poisoned = true; }
+
+}  // extern "C"

@@ -1,0 +1,96 @@
+// sg_internal.cuh — internal declarations shared by the libsg translation units (CUDA side only;
+// nothing here is shared with oracle/). Layout and kernel design: DESIGN.md §6-§7.
+#pragma once
+#include <cuda_runtime.h>
+#include <cstdint>
+#include <cstddef>
+#include "sg.h"
+
+namespace sg {
+
+// ---- routing classes and bins (heavy iff w > t; R13: w == t light) --
+constexpr int NBIN_LIGHT = 13;   // light bin b holds 2^(b-1) < w <= 2^b  (b = 0: w == 1); U_b = 2^b
+constexpr int BIN_EMPTY = 13;    // w == 0 (R7)
+constexpr int BIN_HEAVY = 14;    // w > thr
+constexpr int NBINS = 15;
+
+// ---- heavy path geometry ---------------------------------------------------
+constexpr int TW = 8192;          // column tile width of the heavy path (tile = unit of range planning)
+constexpr int CAPU = 4096;        // max entries of a hashed (multi-tile) heavy range
+constexpr int PH = 12288;         // heavy accumulator slots per CTA (int32 key + fp64 value)
+constexpr int HH = PH - CAPU;     // home range of the order-preserving hash (overflow room = CAPU)
+constexpr int LONG_ROW = 32;      // B rows longer than this get per-tile pointers
+constexpr int WIN = 1 << 20;      // heavy symbolic bitmap window (columns); 128 KB of smem
+constexpr int HEAVY_THREADS = 1024;
+
+constexpr int32_t EMPTY_KEY = -1;
+constexpr uint64_t TAG_SAMPLE = 0x53414d504c450001ULL;  // DESIGN.md R4 (stream tag of the row sampler)
+
+struct RangeRec {  // one heavy numeric work item: row x tiles [t0, t1)
+    int32_t row;   // local row index (row - row_begin); -1 = unused slot
+    int32_t t0, t1;
+    int32_t cnt;   // exact number of C entries in the range
+    int32_t off;   // offset of the range's first entry within the row
+    int32_t pad;
+};
+
+struct Mat {  // device CSR view
+    int64_t nrows, ncols, nnz;
+    const int64_t* rp;
+    const int32_t* col;
+    const void* val;
+    int dt;  // 0 f64, 1 f32
+};
+
+struct CostModelD {
+    int64_t kL, lL, sL, rL, kH, lH, tH, mH, tiles_fixed, capu, cap_L;
+};
+
+// ---- launchers (sg_kernels.cu) ------------------------------------------------------------------
+cudaError_t launch_row_work(const Mat& A, const Mat& B, int64_t rb, int64_t re, int64_t* w, cudaStream_t s);
+cudaError_t launch_row_work_list(const Mat& A, const Mat& B, const int64_t* rows, int64_t nr, int64_t* w_rows,
+                                 int64_t* a_rows, cudaStream_t s);
+// exclusive scan in[0..n) -> out[0..n] (out[0] = 0, out[n] = total); tmp: scan_tmp_bytes(n) bytes
+size_t scan_tmp_bytes(int64_t n);
+cudaError_t scan_exclusive(const int64_t* in, int64_t* out, int64_t n, void* tmp, cudaStream_t s);
+// stable selection of sampled rows: count then write
+cudaError_t launch_sample_select(int64_t rb, int64_t re, uint64_t seed, uint64_t Tf, bool all,
+                                 int64_t* out_rows, int64_t* d_count, void* tmp, size_t tmp_bytes, cudaStream_t s);
+size_t sample_tmp_bytes(int64_t n);
+// binning: w of nr rows (rows = list or rb + j); bins by thr; cls optional
+cudaError_t launch_bin_count(const int64_t* w, int64_t nr, int64_t thr, int64_t* d_cnt /*NBINS*/, int8_t* cls,
+                             cudaStream_t s);
+cudaError_t launch_bin_scatter(const int64_t* w, int64_t nr, int64_t thr, int64_t* d_cursor /*NBINS*/,
+                               int32_t* lists, cudaStream_t s);
+// symbolic light: bin b, rows = lists entries (local index j); global row = rowmap ? rowmap[j] : rb + j
+cudaError_t launch_sym_light(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt,
+                             const int64_t* rowmap, int64_t rb, int64_t* u, cudaStream_t s);
+cudaError_t launch_sym_heavy(const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, const int64_t* rowmap,
+                             int64_t rb, const int64_t* w, int64_t* u, const int64_t* range_off, RangeRec* ranges,
+                             cudaStream_t s);
+cudaError_t launch_range_bounds(const int32_t* heavy_list, int64_t nheavy, const int64_t* w, int64_t p,
+                                int64_t* bounds, cudaStream_t s);
+cudaError_t launch_fill_ranges_unused(RangeRec* ranges, int64_t n, cudaStream_t s);
+// B tile pointers for long rows
+cudaError_t launch_long_rows(const Mat& B, int32_t* long_id, int64_t* d_nlong, cudaStream_t s);
+cudaError_t launch_build_tp(const Mat& B, const int32_t* long_id, int T, uint32_t* tp, cudaStream_t s);
+// numeric
+cudaError_t launch_num_light(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, int64_t rb,
+                             const int64_t* C_rp, int32_t* C_col, void* C_val, cudaStream_t s);
+cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const RangeRec* ranges, int64_t nslots, int64_t rb,
+                             const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp,
+                             int32_t* C_col, void* C_val, unsigned long long* d_counter, cudaStream_t s);
+// threshold: cost histogram over rows then argmin over t in [0, cap_L]
+struct ThrResult { long long thr, Jmin, base, W_L, W_all, nonempty; };
+cudaError_t launch_cost_hist(const CostModelD& cm, const int64_t* w, const int64_t* a, const int64_t* u, int64_t nr,
+                             long long* hist_d /*cap_L+1*/, long long* hist_c /*cap_L+1*/, long long* hist_w,
+                             long long* sums /*4*/, cudaStream_t s);
+cudaError_t launch_argmin(const CostModelD& cm, const long long* hist_d, const long long* hist_c,
+                          const long long* hist_w, const long long* sums, ThrResult* out, cudaStream_t s);
+cudaError_t launch_cost_curve(const CostModelD& cm, const int64_t* w, const int64_t* a, const int64_t* u, int64_t nr,
+                              const int64_t* t, int nt, long long* J, cudaStream_t s);
+cudaError_t launch_cuts(const int64_t* P, int64_t n, int G, int64_t* cuts, cudaStream_t s);
+cudaError_t launch_gather_rows(const int64_t* src, const int64_t* rows, int64_t nr, int64_t* dst, cudaStream_t s);
+cudaError_t launch_add_offset(int64_t* x, int64_t n, int64_t off, cudaStream_t s);
+
+}  // namespace sg

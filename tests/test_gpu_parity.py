@@ -1,0 +1,287 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the same seeded inputs.
+
+Structure (C.row_ptr, C.col) and every integer quantity (w, classes, sample set, thresholds, cuts)
+must be bit-exact; values within rtol * sum_k |a_ik b_kj| (1e-12 fp64, 1e-5 fp32; north_star), and
+bit-exact in integer-value mode (R11).
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import sginputs as gen
+from _util import compare_rows
+
+pytestmark = pytest.mark.gpu
+
+sg = pytest.importorskip("paper_conf_icpp_hardhikbrks17_b200")
+
+
+def _dev(H):
+    return sg.DeviceCSR.from_host(H)
+
+
+def _model_from(cm_sg):
+    o = oracle.CostModel()
+    for k, v in cm_sg.as_dict().items():
+        setattr(o, k, v)
+    return o
+
+
+def _full_product(A, B, thr):
+    dA, dB = _dev(A), (_dev(B) if B is not A else None)
+    dB = dB or dA
+    plan = sg.sg_symbolic(dA, dB, thr)
+    col, val = sg.sg_numeric(plan, dA, dB)
+    torch.cuda.synchronize()
+    info = plan.info()
+    cls = plan.classes().cpu().numpy()
+    out = plan.row_ptr.cpu().numpy(), col.cpu().numpy(), val.cpu().numpy()
+    plan.destroy()
+    return out, info, cls
+
+
+# ---- a1 row work ----------------------------------------------------------------------------
+
+@pytest.mark.parametrize("name", ["C1", "C2", "rmat12", "rmat16"])
+def test_row_work_bit_exact(name):
+    A = gen.config(name)
+    w, W = sg.sg_row_work(_dev(A), _dev(A), with_total=True)
+    wo = oracle.row_work(A, A)
+    assert np.array_equal(w.cpu().numpy(), wo)
+    assert W == int(wo.sum())
+
+
+def test_row_work_subrange_and_empty():
+    A = gen.config("rmat12")
+    dA = _dev(A)
+    w = sg.sg_row_work(dA, dA, 100, 2000).cpu().numpy()
+    assert np.array_equal(w, oracle.row_work(A, A)[100:2000])
+    assert sg.sg_row_work(dA, dA, 5, 5).numel() == 0
+
+
+# ---- a3 sampler ---------------------------------------------------------------------------------
+
+@pytest.mark.parametrize("n,f,seed", [(1000, 0.05, 1), (262_144, 0.01, 7), (1 << 20, 0.1, 3), (777, 1.0, 2)])
+def test_sample_rows_bit_exact(n, f, seed):
+    S = sg.sg_sample_rows(n, f, seed).cpu().numpy()
+    assert np.array_equal(S, oracle.sample_rows(n, seed, f))
+
+
+@pytest.mark.parametrize("name,f,seed", [("C1", 0.2, 1), ("C2", 0.01, 3), ("rmat12", 0.05, 5),
+                                         ("rmat14", 0.02, 11), ("rmat14", 1.0, 0)])
+def test_sampled_threshold_bit_exact(name, f, seed):
+    A = gen.config(name)
+    dA = _dev(A)
+    cm = sg.sg_default_cost_model()
+    thr, rep = sg.sg_sample_threshold(dA, dA, f, seed, cm)
+    o = oracle.sampled_threshold(A, A, f, seed, _model_from(cm))
+    assert thr == o.thr
+    assert rep["sample_rows"] == len(o.rows)
+    assert rep["sample_nonempty"] == o.nonempty
+    assert rep["J_min"] == o.Jmin
+    assert rep["W_est_L"] == o.W_est_L and rep["W_est_H"] == o.W_est_H
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_sampled_threshold_random_models(seed):
+    rng = np.random.default_rng(seed)
+    A = gen.config("rmat12")
+    dA = _dev(A)
+    cm = sg.CostModel(kappa_L=int(rng.integers(0, 5000)), lambda_L=int(rng.integers(1, 200)),
+                      sigma_L=int(rng.integers(0, 5)), rho_L=int(rng.integers(0, 300)),
+                      kappa_H=int(rng.integers(0, 10**6)), lambda_H=int(rng.integers(1, 200)),
+                      tau_H=int(rng.integers(0, 1000)), mu_H=int(rng.integers(0, 300)),
+                      tiles_fixed=int(rng.integers(1, 5)), capu=int(rng.choice([0, 1024, 4096])),
+                      cap_L=int(rng.integers(16, 4097)))
+    thr, rep = sg.sg_sample_threshold(dA, dA, 0.1, seed, cm)
+    o = oracle.sampled_threshold(A, A, 0.1, seed, _model_from(cm))
+    assert thr == o.thr and rep["J_min"] == o.Jmin
+    ts, Js = sg.sg_exhaustive_threshold(dA, dA, cm)
+    to, Jo = oracle.exhaustive_threshold(A, A, _model_from(cm))
+    assert (ts, Js) == (to, Jo)
+
+
+def test_cost_curve_matches_plain_J():
+    A = gen.config("rmat11")
+    dA = _dev(A)
+    cm = sg.sg_default_cost_model()
+    ts = [0, 1, 7, 64, 500, 4096, 10**6]
+    J = sg.sg_cost_curve(dA, dA, ts, cm)
+    w = oracle.row_work(A, A)
+    u = oracle.counts(A, A)
+    a = np.diff(A.row_ptr)
+    assert J == [oracle.J(_model_from(cm), w, a, u, t) for t in ts]
+
+
+def test_empty_sample_is_an_error():
+    Z = gen.empty_rows(50, 50)
+    dZ = _dev(Z)
+    with pytest.raises(sg.SgError) as e:
+        sg.sg_sample_threshold(dZ, dZ, 0.5, 1)
+    assert "EMPTY_SAMPLE" in str(e.value)
+
+
+# ---- a4 partition -------------------------------------------------------------------------------
+
+@pytest.mark.parametrize("name", ["C2", "rmat14"])
+@pytest.mark.parametrize("G", [1, 2, 3, 8])
+def test_partition_bit_exact(name, G):
+    A = gen.config(name)
+    cuts, W = sg.sg_partition(_dev(A), _dev(A), G)
+    w = oracle.row_work(A, A)
+    assert cuts == list(oracle.partition(w, G))
+    assert W == int(w.sum())
+
+
+def test_partition_plateaus_and_ties():
+    # rows with zero work create plateaus in the prefix; ties go to the smaller boundary
+    A = gen.banded(64, [0], [1.0])
+    rp = A.row_ptr.copy()
+    keep = np.ones(64, bool)
+    keep[10:30] = False  # empty rows 10..29
+    cols, vals, nrp = [], [], [0]
+    for i in range(64):
+        if keep[i]:
+            cols.append(i); vals.append(1.0)
+        nrp.append(len(cols))
+    A = gen.CSR(64, 64, np.array(nrp, np.int64), np.array(cols, np.int32), np.array(vals), "plateau")
+    for G in (2, 3, 5, 7):
+        cuts, _ = sg.sg_partition(_dev(A), _dev(A), G)
+        assert cuts == list(oracle.partition(oracle.row_work(A, A), G))
+
+
+# ---- a5-a8 symbolic + numeric ---------------------------------------------------------------------
+
+@pytest.mark.parametrize("name", ["C1", "rmat10", "rmat12"])
+@pytest.mark.parametrize("thr", [0, 1, 64, 300, 4096])
+def test_full_product_bit_exact_structure(name, thr):
+    A = gen.config(name)
+    (rp, col, val), info, cls = _full_product(A, A, thr)
+    R = oracle.spgemm(A, A, with_absmag=True)
+    assert np.array_equal(rp, R.row_ptr)
+    compare_rows(rp, col, val, R, "f64")
+    w = oracle.row_work(A, A)
+    exp_cls = np.where(w == 0, 0, np.where(w > thr, 2, 1))
+    assert np.array_equal(cls, exp_cls)
+    assert info["n_heavy"] == int((exp_cls == 2).sum()) and info["flops"] == int(w.sum())
+
+
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+def test_integer_values_bit_exact(dtype):
+    A = gen.config("rmat12", mode="int", dtype=dtype)
+    for thr in (0, 128, 4096):
+        (rp, col, val), _, _ = _full_product(A, A, thr)
+        R = oracle.spgemm(A, A, with_absmag=True)
+        compare_rows(rp, col, val, R, dtype, exact_values=True)
+
+
+def test_fp32_tolerance():
+    A = gen.config("rmat12", dtype="f32")
+    (rp, col, val), _, _ = _full_product(A, A, 256)
+    assert val.dtype == np.float32
+    R = oracle.spgemm(A, A, with_absmag=True)
+    compare_rows(rp, col, val, R, "f32")
+
+
+def test_er_2pow18_full():
+    """Config 2 (ER 2^18, 16/row), every row, at the sampled threshold."""
+    A = gen.config("C2")
+    dA = _dev(A)
+    thr, _ = sg.sg_sample_threshold(dA, dA, 0.01, 1)
+    (rp, col, val), _, _ = _full_product(A, A, thr)
+    R = oracle.spgemm(A, A, with_absmag=True)
+    assert np.array_equal(rp, R.row_ptr)
+    compare_rows(rp, col, val, R, "f64")
+
+
+@pytest.mark.parametrize("thr", [0, 2048])
+def test_rmat16_heavy_ranges(thr):
+    """Several heavy rows span many column tiles / hashed ranges (p = 65536 -> 8 tiles)."""
+    A = gen.config("rmat16")
+    (rp, col, val), info, _ = _full_product(A, A, thr)
+    R = oracle.spgemm(A, A, with_absmag=True)
+    assert np.array_equal(rp, R.row_ptr)
+    compare_rows(rp, col, val, R, "f64")
+    assert info["n_ranges"] > 0
+
+
+def test_rmat18_sampled_rows():
+    """R-MAT 18 (config 5): structure bit-exact on every row (row_ptr), values on a seeded row
+    sample plus the 64 heaviest rows."""
+    A = gen.config("R18")
+    dA = _dev(A)
+    thr, _ = sg.sg_sample_threshold(dA, dA, 0.01, 1)
+    (rp, col, val), _, _ = _full_product(A, A, thr)
+    u = oracle.counts(A, A)
+    assert np.array_equal(np.diff(rp), u)
+    w = oracle.row_work(A, A)
+    rows = np.union1d(oracle.sample_rows(A.nrows, 99, 0.002), np.argsort(w)[-64:]).astype(np.int64)
+    R = oracle.spgemm(A, A, rows=rows, with_absmag=True)
+    compare_rows(rp, col, val, R, "f64")
+
+
+def test_special_matrices():
+    n = 3000
+    A = gen.config("C1")
+    I = gen.identity(A.nrows)
+    for X, Y in ((A, I), (I, A)):
+        (rp, col, val), _, _ = _full_product(X, Y, 64)
+        assert np.array_equal(rp, A.row_ptr) and np.array_equal(col, A.col) and np.array_equal(val, A.val)
+    P = gen.permutation(n, 4)
+    T = gen.tridiag(n, 2.0, 3.0, 5.0)
+    for X, Y in ((P, T), (T, P), (T, T)):
+        for thr in (0, 8):
+            (rp, col, val), _, _ = _full_product(X, Y, thr)
+            R = oracle.spgemm(X, Y, with_absmag=True)
+            assert np.array_equal(rp, R.row_ptr)
+            compare_rows(rp, col, val, R, "f64", exact_values=True)
+
+
+def test_rectangular_and_ragged():
+    A = gen.random_pattern(37, 5000, 0.01, 3)
+    B = gen.random_pattern(5000, 70000, 0.002, 4)
+    for thr in (0, 16, 4096):
+        (rp, col, val), _, _ = _full_product(A, B, thr)
+        R = oracle.spgemm(A, B, with_absmag=True)
+        assert np.array_equal(rp, R.row_ptr)
+        compare_rows(rp, col, val, R, "f64")
+
+
+def test_empty_inputs():
+    Z = gen.empty_rows(100, 100)
+    (rp, col, val), info, cls = _full_product(Z, Z, 10)
+    assert np.all(rp == 0) and col.size == 0 and info["n_empty"] == 100
+    A = gen.random_pattern(1, 1, 1.0, 1)
+    (rp, col, val), _, _ = _full_product(A, A, 0)
+    assert list(rp) == [0, 1] and list(col) == [0]
+
+
+def test_row_subrange_concatenation_equals_whole():
+    A = gen.config("rmat12")
+    dA = _dev(A)
+    cuts, _ = sg.sg_partition(dA, dA, 3)
+    whole = oracle.spgemm(A, A)
+    cols, nnzs = [], []
+    for g in range(3):
+        plan = sg.sg_symbolic(dA, dA, 512, cuts[g], cuts[g + 1])
+        c, v = sg.sg_numeric(plan, dA, dA)
+        cols.append(c.cpu().numpy())
+        nnzs.append(plan.nnz)
+        plan.destroy()
+    assert np.array_equal(np.concatenate(cols), whole.col)
+
+
+def test_errors():
+    A = gen.config("C1")
+    dA = _dev(A)
+    with pytest.raises(sg.SgError, match="INVALID_ARG"):
+        sg.sg_symbolic(dA, dA, sg.SG_CAP_L_MAX + 1)
+    with pytest.raises(sg.SgError, match="INVALID_ARG"):
+        sg.sg_sample_threshold(dA, dA, 0.0, 1)
+    B = _dev(gen.random_pattern(7, 9, 0.3, 1))
+    with pytest.raises(sg.SgError, match="SHAPE"):
+        sg.sg_symbolic(dA, B, 10)
+    A32 = _dev(A.astype("f32"))
+    with pytest.raises(sg.SgError, match="DTYPE"):
+        sg.sg_symbolic(dA, A32, 10)
