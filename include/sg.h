@@ -175,6 +175,16 @@ void sg_plan_destroy(sg_plan* plan);
 sg_status sg_sample_rows(int64_t row_begin, int64_t row_end, double sample_frac, uint64_t seed,
                          int64_t* rows_out, int64_t rows_cap, int64_t* count_out /*host*/, void* stream);
 
+/* ---- instrumentation (bench.py's measured kernel durations) -------------------
+ * Every kernel launch is counted. With profiling enabled, a CUDA event pair is recorded on the
+ * launching stream around each launch; sg_profile_read (after the stream is synchronised) copies
+ * up to max records: names as 32-byte NUL-terminated strings, durations in ms. */
+void sg_profile_enable(int on);
+int64_t sg_launch_count(void);
+int64_t sg_profile_count(void);
+int64_t sg_profile_read(char* names /*host, 32*max bytes, nullable*/, double* ms /*host, max, nullable*/, int64_t max);
+void sg_profile_reset(void);
+
 #ifdef __cplusplus
 }
 #endif

@@ -35,7 +35,8 @@ _STATUS = ["SG_OK", "SG_ERR_INVALID_ARG", "SG_ERR_SHAPE", "SG_ERR_DTYPE", "SG_ER
 # every symbol include/sg.h declares (checked by tests/test_abi.py)
 EXPORTS = ["sg_status_string", "sg_version", "sg_default_cost_model", "sg_row_work", "sg_sample_threshold",
            "sg_exhaustive_threshold", "sg_cost_curve", "sg_partition", "sg_symbolic", "sg_numeric", "sg_gather",
-           "sg_plan_get_info", "sg_plan_get_classes", "sg_plan_get_work", "sg_plan_destroy", "sg_sample_rows"]
+           "sg_plan_get_info", "sg_plan_get_classes", "sg_plan_get_work", "sg_plan_destroy", "sg_sample_rows",
+           "sg_profile_enable", "sg_launch_count", "sg_profile_count", "sg_profile_read", "sg_profile_reset"]
 
 
 class SgError(RuntimeError):
@@ -115,6 +116,11 @@ def load(build_if_missing: bool = True):
         "sg_plan_get_classes": (st, [P, P, P]),
         "sg_plan_get_work": (st, [P, P, P]),
         "sg_plan_destroy": (None, [P]),
+        "sg_profile_enable": (None, [ctypes.c_int]),
+        "sg_launch_count": (i64, []),
+        "sg_profile_count": (i64, []),
+        "sg_profile_read": (i64, [P, P, i64]),
+        "sg_profile_reset": (None, []),
     }
     for name, (res, args) in sigs.items():
         f = getattr(L, name)
@@ -333,6 +339,46 @@ def sg_gather(plan: Plan, comm_ptr: int, local_col=None, local_val=None, gather_
                            _ptr(local_col), _ptr(local_val), _ptr(rp), _ptr(col), _ptr(val), ctypes.byref(tot),
                            _stream()), "sg_gather")
     return rp, col, val, int(tot.value)
+
+
+class profile:
+    """Context manager: per-launch CUDA-event timing of every libsg kernel launched inside.
+    After exit (the stream synchronised), .records is a list of (kernel_name, ms)."""
+
+    def __init__(self):
+        self.records = []
+
+    def __enter__(self):
+        lib().sg_profile_reset()
+        lib().sg_profile_enable(1)
+        self.launches0 = int(lib().sg_launch_count())
+        return self
+
+    def __exit__(self, *exc):
+        torch.cuda.synchronize()
+        L = lib()
+        L.sg_profile_enable(0)
+        n = int(L.sg_profile_count())
+        names = ctypes.create_string_buffer(32 * max(n, 1))
+        import numpy as np
+        ms = np.zeros(max(n, 1), dtype=np.float64)
+        n = int(L.sg_profile_read(names, ms.ctypes.data_as(ctypes.c_void_p), n))
+        raw = names.raw
+        self.records = [(raw[32 * i:32 * i + 32].split(b"\0")[0].decode(), float(ms[i])) for i in range(n)]
+        self.launches = int(L.sg_launch_count()) - self.launches0
+        L.sg_profile_reset()
+        return False
+
+    def by_kernel(self):
+        out = {}
+        for name, t in self.records:
+            c, s = out.get(name, (0, 0.0))
+            out[name] = (c + 1, s + t)
+        return out
+
+
+def launch_count() -> int:
+    return int(lib().sg_launch_count())
 
 
 def spgemm(A: DeviceCSR, B: DeviceCSR, sample_frac: float = 0.01, seed: int = 1, cm: CostModel | None = None,

@@ -21,10 +21,14 @@ struct sg_plan {
     int64_t bin_cnt[NBINS] = {0};
     int64_t bin_off[NBINS + 1] = {0};
     int64_t nheavy = 0;
+    int32_t* heavy = nullptr;       // heavy rows (local ids), heaviest first
     int64_t* range_bounds = nullptr;
     int64_t* range_off = nullptr;
+    int32_t* nranges = nullptr;
     RangeRec* ranges = nullptr;
-    int64_t nslots = 0;
+    int64_t nslots = 0, amax = 0;
+    int2* span = nullptr;           // light rows: [cmin, cmax] of the output columns
+    int4* gscr = nullptr;           // heavy rows with more than KC entries: per-k cursor scratch
     int32_t* long_id = nullptr;
     uint32_t* tp = nullptr;
     int64_t nlong = 0;
@@ -113,7 +117,7 @@ sg_status validate_one(const sg_csr_view* v, cudaStream_t s) {
         if (!bad) return SG_ERR_OOM;
         CK(cudaMemsetAsync(bad, 0, sizeof(int), s));
         Mat m = mat_of(v);
-        if (m.nrows > 0) k_validate<<<(unsigned)((m.nrows + 255) / 256 < 4096 ? (m.nrows + 255) / 256 : 4096), 256, 0, s>>>(m, bad);
+        if (m.nrows > 0) SG_LAUNCH("k_validate", s, k_validate<<<(unsigned)((m.nrows + 255) / 256 < 4096 ? (m.nrows + 255) / 256 : 4096), 256, 0, s>>>(m, bad));
         CK(cudaGetLastError());
         int h = 0;
         CK(cudaMemcpyAsync(&h, bad, sizeof(int), cudaMemcpyDeviceToHost, s));
@@ -144,7 +148,7 @@ CostModelD cm_of(const sg_cost_model* c) {
 const sg_cost_model kDefaultModel = {
     /*kappa_L*/ 3000, /*lambda_L*/ 120, /*sigma_L*/ 0, /*rho_L*/ 150,
     /*kappa_H*/ 250000, /*lambda_H*/ 60, /*tau_H*/ 400, /*mu_H*/ 120,
-    /*tiles_fixed*/ 1, /*capu*/ CAPU, /*cap_L*/ SG_CAP_L_MAX};
+    /*tiles_fixed*/ 1, /*capu*/ 12288, /*cap_L*/ SG_CAP_L_MAX};
 
 // Identify over a row list (rows == nullptr: rows [0, nr)). Computes w, a, u of those rows on the
 // device (exact sample-symbolic at routing threshold cap_L), then the cost histogram.
@@ -187,8 +191,11 @@ sg_status row_stats(const Mat& A, const Mat& B, const int64_t* rows, int64_t nr,
     CK(cudaMemcpyAsync(dbin + NBINS, off, sizeof(int64_t) * NBINS, cudaMemcpyHostToDevice, s));
     CK(launch_bin_scatter(rs.w, nr, cap, dbin + NBINS, lists, s));
     for (int b = 0; b < NBIN_LIGHT; ++b)
-        CK(launch_sym_light(b, A, B, lists + off[b], cnt[b], rows, 0, rs.u, s));
-    CK(launch_sym_heavy(A, B, lists + off[BIN_HEAVY], cnt[BIN_HEAVY], rows, 0, rs.w, rs.u, nullptr, nullptr, s));
+        CK(launch_sym_light(b, A, B, lists + off[b], cnt[b], rows, 0, rs.u, nullptr, s));
+    unsigned long long* counter = (unsigned long long*)sc.get(sizeof(unsigned long long));
+    if (!counter) return SG_ERR_OOM;
+    CK(launch_sym_heavy(A, B, lists + off[BIN_HEAVY], cnt[BIN_HEAVY], rows, 0, rs.u, nullptr, nullptr, nullptr,
+                        counter, s));
     return SG_OK;
 }
 
@@ -432,10 +439,12 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
     pl->u = (int64_t*)palloc(pl, 8 * nrb);
     pl->dbin = (int64_t*)palloc(pl, sizeof(int64_t) * (2 * NBINS + 2));
     pl->long_id = (int32_t*)palloc(pl, 4 * (size_t)(pl->m > 0 ? pl->m : 1));
-    pl->counter = (unsigned long long*)palloc(pl, sizeof(unsigned long long));
+    pl->counter = (unsigned long long*)palloc(pl, sizeof(unsigned long long) * 2);
+    pl->span = (int2*)palloc(pl, sizeof(int2) * nrb);
     void* stmp = palloc(pl, scan_tmp_bytes(nr + 1));
-    if (!pl->w || !pl->cls || !pl->lists || !pl->u || !pl->dbin || !pl->long_id || !pl->counter || !stmp)
+    if (!pl->w || !pl->cls || !pl->lists || !pl->u || !pl->dbin || !pl->long_id || !pl->counter || !pl->span || !stmp)
         return fail(SG_ERR_OOM);
+    if (B->nnz >= INT32_MAX) return fail(SG_ERR_OVERFLOW);  // heavy cursors hold B positions in int32
     pl->T = (int)((pl->p + TW - 1) / TW);
     if (pl->T < 1) pl->T = 1;
 #define CKF(x) do { if ((x) != cudaSuccess) { cudaGetLastError(); return fail(SG_ERR_CUDA); } } while (0)
@@ -453,30 +462,41 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
     pl->nlong = hc[NBINS];
     CKF(cudaMemcpyAsync(pl->dbin + NBINS + 1, pl->bin_off, sizeof(int64_t) * NBINS, cudaMemcpyHostToDevice, s));
     CKF(launch_bin_scatter(pl->w, nr, thr, pl->dbin + NBINS + 1, pl->lists, s));
-    // heavy: range-slot bounds -> offsets
+    // heavy rows heaviest-first, range-slot bounds -> offsets, B tile pointers
     pl->nheavy = pl->bin_cnt[BIN_HEAVY];
-    const int32_t* heavy = pl->lists + pl->bin_off[BIN_HEAVY];
     if (pl->nheavy > 0) {
+        pl->heavy = (int32_t*)palloc(pl, 4 * (size_t)pl->nheavy);
+        unsigned int* hist = (unsigned int*)palloc(pl, 128 * sizeof(unsigned int));
         pl->range_bounds = (int64_t*)palloc(pl, 8 * (size_t)pl->nheavy);
         pl->range_off = (int64_t*)palloc(pl, 8 * (size_t)(pl->nheavy + 1));
+        pl->nranges = (int32_t*)palloc(pl, 4 * (size_t)pl->nheavy);
         void* t2 = palloc(pl, scan_tmp_bytes(pl->nheavy));
-        if (!pl->range_bounds || !pl->range_off || !t2) return fail(SG_ERR_OOM);
-        CKF(launch_range_bounds(heavy, pl->nheavy, pl->w, pl->p, pl->range_bounds, s));
+        if (!pl->heavy || !hist || !pl->range_bounds || !pl->range_off || !pl->nranges || !t2) return fail(SG_ERR_OOM);
+        CKF(launch_heavy_order(pl->lists + pl->bin_off[BIN_HEAVY], pl->nheavy, pl->w, hist, pl->heavy, s));
+        CKF(launch_range_bounds(pl->heavy, pl->nheavy, pl->w, pl->p, pl->range_bounds, s));
         CKF(scan_exclusive(pl->range_bounds, pl->range_off, pl->nheavy, t2, s));
-        CKF(cudaMemcpyAsync(&pl->nslots, pl->range_off + pl->nheavy, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        CKF(cudaMemsetAsync(pl->counter + 1, 0, sizeof(unsigned long long), s));
+        CKF(launch_max_a(a, pl->heavy, pl->nheavy, row_begin, pl->counter + 1, s));
+        int64_t hb[2];
+        CKF(cudaMemcpyAsync(&hb[0], pl->range_off + pl->nheavy, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        CKF(cudaMemcpyAsync(&hb[1], pl->counter + 1, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
         CKF(cudaStreamSynchronize(s));
-        pl->ranges = (RangeRec*)palloc(pl, sizeof(RangeRec) * (size_t)pl->nslots);
-        if (!pl->ranges) return fail(SG_ERR_OOM);
-        CKF(launch_fill_ranges_unused(pl->ranges, pl->nslots, s));
-        // B tile pointers for long rows (numeric heavy path)
+        pl->nslots = hb[0];
+        pl->amax = hb[1];
+        pl->ranges = (RangeRec*)palloc(pl, sizeof(RangeRec) * (size_t)(pl->nslots > 0 ? pl->nslots : 1));
         pl->tp = (uint32_t*)palloc(pl, 4 * (size_t)(pl->nlong > 0 ? pl->nlong : 1) * (size_t)(pl->T + 1));
-        if (!pl->tp) return fail(SG_ERR_OOM);
+        if (!pl->ranges || !pl->tp) return fail(SG_ERR_OOM);
+        if (pl->amax > heavy_kc()) {
+            pl->gscr = (int4*)palloc(pl, sizeof(int4) * 148 * (size_t)pl->amax);
+            if (!pl->gscr) return fail(SG_ERR_OOM);
+        }
         if (pl->nlong > 0) CKF(launch_build_tp(b, pl->long_id, pl->T, pl->tp, s));
     }
     // a6 symbolic
     for (int k = 0; k < NBIN_LIGHT; ++k)
-        CKF(launch_sym_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], nullptr, row_begin, pl->u, s));
-    CKF(launch_sym_heavy(a, b, heavy, pl->nheavy, nullptr, row_begin, pl->w, pl->u, pl->range_off, pl->ranges, s));
+        CKF(launch_sym_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], nullptr, row_begin, pl->u, pl->span, s));
+    CKF(launch_sym_heavy(a, b, pl->heavy, pl->nheavy, nullptr, row_begin, pl->u, pl->range_off, pl->ranges,
+                         pl->nranges, pl->counter, s));
     CKF(scan_exclusive(pl->u, C_row_ptr, nr, stmp, s));
     CKF(cudaMemcpyAsync(&pl->nnz_c, C_row_ptr + nr, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     CKF(cudaStreamSynchronize(s));
@@ -498,10 +518,11 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
     if (pl->nnz_c == 0) return SG_OK;
     Mat a = mat_of(A), b = mat_of(B);
     for (int k = 0; k < NBIN_LIGHT; ++k)
-        CKP(pl, launch_num_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], pl->rb, pl->C_rp, C_col, C_val, s));
+        CKP(pl, launch_num_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], pl->rb, pl->span, pl->C_rp,
+                                 C_col, C_val, s));
     if (pl->nheavy > 0)
-        CKP(pl, launch_num_heavy(a, b, pl->ranges, pl->nslots, pl->rb, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
-                                 C_val, pl->counter, s));
+        CKP(pl, launch_num_heavy(a, b, pl->heavy, pl->nheavy, pl->rb, pl->range_off, pl->nranges, pl->ranges,
+                                 pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter, pl->gscr, pl->amax, s));
     return SG_OK;
 }
 

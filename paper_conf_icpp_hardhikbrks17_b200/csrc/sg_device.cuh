@@ -1,0 +1,189 @@
+// sg_device.cuh — device helpers shared by the libsg kernels: warp primitives, group barriers,
+// the flattened product iterator and the order-preserving hash accumulator.
+#pragma once
+#include "sg_internal.cuh"
+#include <climits>
+
+namespace sg {
+
+constexpr unsigned FULL = 0xffffffffu;
+
+template <class T> __device__ __forceinline__ T warp_sum(T v) {
+    #pragma unroll
+    for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
+    return v;
+}
+__device__ __forceinline__ int warp_min(int v) {
+    #pragma unroll
+    for (int o = 16; o; o >>= 1) v = min(v, __shfl_xor_sync(FULL, v, o));
+    return v;
+}
+__device__ __forceinline__ int warp_max(int v) {
+    #pragma unroll
+    for (int o = 16; o; o >>= 1) v = max(v, __shfl_xor_sync(FULL, v, o));
+    return v;
+}
+template <class T> __device__ __forceinline__ T warp_incl_scan(T v) {
+    const int lane = threadIdx.x & 31;
+    #pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        T y = __shfl_up_sync(FULL, v, o);
+        if (lane >= o) v += y;
+    }
+    return v;
+}
+__device__ __forceinline__ unsigned lanemask_lt() {
+    unsigned m;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+    return m;
+}
+
+template <class VT> __device__ __forceinline__ double ldv(const void* v, int64_t q) {
+    return (double)__ldg(reinterpret_cast<const VT*>(v) + q);
+}
+
+static inline int grid_for(int64_t work, int per_block, int max_blocks) {
+    int64_t g = (work + per_block - 1) / per_block;
+    if (g < 1) g = 1;
+    if (g > max_blocks) g = max_blocks;
+    return (int)g;
+}
+
+// ---- groups: G threads own one row (G = 32: a warp; G = BLK: the block; else named barriers) ----
+template <int G, int BLK> __device__ __forceinline__ void group_bar() {
+    if constexpr (G == 32) __syncwarp();
+    else if constexpr (G == BLK) __syncthreads();
+    else {
+        const int g = threadIdx.x / G;
+        asm volatile("bar.sync %0, %1;" ::"r"(1 + g), "r"(G) : "memory");
+    }
+}
+
+// ---- flattened products of up to 32 consecutive A entries [pa0, pa1) of one row -------------------
+// Lane l loads k_l = A.col[pa0 + l] and its B-row segment; an exclusive scan of the segment lengths
+// flattens the products so that every lane gathers an independent (col, val) per round, UNR rounds
+// in flight (memory-level parallelism instead of one dependent chain per k).
+// seg(k, q0, len) may narrow the segment (heavy ranges); f(c, v) consumes a product.
+template <bool VAL, class VT, int UNR, class SEG, class F>
+__device__ __forceinline__ void chunk_products(const Mat& A, const Mat& B, int64_t pa0, int64_t pa1, SEG&& seg,
+                                               F&& f) {
+    const int lane = threadIdx.x & 31;
+    const int64_t pa = pa0 + lane;
+    int len = 0;
+    int64_t q0 = 0;
+    double a = 0.0;
+    if (pa < pa1) {
+        const int k = __ldg(A.col + pa);
+        q0 = __ldg(B.rp + k);
+        len = (int)(__ldg(B.rp + k + 1) - q0);
+        if (VAL) a = ldv<VT>(A.val, pa);
+        seg(k, q0, len);
+    }
+    const int inc = warp_incl_scan(len);
+    const int off = inc - len;
+    const int tot = __shfl_sync(FULL, inc, 31);
+    for (int j0 = 0; j0 < tot; j0 += 32 * UNR) {
+        int c[UNR];
+        double v[UNR];
+        #pragma unroll
+        for (int r = 0; r < UNR; ++r) {
+            const int j = j0 + 32 * r + lane;
+            int s = 0;
+            #pragma unroll
+            for (int b = 16; b; b >>= 1) {
+                const int o = __shfl_sync(FULL, off, s + b);
+                if (o <= j) s += b;
+            }
+            const int64_t q = __shfl_sync(FULL, q0, s) + (j - __shfl_sync(FULL, off, s));
+            const double as = VAL ? __shfl_sync(FULL, a, s) : 0.0;
+            c[r] = -1;
+            if (j < tot) {
+                c[r] = __ldg(B.col + q);
+                if (VAL) v[r] = as * ldv<VT>(B.val, q);
+            }
+        }
+        #pragma unroll
+        for (int r = 0; r < UNR; ++r)
+            if (c[r] >= 0) f(c[r], VAL ? v[r] : 0.0);
+    }
+}
+
+// ---- the order-preserving hash accumulator -----------------------------------------------------
+// home(c) = identity (c - lo) when the span fits the table, else floor((c - lo) * mult / 2^32),
+// monotone in c; linear probing moves forward only, never wraps (overflow room >= capacity).
+// Returns the slot used.
+__device__ __forceinline__ int acc_insert(int32_t* keys, double* vals, int32_t c, double v, uint32_t d, bool ident,
+                                          uint64_t mult) {
+    uint32_t h;
+    if (ident) {
+        h = d;
+        if (keys[h] != c) keys[h] = c;  // idempotent: every writer stores the same key
+    } else {
+        h = (uint32_t)(((uint64_t)d * mult) >> 32);
+        while (true) {
+            int32_t old = keys[h];
+            if (old == c) break;
+            if (old == EMPTY_KEY) {
+                old = atomicCAS(&keys[h], EMPTY_KEY, c);
+                if (old == EMPTY_KEY || old == c) break;
+            }
+            ++h;
+        }
+    }
+    atomicAdd(&vals[h], v);
+    return (int)h;
+}
+
+// sort the occupied run starting at slot s (insertion sort; runs are short at load <= 1/2)
+__device__ __forceinline__ void sort_run(int32_t* keys, double* vals, int s, int nslots) {
+    int e = s + 1;
+    while (e < nslots && keys[e] != EMPTY_KEY) ++e;
+    for (int i = s + 1; i < e; ++i) {
+        const int32_t k = keys[i];
+        const double v = vals[i];
+        int q = i - 1;
+        while (q >= s && keys[q] > k) { keys[q + 1] = keys[q]; vals[q + 1] = vals[q]; --q; }
+        keys[q + 1] = k;
+        vals[q + 1] = v;
+    }
+}
+
+// Group-wide emission of slots [0, nslots) in slot order into C at `base`, clearing each slot.
+// Each warp of the group owns a contiguous chunk of slots; one group-level exclusive scan of the
+// per-warp counts places the chunks (ws: >= G/32 ints of shared memory per group).
+template <int G, int BLK, class VT>
+__device__ __forceinline__ void emit_slots(int32_t* keys, double* vals, int nslots, int64_t base,
+                                           int32_t* __restrict__ C_col, VT* __restrict__ C_val, int* ws) {
+    constexpr int NW = G / 32;
+    const int lane = threadIdx.x & 31;
+    const int w = (threadIdx.x % G) / 32;
+    const int chunk = ((nslots + NW - 1) / NW + 31) & ~31;
+    const int s_lo = w * chunk, s_hi = min(nslots, s_lo + chunk);
+    int64_t pos = base;
+    if constexpr (NW > 1) {
+        int cnt = 0;
+        for (int s0 = s_lo; s0 < s_hi; s0 += 32) {
+            const int s = s0 + lane;
+            cnt += __popc(__ballot_sync(FULL, s < s_hi && keys[s] != EMPTY_KEY));
+        }
+        if (lane == 0) ws[w] = cnt;
+        group_bar<G, BLK>();
+        for (int q = 0; q < w; ++q) pos += ws[q];
+        group_bar<G, BLK>();
+    }
+    for (int s0 = s_lo; s0 < s_hi; s0 += 32) {
+        const int s = s0 + lane;
+        const int32_t k = s < s_hi ? keys[s] : EMPTY_KEY;
+        const unsigned m = __ballot_sync(FULL, k != EMPTY_KEY);
+        if (k != EMPTY_KEY) {
+            const int64_t o = pos + __popc(m & lanemask_lt());
+            C_col[o] = k;
+            C_val[o] = (VT)vals[s];
+            keys[s] = EMPTY_KEY;
+            vals[s] = 0.0;
+        }
+        pos += __popc(m);
+    }
+}
+
+}  // namespace sg

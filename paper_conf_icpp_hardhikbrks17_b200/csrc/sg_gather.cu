@@ -102,7 +102,7 @@ extern "C" sg_status sg_gather(sg_plan* plan, void* nccl_comm, int gather_values
         }
         if (n > 0) {
             int grid = (int)((n + 255) / 256 < 148 * 8 ? (n + 255) / 256 : 148 * 8);
-            k_fix_offsets<<<grid, 256, 0, s>>>(C_row_ptr_global, dlay, dlay + nranks, nranks, n);
+            SG_LAUNCH("k_fix_offsets", s, k_fix_offsets<<<grid, 256, 0, s>>>(C_row_ptr_global, dlay, dlay + nranks, nranks, n));
         }
         if (cudaGetLastError() != cudaSuccess || cudaStreamSynchronize(s) != cudaSuccess) { st = SG_ERR_CUDA; break; }
         *nnz_total_out = total;

@@ -1,0 +1,565 @@
+// sg_heavy.cu — the HEAVY path (w_i > thr, "more than t"): one CTA (1024 threads)
+// per heavy row, rows taken heaviest-first from a dynamic counter.
+//
+// Symbolic: the row's products set bits of a shared-memory bitmap over a 2^20-column window;
+// per-8192-column-tile popcounts give u_i and a plan of column RANGES, each holding at most
+// RCAP = 16384 output entries and spanning at most RW_TILES tiles (the numeric accumulator).
+//
+// Numeric, per range [lo, hi): pass 1 rebuilds the range's bitmap, a block scan turns word
+// popcounts into a rank prefix, pass 2 accumulates every product into a COMPACT fp64 array at
+// rank(c) = prefix[word] + popc(word & below) — a rank-indexed dense accumulator: no hashing, no
+// probing, and the emission (bitmap scan + contiguous value copy) is sorted by construction.
+// Products are flattened over the whole block (one k per thread, block scan of segment lengths,
+// per-product binary search), so rows with few k (median 9 on R-MAT) still use every warp.
+// Per-k cursors advance monotonically across ranges; B rows longer than LONG_ROW locate their
+// segment through the tile-pointer table tp (one load), short rows by a bounded scan.
+#include "sg_device.cuh"
+
+namespace sg {
+
+constexpr int KC = HEAVY_THREADS;  // k entries per chunk: one per thread
+constexpr int RW_TILES = 32;       // max tiles per numeric range -> 256K columns, 32 KB bitmap
+constexpr int RW_WORDS = RW_TILES * TW / 32;
+constexpr int RCAP = 16384;        // max entries per numeric range (fp64 accumulator 128 KB)
+constexpr int RHALF = RCAP / 2;    // range key granularity (a range = run of tiles with equal key)
+
+__device__ __forceinline__ int64_t lower_bound_col(const int32_t* __restrict__ col, int64_t lo, int64_t hi, int64_t x) {
+    while (lo < hi) {
+        int64_t mid = (lo + hi) >> 1;
+        if ((int64_t)__ldg(col + mid) < x) lo = mid + 1; else hi = mid;
+    }
+    return lo;
+}
+
+// exclusive scan of one int per thread over a 1024-thread block; *total for everyone
+__device__ __forceinline__ int block_scan1024(int v, int* total, int* ws) {
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    int inc = warp_incl_scan(v);
+    if (lane == 31) ws[wid] = inc;
+    __syncthreads();
+    if (wid == 0) {
+        int x = ws[lane];
+        int xi = warp_incl_scan(x);
+        ws[lane] = xi - x;
+        if (lane == 31) ws[32] = xi;
+    }
+    __syncthreads();
+    int r = ws[wid] + inc - v;
+    *total = ws[32];
+    __syncthreads();
+    return r;
+}
+
+// largest i in [0, nk) with off[i] <= j (that entry has len > 0)
+__device__ __forceinline__ int find_k(const int* off, int nk, int j) {
+    int lo = 0, hi = nk - 1;
+    while (lo < hi) {
+        int mid = (lo + hi + 1) >> 1;
+        if (off[mid] <= j) lo = mid; else hi = mid - 1;
+    }
+    return lo;
+}
+
+// ------------------------------------------------------------------------------------------------
+// B tile pointers: for B rows longer than LONG_ROW, tp[id][t] = #entries with col < t*TW
+// ------------------------------------------------------------------------------------------------
+__global__ void k_long_rows(Mat B, int32_t* __restrict__ long_id, unsigned long long* nlong) {
+    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < B.nrows; k += (int64_t)gridDim.x * blockDim.x) {
+        int64_t len = B.rp[k + 1] - B.rp[k];
+        long_id[k] = len > LONG_ROW ? (int32_t)atomicAdd(nlong, 1ull) : -1;
+    }
+}
+
+cudaError_t launch_long_rows(const Mat& B, int32_t* long_id, int64_t* d_nlong, cudaStream_t s) {
+    if (B.nrows <= 0) return cudaSuccess;
+    SG_LAUNCH("k_long_rows", s, (k_long_rows<<<grid_for(B.nrows, 256, 148 * 8), 256, 0, s>>>(B, long_id, (unsigned long long*)d_nlong)));
+    return cudaGetLastError();
+}
+
+__global__ void k_build_tp(Mat B, const int32_t* __restrict__ long_id, int T, uint32_t* __restrict__ tp) {
+    const int lane = threadIdx.x & 31;
+    int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t k = warp; k < B.nrows; k += nw) {
+        int id = long_id[k];
+        if (id < 0) continue;
+        int64_t q0 = B.rp[k], q1 = B.rp[k + 1];
+        uint32_t* row = tp + (int64_t)id * (T + 1);
+        for (int t = lane; t <= T; t += 32)
+            row[t] = (uint32_t)(lower_bound_col(B.col, q0, q1, (int64_t)t * TW) - q0);
+    }
+}
+
+cudaError_t launch_build_tp(const Mat& B, const int32_t* long_id, int T, uint32_t* tp, cudaStream_t s) {
+    if (B.nrows <= 0) return cudaSuccess;
+    SG_LAUNCH("k_build_tp", s, (k_build_tp<<<grid_for(B.nrows, 8, 148 * 16), 256, 0, s>>>(B, long_id, T, tp)));
+    return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------------
+// heavy rows heaviest-first: counting sort of the heavy list by descending ceil(log2 w)
+// ------------------------------------------------------------------------------------------------
+__global__ void k_heavy_hist(const int32_t* __restrict__ heavy, int64_t nh, const int64_t* __restrict__ w,
+                             unsigned int* hist) {
+    __shared__ unsigned int sh[64];
+    if (threadIdx.x < 64) sh[threadIdx.x] = 0;
+    __syncthreads();
+    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < nh; j += (int64_t)gridDim.x * blockDim.x)
+        atomicAdd(&sh[63 - (64 - __clzll((unsigned long long)w[heavy[j]]))], 1u);  // descending log2
+    __syncthreads();
+    if (threadIdx.x < 64 && sh[threadIdx.x]) atomicAdd(&hist[threadIdx.x], sh[threadIdx.x]);
+}
+
+__global__ void k_heavy_scatter(const int32_t* __restrict__ heavy, int64_t nh, const int64_t* __restrict__ w,
+                                unsigned int* hist /*64 counts -> cursors*/, int32_t* __restrict__ out) {
+    __shared__ unsigned int base[64];
+    if (threadIdx.x == 0) {
+        // every block recomputes the exclusive offsets from the counts in hist[0..64)
+        unsigned int a = 0;
+        for (int b = 0; b < 64; ++b) { base[b] = a; a += hist[b]; }
+    }
+    __syncthreads();
+    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < nh; j += (int64_t)gridDim.x * blockDim.x) {
+        int b = 63 - (64 - __clzll((unsigned long long)w[heavy[j]]));
+        unsigned int pos = atomicAdd(&hist[64 + b], 1u);
+        out[base[b] + pos] = heavy[j];
+    }
+}
+
+cudaError_t launch_heavy_order(const int32_t* heavy, int64_t nh, const int64_t* w, unsigned int* hist128,
+                               int32_t* out, cudaStream_t s) {
+    if (nh <= 0) return cudaSuccess;
+    cudaError_t e = cudaMemsetAsync(hist128, 0, 128 * sizeof(unsigned int), s);
+    if (e != cudaSuccess) return e;
+    int g = grid_for(nh, 1024, 148 * 4);
+    SG_LAUNCH("k_heavy_hist", s, (k_heavy_hist<<<g, 256, 0, s>>>(heavy, nh, w, hist128)));
+    SG_LAUNCH("k_heavy_scatter", s, (k_heavy_scatter<<<g, 256, 0, s>>>(heavy, nh, w, hist128, out)));
+    return cudaGetLastError();
+}
+
+// per heavy row: an upper bound on its range count
+__global__ void k_range_bounds(const int32_t* __restrict__ heavy, int64_t nh, const int64_t* __restrict__ w,
+                               int64_t p, int64_t* __restrict__ bounds) {
+    int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (j >= nh) return;
+    int64_t wi = w[heavy[j]];
+    int64_t mu = wi < p ? wi : p;
+    int64_t T = (p + TW - 1) / TW;
+    int64_t nwin = (p + WIN - 1) / WIN;
+    // distinct keys per window <= u_win / RHALF + 1 + (tiles per window / RW_TILES)
+    int64_t b = mu / RHALF + nwin * (1 + (WIN / TW) / RW_TILES) + 1;
+    bounds[j] = b < T ? b : T;
+}
+
+cudaError_t launch_range_bounds(const int32_t* heavy, int64_t nh, const int64_t* w, int64_t p, int64_t* bounds,
+                                cudaStream_t s) {
+    if (nh <= 0) return cudaSuccess;
+    SG_LAUNCH("k_range_bounds", s, (k_range_bounds<<<(unsigned)((nh + 255) / 256), 256, 0, s>>>(heavy, nh, w, p, bounds)));
+    return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------------
+// a6 heavy symbolic
+// ------------------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(HEAVY_THREADS, 1) k_sym_heavy(Mat A, Mat B, const int32_t* __restrict__ list,
+                                                                 int64_t cnt, const int64_t* __restrict__ rowmap,
+                                                                 int64_t rb, int64_t* __restrict__ u,
+                                                                 const int64_t* __restrict__ range_off,
+                                                                 RangeRec* __restrict__ ranges,
+                                                                 int32_t* __restrict__ nranges,
+                                                                 unsigned long long* counter) {
+    extern __shared__ uint32_t bm[];  // WIN/32 words
+    __shared__ int64_t s_beg[KC];
+    __shared__ int s_off[KC];
+    __shared__ int tcnt[WIN / TW];
+    __shared__ int Ps[WIN / TW];
+    __shared__ unsigned char st[WIN / TW];
+    __shared__ int ws[33];
+    __shared__ long long s_j;
+    __shared__ int s_nr, s_u;
+    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5, nwarps = HEAVY_THREADS / 32;
+    const int64_t p = B.ncols;
+    const int64_t nwin = (p + WIN - 1) / WIN;
+    while (true) {
+        if (tid == 0) s_j = (long long)atomicAdd(counter, 1ull);
+        __syncthreads();
+        const int64_t j = s_j;
+        __syncthreads();
+        if (j >= cnt) break;
+        const int64_t li = list[j];
+        const int64_t row = rowmap ? rowmap[li] : rb + li;
+        const int64_t s0 = __ldg(A.rp + row), s1 = __ldg(A.rp + row + 1);
+        int utot = 0, nr = 0;
+        for (int64_t win = 0; win < nwin; ++win) {
+            const int64_t wlo = win * WIN, whi = min(p, wlo + WIN);
+            const int nwords = (int)((whi - wlo + 31) / 32);
+            for (int q = tid; q < nwords; q += HEAVY_THREADS) bm[q] = 0u;
+            for (int64_t c0 = s0; c0 < s1; c0 += KC) {
+                const int64_t i = c0 + tid;
+                int len = 0;
+                int64_t beg = 0;
+                if (i < s1) {
+                    const int k = __ldg(A.col + i);
+                    int64_t q0 = __ldg(B.rp + k), q1 = __ldg(B.rp + k + 1);
+                    if (nwin > 1) {
+                        q0 = lower_bound_col(B.col, q0, q1, wlo);
+                        q1 = lower_bound_col(B.col, q0, q1, whi);
+                    }
+                    beg = q0;
+                    len = (int)(q1 - q0);
+                }
+                int tot;
+                const int off = block_scan1024(len, &tot, ws);  // (its barriers also order the bitmap clear)
+                s_beg[tid] = beg;
+                s_off[tid] = off;
+                __syncthreads();
+                const int nk = (int)min((int64_t)KC, s1 - c0);
+                for (int jb = tid; jb < tot; jb += HEAVY_THREADS * 4) {
+                    int c[4];
+                    #pragma unroll
+                    for (int r = 0; r < 4; ++r) {
+                        const int jj = jb + r * HEAVY_THREADS;
+                        c[r] = -1;
+                        if (jj < tot) {
+                            const int kk = find_k(s_off, nk, jj);
+                            c[r] = __ldg(B.col + s_beg[kk] + (jj - s_off[kk]));
+                        }
+                    }
+                    #pragma unroll
+                    for (int r = 0; r < 4; ++r)
+                        if (c[r] >= 0) {
+                            const uint32_t d = (uint32_t)(c[r] - wlo);
+                            atomicOr(&bm[d >> 5], 1u << (d & 31));
+                        }
+                }
+                __syncthreads();
+            }
+            // per-tile popcounts
+            const int nt = (int)((whi - wlo + TW - 1) / TW);
+            for (int tt = wid; tt < nt; tt += nwarps) {
+                const int a = tt * (TW / 32), b = min(nwords, a + TW / 32);
+                int c = 0;
+                for (int q = a + lane; q < b; q += 32) c += __popc(bm[q]);
+                c = warp_sum(c);
+                if (lane == 0) tcnt[tt] = c;
+            }
+            __syncthreads();
+            // range plan (warp 0): key(t) = (ceil(P_t / RHALF) - 1, t / RW_TILES); a range is a run of
+            // equal keys -> count <= RHALF + cnt(first tile) <= RCAP, width <= RW_TILES tiles.
+            if (wid == 0) {
+                int c4[4], loc = 0;
+                #pragma unroll
+                for (int q = 0; q < 4; ++q) { const int t = 4 * lane + q; c4[q] = t < nt ? tcnt[t] : 0; loc += c4[q]; }
+                int pre = warp_incl_scan(loc) - loc;
+                int key[4];
+                #pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const int t = 4 * lane + q;
+                    pre += c4[q];
+                    key[q] = ((pre + RHALF - 1) / RHALF - 1) * 8 + t / RW_TILES;
+                    if (t < nt) Ps[t] = pre;
+                }
+                const int prevkey = __shfl_up_sync(FULL, key[3], 1);
+                #pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const int t = 4 * lane + q;
+                    const int kp = q == 0 ? prevkey : key[q - 1];
+                    if (t < nt) st[t] = (t == 0 || key[q] != kp) ? 1 : 0;
+                }
+                __syncwarp();
+                for (int t0 = 0; t0 < nt; t0 += 32) {
+                    const int t = t0 + lane;
+                    int e = t + 1, cntr = 0;
+                    bool valid = false;
+                    if (t < nt && st[t]) {
+                        while (e < nt && !st[e]) ++e;
+                        cntr = Ps[e - 1] - (t > 0 ? Ps[t - 1] : 0);
+                        valid = cntr > 0;
+                    }
+                    const unsigned m = __ballot_sync(FULL, valid);
+                    if (valid && ranges) {
+                        RangeRec r;
+                        r.row = (int32_t)li;
+                        r.t0 = (int32_t)(wlo / TW) + t;
+                        r.t1 = (int32_t)(wlo / TW) + e;
+                        r.cnt = cntr;
+                        r.off = utot + (t > 0 ? Ps[t - 1] : 0);
+                        r.pad = 0;
+                        ranges[range_off[j] + nr + __popc(m & lanemask_lt())] = r;
+                    }
+                    nr += __popc(m);
+                }
+                if (lane == 0) { s_nr = nr; s_u = utot + Ps[nt - 1]; }
+            }
+            __syncthreads();
+            nr = s_nr;
+            utot = s_u;
+            __syncthreads();
+        }
+        if (tid == 0) {
+            u[li] = utot;
+            if (nranges) nranges[j] = nr;
+        }
+    }
+}
+
+cudaError_t launch_sym_heavy(const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, const int64_t* rowmap,
+                             int64_t rb, int64_t* u, const int64_t* range_off, RangeRec* ranges, int32_t* nranges,
+                             unsigned long long* counter, cudaStream_t s) {
+    if (cnt <= 0) return cudaSuccess;
+    const int smem = (WIN / 32) * 4;
+    cudaError_t e = cudaFuncSetAttribute(k_sym_heavy, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    if ((e = cudaMemsetAsync(counter, 0, sizeof(unsigned long long), s)) != cudaSuccess) return e;
+    const int grid = (int)(cnt < 148 ? cnt : 148);
+    SG_LAUNCH("k_sym_heavy", s, (k_sym_heavy<<<grid, HEAVY_THREADS, smem, s>>>(A, B, list, cnt, rowmap, rb, u, range_off,
+                                                                                ranges, nranges, counter)));
+    return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------------
+// a7 + a8 heavy numeric: rank-indexed compact accumulator per range
+// ------------------------------------------------------------------------------------------------
+struct HeavySmem {
+    uint32_t bm[RW_WORDS];       // 32 KB  range bitmap
+    double vals[RCAP];           // 128 KB compact accumulator (by rank)
+    uint16_t pref[RW_WORDS];     // 16 KB  rank prefix per bitmap word
+    int32_t s_beg[KC];           // segment begin (B position) of chunk entry
+    int32_t s_off[KC];           // exclusive prefix of segment lengths
+    double s_a[KC];              // a_ik
+    int32_t c_cur[KC];           // single-chunk rows: cursor (B position)
+    int32_t c_nextc[KC];         //                    column at the cursor (INT_MAX: exhausted)
+    int32_t c_end[KC];           //                    end of the B row
+    int32_t c_q0[KC];            //                    start of the B row
+    int32_t c_lid[KC];           //                    long-row id or -1
+    int ws[33];
+};
+
+template <class VT>
+__global__ void __launch_bounds__(HEAVY_THREADS, 1) k_num_heavy(
+    Mat A, Mat B, const int32_t* __restrict__ heavy, int64_t nheavy, int64_t rb, const int64_t* __restrict__ range_off,
+    const int32_t* __restrict__ nranges, const RangeRec* __restrict__ ranges, const int32_t* __restrict__ long_id,
+    const uint32_t* __restrict__ tp, int T, const int64_t* __restrict__ C_rp, int32_t* __restrict__ C_col,
+    VT* __restrict__ C_val, unsigned long long* counter, int4* __restrict__ gscr, int64_t amax) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    HeavySmem& S = *reinterpret_cast<HeavySmem*>(smem_raw);
+    __shared__ long long s_j;
+    const int tid = threadIdx.x;
+    const int64_t p = B.ncols;
+    int4* gs = gscr + (int64_t)blockIdx.x * amax;  // multi-chunk rows: per-k (cur, nextc, beg, len)
+    for (int q = tid; q < RW_WORDS; q += HEAVY_THREADS) S.bm[q] = 0u;
+    for (int q = tid; q < RCAP; q += HEAVY_THREADS) S.vals[q] = 0.0;
+    while (true) {
+        if (tid == 0) s_j = (long long)atomicAdd(counter, 1ull);
+        __syncthreads();
+        const int64_t h = s_j;
+        __syncthreads();
+        if (h >= nheavy) break;
+        const int64_t li = heavy[h];
+        const int64_t row = rb + li;
+        const int64_t s0 = __ldg(A.rp + row), s1 = __ldg(A.rp + row + 1);
+        const int na = (int)(s1 - s0);
+        const bool single = na <= KC;
+        // per-k cursor state
+        for (int i = tid; i < na; i += HEAVY_THREADS) {
+            const int k = __ldg(A.col + s0 + i);
+            const int32_t q0 = (int32_t)__ldg(B.rp + k), q1 = (int32_t)__ldg(B.rp + k + 1);
+            const int32_t nc = q0 < q1 ? __ldg(B.col + q0) : INT_MAX;
+            if (single) {
+                S.c_cur[i] = q0; S.c_nextc[i] = nc; S.c_end[i] = q1; S.c_q0[i] = q0;
+                S.c_lid[i] = q1 - q0 > LONG_ROW ? __ldg(long_id + k) : -1;
+                S.s_a[i] = ldv<VT>(A.val, s0 + i);
+            } else {
+                gs[i] = make_int4(q0, nc, 0, 0);
+            }
+        }
+        __syncthreads();
+        const int nr = nranges[h];
+        const RangeRec* rr = ranges + range_off[h];
+        const int64_t crow = C_rp[li];
+        for (int ri = 0; ri < nr; ++ri) {
+            const RangeRec R = rr[ri];
+            const int64_t lo = (int64_t)R.t0 * TW, hi = min(p, (int64_t)R.t1 * TW);
+            const int nwords = (int)((hi - lo + 31) / 32);
+            int tot = 0;
+            // ---- pass 1: segments (advance cursors) + bitmap of the range ----
+            for (int c0 = 0; c0 < na; c0 += KC) {
+                const int i = c0 + tid;
+                int len = 0, beg = 0;
+                if (i < na) {
+                    if (single) {
+                        const int nc = S.c_nextc[i];
+                        if (nc < hi) {
+                            const int cur = S.c_cur[i], e1 = S.c_end[i], lid = S.c_lid[i];
+                            int end;
+                            if (lid >= 0) end = S.c_q0[i] + (int)__ldg(tp + (int64_t)lid * (T + 1) + R.t1);
+                            else { end = cur + 1; while (end < e1 && __ldg(B.col + end) < hi) ++end; }
+                            beg = cur; len = end - cur;
+                            S.c_cur[i] = end;
+                            S.c_nextc[i] = end < e1 ? __ldg(B.col + end) : INT_MAX;
+                        }
+                    } else {
+                        const int4 g = gs[i];
+                        if (g.y < hi) {
+                            const int k = __ldg(A.col + s0 + i);
+                            const int32_t q0 = (int32_t)__ldg(B.rp + k), e1 = (int32_t)__ldg(B.rp + k + 1);
+                            int end;
+                            if (e1 - q0 > LONG_ROW) end = q0 + (int)__ldg(tp + (int64_t)__ldg(long_id + k) * (T + 1) + R.t1);
+                            else { end = g.x + 1; while (end < e1 && __ldg(B.col + end) < hi) ++end; }
+                            beg = g.x; len = end - g.x;
+                            gs[i] = make_int4(end, end < e1 ? __ldg(B.col + end) : INT_MAX, beg, len);
+                        } else {
+                            gs[i] = make_int4(g.x, g.y, g.x, 0);
+                        }
+                    }
+                }
+                int ctot;
+                const int off = block_scan1024(len, &ctot, S.ws);
+                S.s_beg[tid] = beg;
+                S.s_off[tid] = off;
+                __syncthreads();
+                const int nk = min(KC, na - c0);
+                for (int jb = tid; jb < ctot; jb += HEAVY_THREADS * 4) {
+                    int c[4];
+                    #pragma unroll
+                    for (int r = 0; r < 4; ++r) {
+                        const int jj = jb + r * HEAVY_THREADS;
+                        c[r] = -1;
+                        if (jj < ctot) {
+                            const int kk = find_k(S.s_off, nk, jj);
+                            c[r] = __ldg(B.col + S.s_beg[kk] + (jj - S.s_off[kk]));
+                        }
+                    }
+                    #pragma unroll
+                    for (int r = 0; r < 4; ++r)
+                        if (c[r] >= 0) {
+                            const uint32_t d = (uint32_t)(c[r] - lo);
+                            atomicOr(&S.bm[d >> 5], 1u << (d & 31));
+                        }
+                }
+                tot += ctot;
+                if (!single) __syncthreads();
+            }
+            __syncthreads();
+            // ---- rank prefix over the range's words (8 consecutive words per thread) ----
+            {
+                const int w0 = tid * 8;
+                int cw[8], loc = 0;
+                #pragma unroll
+                for (int q = 0; q < 8; ++q) { cw[q] = w0 + q < nwords ? __popc(S.bm[w0 + q]) : 0; loc += cw[q]; }
+                int t2;
+                int pre = block_scan1024(loc, &t2, S.ws);
+                #pragma unroll
+                for (int q = 0; q < 8; ++q) { if (w0 + q < nwords) S.pref[w0 + q] = (uint16_t)pre; pre += cw[q]; }
+            }
+            __syncthreads();
+            // ---- pass 2: accumulate into the compact array at rank(c) ----
+            for (int c0 = 0; c0 < na; c0 += KC) {
+                const int nk = min(KC, na - c0);
+                int ctot;
+                if (single) {
+                    ctot = tot;  // segments of pass 1 are still in S.s_beg / S.s_off
+                } else {
+                    const int i = c0 + tid;
+                    int len = 0, beg = 0;
+                    if (i < na) { const int4 g = gs[i]; beg = g.z; len = g.w; S.s_a[tid] = ldv<VT>(A.val, s0 + i); }
+                    const int off = block_scan1024(len, &ctot, S.ws);
+                    S.s_beg[tid] = beg;
+                    S.s_off[tid] = off;
+                    __syncthreads();
+                }
+                for (int jb = tid; jb < ctot; jb += HEAVY_THREADS * 4) {
+                    int c[4];
+                    double v[4];
+                    #pragma unroll
+                    for (int r = 0; r < 4; ++r) {
+                        const int jj = jb + r * HEAVY_THREADS;
+                        c[r] = -1;
+                        if (jj < ctot) {
+                            const int kk = find_k(S.s_off, nk, jj);
+                            const int64_t q = S.s_beg[kk] + (jj - S.s_off[kk]);
+                            c[r] = __ldg(B.col + q);
+                            v[r] = S.s_a[kk] * ldv<VT>(B.val, q);
+                        }
+                    }
+                    #pragma unroll
+                    for (int r = 0; r < 4; ++r)
+                        if (c[r] >= 0) {
+                            const uint32_t d = (uint32_t)(c[r] - lo);
+                            const uint32_t wv = S.bm[d >> 5];
+                            const int rank = S.pref[d >> 5] + __popc(wv & ((1u << (d & 31)) - 1u));
+                            atomicAdd(&S.vals[rank], v[r]);
+                        }
+                }
+                if (!single) __syncthreads();
+            }
+            __syncthreads();
+            // ---- emission: columns from the bitmap, values from the compact array ----
+            const int64_t base = crow + R.off;
+            for (int wd = tid; wd < nwords; wd += HEAVY_THREADS) {
+                uint32_t bits = S.bm[wd];
+                if (!bits) continue;
+                int o = S.pref[wd];
+                S.bm[wd] = 0u;
+                while (bits) {
+                    const int b = __ffs(bits) - 1;
+                    bits &= bits - 1;
+                    C_col[base + o++] = (int32_t)(lo + wd * 32 + b);
+                }
+            }
+            for (int e = tid; e < R.cnt; e += HEAVY_THREADS) {
+                C_val[base + e] = (VT)S.vals[e];
+                S.vals[e] = 0.0;
+            }
+            __syncthreads();
+        }
+    }
+}
+
+cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, int64_t nheavy, int64_t rb,
+                             const int64_t* range_off, const int32_t* nranges, const RangeRec* ranges,
+                             const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
+                             void* C_val, unsigned long long* counter, int4* gscr, int64_t amax, cudaStream_t s) {
+    if (nheavy <= 0) return cudaSuccess;
+    const int smem = (int)sizeof(HeavySmem);
+    cudaError_t e = cudaMemsetAsync(counter, 0, sizeof(unsigned long long), s);
+    if (e != cudaSuccess) return e;
+    const int grid = (int)(nheavy < 148 ? nheavy : 148);
+    if (A.dt == 0) {
+        if ((e = cudaFuncSetAttribute(k_num_heavy<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
+        SG_LAUNCH("k_num_heavy", s, (k_num_heavy<double><<<grid, HEAVY_THREADS, smem, s>>>(
+                                        A, B, heavy, nheavy, rb, range_off, nranges, ranges, long_id, tp, T, C_rp, C_col,
+                                        (double*)C_val, counter, gscr, amax)));
+    } else {
+        if ((e = cudaFuncSetAttribute(k_num_heavy<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
+        SG_LAUNCH("k_num_heavy", s, (k_num_heavy<float><<<grid, HEAVY_THREADS, smem, s>>>(
+                                        A, B, heavy, nheavy, rb, range_off, nranges, ranges, long_id, tp, T, C_rp, C_col,
+                                        (float*)C_val, counter, gscr, amax)));
+    }
+    return cudaGetLastError();
+}
+
+int heavy_kc() { return KC; }
+
+}  // namespace sg
+
+namespace sg {
+__global__ void k_max_a(Mat A, const int32_t* __restrict__ list, int64_t cnt, int64_t rb, unsigned long long* out) {
+    unsigned long long m = 0;
+    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < cnt; j += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = rb + list[j];
+        const unsigned long long a = (unsigned long long)(A.rp[r + 1] - A.rp[r]);
+        m = a > m ? a : m;
+    }
+    #pragma unroll
+    for (int o = 16; o; o >>= 1) { unsigned long long y = __shfl_xor_sync(FULL, m, o); m = y > m ? y : m; }
+    if ((threadIdx.x & 31) == 0 && m) atomicMax(out, m);
+}
+
+cudaError_t launch_max_a(const Mat& A, const int32_t* list, int64_t cnt, int64_t rb, unsigned long long* out,
+                         cudaStream_t s) {
+    if (cnt <= 0) return cudaSuccess;
+    SG_LAUNCH("k_max_a", s, (k_max_a<<<grid_for(cnt, 1024, 148 * 4), 256, 0, s>>>(A, list, cnt, rb, out)));
+    return cudaGetLastError();
+}
+}  // namespace sg

@@ -8,6 +8,15 @@
 
 namespace sg {
 
+// ---- launch accounting / optional per-launch CUDA-event timing (sg_profile.cu) ------------------
+struct Prof {
+    Prof(const char* name, cudaStream_t s);
+    ~Prof();
+    cudaStream_t s;
+    long long idx;
+};
+#define SG_LAUNCH(name, stream, ...) do { ::sg::Prof _sg_prof(name, stream); __VA_ARGS__; } while (0)
+
 // ---- routing classes and bins (heavy iff w > t; R13: w == t light) --
 constexpr int NBIN_LIGHT = 13;   // light bin b holds 2^(b-1) < w <= 2^b  (b = 0: w == 1); U_b = 2^b
 constexpr int BIN_EMPTY = 13;    // w == 0 (R7)
@@ -16,10 +25,7 @@ constexpr int NBINS = 15;
 
 // ---- heavy path geometry ---------------------------------------------------
 constexpr int TW = 8192;          // column tile width of the heavy path (tile = unit of range planning)
-constexpr int CAPU = 4096;        // max entries of a hashed (multi-tile) heavy range
-constexpr int PH = 12288;         // heavy accumulator slots per CTA (int32 key + fp64 value)
-constexpr int HH = PH - CAPU;     // home range of the order-preserving hash (overflow room = CAPU)
-constexpr int LONG_ROW = 32;      // B rows longer than this get per-tile pointers
+constexpr int LONG_ROW = 8;       // B rows longer than this get per-tile pointers
 constexpr int WIN = 1 << 20;      // heavy symbolic bitmap window (columns); 128 KB of smem
 constexpr int HEAVY_THREADS = 1024;
 
@@ -62,24 +68,28 @@ cudaError_t launch_bin_count(const int64_t* w, int64_t nr, int64_t thr, int64_t*
                              cudaStream_t s);
 cudaError_t launch_bin_scatter(const int64_t* w, int64_t nr, int64_t thr, int64_t* d_cursor /*NBINS*/,
                                int32_t* lists, cudaStream_t s);
-// symbolic light: bin b, rows = lists entries (local index j); global row = rowmap ? rowmap[j] : rb + j
+// light path (sg_light.cu): bin b, rows = list entries (local index li); global row = rowmap ? rowmap[li] : rb + li
 cudaError_t launch_sym_light(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt,
-                             const int64_t* rowmap, int64_t rb, int64_t* u, cudaStream_t s);
-cudaError_t launch_sym_heavy(const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, const int64_t* rowmap,
-                             int64_t rb, const int64_t* w, int64_t* u, const int64_t* range_off, RangeRec* ranges,
-                             cudaStream_t s);
-cudaError_t launch_range_bounds(const int32_t* heavy_list, int64_t nheavy, const int64_t* w, int64_t p,
-                                int64_t* bounds, cudaStream_t s);
-cudaError_t launch_fill_ranges_unused(RangeRec* ranges, int64_t n, cudaStream_t s);
-// B tile pointers for long rows
+                             const int64_t* rowmap, int64_t rb, int64_t* u, int2* span, cudaStream_t s);
+cudaError_t launch_num_light(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, int64_t rb,
+                             const int2* span, const int64_t* C_rp, int32_t* C_col, void* C_val, cudaStream_t s);
+// heavy path (sg_heavy.cu)
 cudaError_t launch_long_rows(const Mat& B, int32_t* long_id, int64_t* d_nlong, cudaStream_t s);
 cudaError_t launch_build_tp(const Mat& B, const int32_t* long_id, int T, uint32_t* tp, cudaStream_t s);
-// numeric
-cudaError_t launch_num_light(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, int64_t rb,
-                             const int64_t* C_rp, int32_t* C_col, void* C_val, cudaStream_t s);
-cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const RangeRec* ranges, int64_t nslots, int64_t rb,
-                             const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp,
-                             int32_t* C_col, void* C_val, unsigned long long* d_counter, cudaStream_t s);
+cudaError_t launch_heavy_order(const int32_t* heavy, int64_t nh, const int64_t* w, unsigned int* hist128,
+                               int32_t* out, cudaStream_t s);
+cudaError_t launch_range_bounds(const int32_t* heavy_list, int64_t nheavy, const int64_t* w, int64_t p,
+                                int64_t* bounds, cudaStream_t s);
+cudaError_t launch_sym_heavy(const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, const int64_t* rowmap,
+                             int64_t rb, int64_t* u, const int64_t* range_off, RangeRec* ranges, int32_t* nranges,
+                             unsigned long long* counter, cudaStream_t s);
+cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, int64_t nheavy, int64_t rb,
+                             const int64_t* range_off, const int32_t* nranges, const RangeRec* ranges,
+                             const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
+                             void* C_val, unsigned long long* counter, int4* gscr, int64_t amax, cudaStream_t s);
+cudaError_t launch_max_a(const Mat& A, const int32_t* list, int64_t cnt, int64_t rb, unsigned long long* out,
+                         cudaStream_t s);
+int heavy_kc();
 // threshold: cost histogram over rows then argmin over t in [0, cap_L]
 struct ThrResult { long long thr, Jmin, base, W_L, W_all, nonempty; };
 cudaError_t launch_cost_hist(const CostModelD& cm, const int64_t* w, const int64_t* a, const int64_t* u, int64_t nr,
