@@ -1,6 +1,7 @@
 // sg_api.cu — the C ABI (include/sg.h): validation, plans/workspace, orchestration of the kernels.
 #include "sg_internal.cuh"
 #include <cstdlib>
+#include <cstdio>
 #include <cstring>
 #include <cmath>
 #include <vector>
@@ -520,9 +521,27 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
     for (int k = 0; k < NBIN_LIGHT; ++k)
         CKP(pl, launch_num_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], pl->rb, pl->span, pl->C_rp,
                                  C_col, C_val, s));
-    if (pl->nheavy > 0)
+    if (pl->nheavy > 0) {
+        // SG_DEBUG_HEAVY=1: per-phase cycle counters of the heavy numeric kernel, printed to stderr
+        const char* dbe = getenv("SG_DEBUG_HEAVY");
+        unsigned long long* dbg = nullptr;
+        if (dbe && dbe[0] == '1') {
+            CKP(pl, cudaMallocAsync((void**)&dbg, 8 * sizeof(unsigned long long), s));
+            CKP(pl, cudaMemsetAsync(dbg, 0, 8 * sizeof(unsigned long long), s));
+        }
         CKP(pl, launch_num_heavy(a, b, pl->heavy, pl->nheavy, pl->rb, pl->range_off, pl->nranges, pl->ranges,
-                                 pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter, pl->gscr, pl->amax, s));
+                                 pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter, pl->gscr, pl->amax, s,
+                                 dbg));
+        if (dbg) {
+            unsigned long long h[8];
+            CKP(pl, cudaMemcpyAsync(h, dbg, sizeof(h), cudaMemcpyDeviceToHost, s));
+            CKP(pl, cudaStreamSynchronize(s));
+            cudaFreeAsync(dbg, s);
+            fprintf(stderr, "[sg heavy] Mcycles (sum over CTAs): fetch %.1f init %.1f seg+compact %.1f pass1 %.1f "
+                            "prefix %.1f pass2 %.1f emit %.1f | ranges %llu\n",
+                    h[0] / 1e6, h[1] / 1e6, h[2] / 1e6, h[3] / 1e6, h[4] / 1e6, h[5] / 1e6, h[6] / 1e6, h[7]);
+        }
+    }
     return SG_OK;
 }
 

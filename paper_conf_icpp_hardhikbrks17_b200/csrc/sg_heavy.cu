@@ -60,6 +60,131 @@ __device__ __forceinline__ int find_k(const int* off, int nk, int j) {
     return lo;
 }
 
+__device__ __forceinline__ long long block_scan1024_ll(long long v, long long* total, long long* ws) {
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    long long inc = warp_incl_scan(v);
+    if (lane == 31) ws[wid] = inc;
+    __syncthreads();
+    if (wid == 0) {
+        long long x = ws[lane];
+        long long xi = warp_incl_scan(x);
+        ws[lane] = xi - x;
+        if (lane == 31) ws[32] = xi;
+    }
+    __syncthreads();
+    long long r = ws[wid] + inc - v;
+    *total = ws[32];
+    __syncthreads();
+    return r;
+}
+
+// One chunk of k entries (one per thread): pack the entries with len > 0, in order, into
+// s_beg / s_off (exclusive prefix of len) / s_a; returns the chunk's product count, *nk = packed.
+template <class BEG>
+__device__ __forceinline__ int chunk_compact(int len, BEG beg, double a, BEG* s_beg, int* s_off, double* s_a, int* nk,
+                                             long long* wsll) {
+    long long tot;
+    const long long ex = block_scan1024_ll(((long long)len << 16) | (len > 0 ? 1 : 0), &tot, wsll);
+    if (len > 0) {
+        const int ci = (int)(ex & 0xFFFF);
+        s_beg[ci] = beg;
+        s_off[ci] = (int)(ex >> 16);
+        if (s_a) s_a[ci] = a;
+    }
+    *nk = (int)(tot & 0xFFFF);
+    __syncthreads();
+    return (int)(tot >> 16);
+}
+
+// Products [0, tot) of a packed chunk, split into one contiguous slice per warp. Within a slice a
+// batch of 32 consecutive products lies in at most 32 consecutive packed entries (each has len >= 1),
+// so every lane finds its entry with a 5-step shuffle search; the next batch's gathers are issued
+// before the current batch is consumed (two batches in flight per warp).
+template <bool VAL, class VT, class BEG, class F>
+__device__ __forceinline__ void warp_slice(const BEG* s_beg, const int* s_off, const double* s_a, int nk, int tot,
+                                           const Mat& B, F&& f) {
+    constexpr int NW = HEAVY_THREADS / 32;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int per = (((tot + NW - 1) / NW) + 31) & ~31;
+    const int j_lo = wid * per, j_hi = min(tot, j_lo + per);
+    if (j_lo >= j_hi) return;
+    int i0 = find_k(s_off, nk, j_lo);
+    auto fetch = [&](int j0, int& c, double& v) {
+        // fast path: the whole batch lies inside entry i0 (long B segments: hub rows of B)
+        const int e0 = i0 + 1 < nk ? s_off[i0 + 1] : tot;
+        if (j0 + 31 < e0) {
+            const int j = j0 + lane;
+            c = -1;
+            v = 0.0;
+            if (j < j_hi) {
+                const int64_t q = (int64_t)s_beg[i0] + (j - s_off[i0]);
+                c = __ldg(B.col + q);
+                if (VAL) v = s_a[i0] * ldv<VT>(B.val, q);
+            }
+            return;
+        }
+        const int ii = i0 + lane;
+        const int o = ii < nk ? s_off[ii] : INT_MAX;
+        const int j = j0 + lane;
+        int s = 0;
+        #pragma unroll
+        for (int b = 16; b; b >>= 1) {
+            const int ob = __shfl_sync(FULL, o, s + b);
+            if (ob <= j) s += b;
+        }
+        const int kk = i0 + s;
+        const int os = __shfl_sync(FULL, o, s);
+        c = -1;
+        v = 0.0;
+        if (j < j_hi) {
+            const int64_t q = (int64_t)s_beg[kk] + (j - os);
+            c = __ldg(B.col + q);
+            if (VAL) v = s_a[kk] * ldv<VT>(B.val, q);
+        }
+        i0 = __shfl_sync(FULL, kk, 31);
+    };
+    // four batches in flight: fetch(j + 96) is issued before batch j is consumed
+    int c0, c1, c2, c3;
+    double v0, v1, v2, v3;
+    fetch(j_lo, c0, v0);
+    fetch(j_lo + 32, c1, v1);
+    fetch(j_lo + 64, c2, v2);
+    for (int j0 = j_lo; j0 < j_hi; j0 += 128) {
+        fetch(j0 + 96, c3, v3);
+        f(c0, v0);  // f is called by every lane (c < 0: no product) so it may use warp collectives
+        if (j0 + 128 >= j_hi) { f(c1, v1); f(c2, v2); f(c3, v3); break; }
+        fetch(j0 + 128, c0, v0);
+        f(c1, v1);
+        fetch(j0 + 160, c1, v1);
+        f(c2, v2);
+        fetch(j0 + 192, c2, v2);
+        f(c3, v3);
+    }
+}
+
+// Warp-uniform bitmap insert of bit (d & 31) of word (d >> 5) (d < 0: nothing). Columns of a
+// B segment are sorted, so lanes hitting the same word are adjacent: when any adjacent pair
+// collides, runs of equal words are OR-reduced (segmented doubling) and only the run head issues
+// the shared-memory atomic, instead of up to 32 serialised same-address atomics.
+__device__ __forceinline__ void warp_set_bit(uint32_t* bm, int d) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t word = d >= 0 ? ((uint32_t)d >> 5) : (0x80000000u | lane);
+    uint32_t acc = d >= 0 ? (1u << (d & 31)) : 0u;
+    const uint32_t prev = __shfl_up_sync(FULL, word, 1);
+    const bool head = lane == 0 || prev != word;
+    const unsigned heads = __ballot_sync(FULL, head);
+    if (heads != FULL) {
+        const unsigned above = heads & (lane == 31 ? 0u : (~0u << (lane + 1)));
+        const int segend = above ? __ffs(above) - 1 : 32;
+        #pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_down_sync(FULL, acc, o);
+            if (lane + o < segend) acc |= y;
+        }
+    }
+    if (head && d >= 0) atomicOr(&bm[word], acc);
+}
+
 // ------------------------------------------------------------------------------------------------
 // B tile pointers: for B rows longer than LONG_ROW, tp[id][t] = #entries with col < t*TW
 // ------------------------------------------------------------------------------------------------
@@ -83,10 +208,22 @@ __global__ void k_build_tp(Mat B, const int32_t* __restrict__ long_id, int T, ui
     for (int64_t k = warp; k < B.nrows; k += nw) {
         int id = long_id[k];
         if (id < 0) continue;
-        int64_t q0 = B.rp[k], q1 = B.rp[k + 1];
+        const int64_t q0 = B.rp[k], q1 = B.rp[k + 1];
+        const int len = (int)(q1 - q0);
         uint32_t* row = tp + (int64_t)id * (T + 1);
-        for (int t = lane; t <= T; t += 32)
-            row[t] = (uint32_t)(lower_bound_col(B.col, q0, q1, (int64_t)t * TW) - q0);
+        // entry q with tile t_q starts every tile in (t_{q-1}, t_q]: one pass over the entries
+        int tprev_chunk = -1;
+        for (int b0 = 0; b0 < len; b0 += 32) {
+            const int q = b0 + lane;
+            const int tq = q < len ? (int)(__ldg(B.col + q0 + q) / TW) : T + 1;
+            int tp_prev = __shfl_up_sync(FULL, tq, 1);
+            if (lane == 0) tp_prev = tprev_chunk;
+            if (q < len)
+                for (int t = tp_prev + 1; t <= tq; ++t) row[t] = (uint32_t)q;
+            tprev_chunk = __shfl_sync(FULL, tq, 31);
+        }
+        const int tlast = len > 0 ? (int)(__ldg(B.col + q1 - 1) / TW) : -1;
+        for (int t = tlast + 1 + lane; t <= T; t += 32) row[t] = (uint32_t)len;
     }
 }
 
@@ -174,7 +311,7 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_sym_heavy(Mat A, Mat B, co
     __shared__ int tcnt[WIN / TW];
     __shared__ int Ps[WIN / TW];
     __shared__ unsigned char st[WIN / TW];
-    __shared__ int ws[33];
+    __shared__ long long wsll[33];
     __shared__ long long s_j;
     __shared__ int s_nr, s_u;
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5, nwarps = HEAVY_THREADS / 32;
@@ -208,30 +345,11 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_sym_heavy(Mat A, Mat B, co
                     beg = q0;
                     len = (int)(q1 - q0);
                 }
-                int tot;
-                const int off = block_scan1024(len, &tot, ws);  // (its barriers also order the bitmap clear)
-                s_beg[tid] = beg;
-                s_off[tid] = off;
-                __syncthreads();
-                const int nk = (int)min((int64_t)KC, s1 - c0);
-                for (int jb = tid; jb < tot; jb += HEAVY_THREADS * 4) {
-                    int c[4];
-                    #pragma unroll
-                    for (int r = 0; r < 4; ++r) {
-                        const int jj = jb + r * HEAVY_THREADS;
-                        c[r] = -1;
-                        if (jj < tot) {
-                            const int kk = find_k(s_off, nk, jj);
-                            c[r] = __ldg(B.col + s_beg[kk] + (jj - s_off[kk]));
-                        }
-                    }
-                    #pragma unroll
-                    for (int r = 0; r < 4; ++r)
-                        if (c[r] >= 0) {
-                            const uint32_t d = (uint32_t)(c[r] - wlo);
-                            atomicOr(&bm[d >> 5], 1u << (d & 31));
-                        }
-                }
+                int nk;
+                const int tot = chunk_compact<int64_t>(len, beg, 0.0, s_beg, s_off, nullptr, &nk, wsll);
+                warp_slice<false, double, int64_t>(s_beg, s_off, nullptr, nk, tot, B, [&](int32_t c, double) {
+                    warp_set_bit(bm, c >= 0 ? (int)(c - wlo) : -1);
+                });
                 __syncthreads();
             }
             // per-tile popcounts
@@ -322,31 +440,48 @@ cudaError_t launch_sym_heavy(const Mat& A, const Mat& B, const int32_t* list, in
 // ------------------------------------------------------------------------------------------------
 struct HeavySmem {
     uint32_t bm[RW_WORDS];       // 32 KB  range bitmap
-    double vals[RCAP];           // 128 KB compact accumulator (by rank)
+    double vals[RCAP];           // 128 KB compact accumulator (by rank); int32 column staging at emission
     uint16_t pref[RW_WORDS];     // 16 KB  rank prefix per bitmap word
-    int32_t s_beg[KC];           // segment begin (B position) of chunk entry
-    int32_t s_off[KC];           // exclusive prefix of segment lengths
-    double s_a[KC];              // a_ik
-    int32_t c_cur[KC];           // single-chunk rows: cursor (B position)
-    int32_t c_nextc[KC];         //                    column at the cursor (INT_MAX: exhausted)
-    int32_t c_end[KC];           //                    end of the B row
-    int32_t c_q0[KC];            //                    start of the B row
-    int32_t c_lid[KC];           //                    long-row id or -1
+    int32_t s_beg[KC];           // packed chunk entries: segment begin (B position)
+    int32_t s_off[KC];           //                       exclusive prefix of segment lengths
+    double s_a[KC];              //                       a_ik
+    int32_t c_cur[KC];           // single-chunk rows, per k: cursor (B position)
+    int32_t c_end[KC];           //   end of the B row
+    int32_t c_q0[KC];            //   start of the B row
+    int32_t c_lid[KC];           //   long-row id or -1 (short row: <= LONG_ROW entries)
+    double c_a[KC];              //   a_ik
+    long long wsll[33];
     int ws[33];
 };
+
+// Segment of one k entry for tiles [.., t1) starting at its cursor: long B rows read the tile
+// pointer (prefetched `tpv`), short rows (<= LONG_ROW entries) count their entries below hi with
+// independent loads. Returns the new cursor.
+__device__ __forceinline__ int seg_end(const Mat& B, int cur, int e1, int q0, bool is_long, uint32_t tpv, int64_t hi) {
+    if (is_long) return q0 + (int)tpv;
+    int n = 0;
+    #pragma unroll
+    for (int q = 0; q < LONG_ROW; ++q)
+        if (cur + q < e1 && __ldg(B.col + cur + q) < hi) ++n;
+    return cur + n;
+}
 
 template <class VT>
 __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_num_heavy(
     Mat A, Mat B, const int32_t* __restrict__ heavy, int64_t nheavy, int64_t rb, const int64_t* __restrict__ range_off,
     const int32_t* __restrict__ nranges, const RangeRec* __restrict__ ranges, const int32_t* __restrict__ long_id,
     const uint32_t* __restrict__ tp, int T, const int64_t* __restrict__ C_rp, int32_t* __restrict__ C_col,
-    VT* __restrict__ C_val, unsigned long long* counter, int4* __restrict__ gscr, int64_t amax) {
+    VT* __restrict__ C_val, unsigned long long* counter, int4* __restrict__ gscr, int64_t amax,
+    unsigned long long* __restrict__ dbg) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
+    unsigned long long tph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    long long t_last = clock64();
+    auto mark = [&](int k) { if (dbg && threadIdx.x == 0) { long long t = clock64(); tph[k] += t - t_last; t_last = t; } };
     HeavySmem& S = *reinterpret_cast<HeavySmem*>(smem_raw);
     __shared__ long long s_j;
-    const int tid = threadIdx.x;
+    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
     const int64_t p = B.ncols;
-    int4* gs = gscr + (int64_t)blockIdx.x * amax;  // multi-chunk rows: per-k (cur, nextc, beg, len)
+    int4* gs = gscr + (int64_t)blockIdx.x * amax;  // multi-chunk rows: per-k (cur, -, beg, len)
     for (int q = tid; q < RW_WORDS; q += HEAVY_THREADS) S.bm[q] = 0u;
     for (int q = tid; q < RCAP; q += HEAVY_THREADS) S.vals[q] = 0.0;
     while (true) {
@@ -355,171 +490,163 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_num_heavy(
         const int64_t h = s_j;
         __syncthreads();
         if (h >= nheavy) break;
+        mark(0);
         const int64_t li = heavy[h];
         const int64_t row = rb + li;
         const int64_t s0 = __ldg(A.rp + row), s1 = __ldg(A.rp + row + 1);
         const int na = (int)(s1 - s0);
         const bool single = na <= KC;
-        // per-k cursor state
-        for (int i = tid; i < na; i += HEAVY_THREADS) {
-            const int k = __ldg(A.col + s0 + i);
-            const int32_t q0 = (int32_t)__ldg(B.rp + k), q1 = (int32_t)__ldg(B.rp + k + 1);
-            const int32_t nc = q0 < q1 ? __ldg(B.col + q0) : INT_MAX;
-            if (single) {
-                S.c_cur[i] = q0; S.c_nextc[i] = nc; S.c_end[i] = q1; S.c_q0[i] = q0;
-                S.c_lid[i] = q1 - q0 > LONG_ROW ? __ldg(long_id + k) : -1;
-                S.s_a[i] = ldv<VT>(A.val, s0 + i);
-            } else {
-                gs[i] = make_int4(q0, nc, 0, 0);
-            }
-        }
-        __syncthreads();
         const int nr = nranges[h];
         const RangeRec* rr = ranges + range_off[h];
         const int64_t crow = C_rp[li];
+        // per-k cursor state; single-chunk rows keep it in shared memory, one k per thread
+        uint32_t tpv = 0;  // prefetched tile pointer of this thread's k for the next range
+        for (int i = tid; i < na; i += HEAVY_THREADS) {
+            const int k = __ldg(A.col + s0 + i);
+            const int32_t q0 = (int32_t)__ldg(B.rp + k), q1 = (int32_t)__ldg(B.rp + k + 1);
+            if (single) {
+                const int lid = q1 - q0 > LONG_ROW ? __ldg(long_id + k) : -1;
+                S.c_cur[i] = q0; S.c_end[i] = q1; S.c_q0[i] = q0; S.c_lid[i] = lid;
+                S.c_a[i] = ldv<VT>(A.val, s0 + i);
+                if (lid >= 0 && nr > 0) tpv = __ldg(tp + (int64_t)lid * (T + 1) + rr[0].t1);
+            } else {
+                gs[i] = make_int4(q0, 0, 0, 0);
+            }
+        }
+        __syncthreads();
+        mark(1);
+        if (dbg && tid == 0) tph[7] += nr;
         for (int ri = 0; ri < nr; ++ri) {
             const RangeRec R = rr[ri];
             const int64_t lo = (int64_t)R.t0 * TW, hi = min(p, (int64_t)R.t1 * TW);
             const int nwords = (int)((hi - lo + 31) / 32);
-            int tot = 0;
+            int tot1 = 0, nk1 = 0;
             // ---- pass 1: segments (advance cursors) + bitmap of the range ----
             for (int c0 = 0; c0 < na; c0 += KC) {
                 const int i = c0 + tid;
                 int len = 0, beg = 0;
+                double a = 0.0;
                 if (i < na) {
                     if (single) {
-                        const int nc = S.c_nextc[i];
-                        if (nc < hi) {
-                            const int cur = S.c_cur[i], e1 = S.c_end[i], lid = S.c_lid[i];
-                            int end;
-                            if (lid >= 0) end = S.c_q0[i] + (int)__ldg(tp + (int64_t)lid * (T + 1) + R.t1);
-                            else { end = cur + 1; while (end < e1 && __ldg(B.col + end) < hi) ++end; }
-                            beg = cur; len = end - cur;
-                            S.c_cur[i] = end;
-                            S.c_nextc[i] = end < e1 ? __ldg(B.col + end) : INT_MAX;
-                        }
+                        const int cur = S.c_cur[i], lid = S.c_lid[i];
+                        const int end = seg_end(B, cur, S.c_end[i], S.c_q0[i], lid >= 0, tpv, hi);
+                        beg = cur; len = end - cur; a = S.c_a[i];
+                        S.c_cur[i] = end;
+                        // prefetch the next range's tile pointer (its latency hides behind this range)
+                        if (lid >= 0 && ri + 1 < nr) tpv = __ldg(tp + (int64_t)lid * (T + 1) + rr[ri + 1].t1);
                     } else {
                         const int4 g = gs[i];
-                        if (g.y < hi) {
-                            const int k = __ldg(A.col + s0 + i);
-                            const int32_t q0 = (int32_t)__ldg(B.rp + k), e1 = (int32_t)__ldg(B.rp + k + 1);
-                            int end;
-                            if (e1 - q0 > LONG_ROW) end = q0 + (int)__ldg(tp + (int64_t)__ldg(long_id + k) * (T + 1) + R.t1);
-                            else { end = g.x + 1; while (end < e1 && __ldg(B.col + end) < hi) ++end; }
-                            beg = g.x; len = end - g.x;
-                            gs[i] = make_int4(end, end < e1 ? __ldg(B.col + end) : INT_MAX, beg, len);
-                        } else {
-                            gs[i] = make_int4(g.x, g.y, g.x, 0);
-                        }
+                        const int k = __ldg(A.col + s0 + i);
+                        const int32_t q0 = (int32_t)__ldg(B.rp + k), e1 = (int32_t)__ldg(B.rp + k + 1);
+                        const bool lng = e1 - q0 > LONG_ROW;
+                        const uint32_t tv = lng ? __ldg(tp + (int64_t)__ldg(long_id + k) * (T + 1) + R.t1) : 0u;
+                        const int end = seg_end(B, g.x, e1, q0, lng, tv, hi);
+                        beg = g.x; len = end - g.x;
+                        gs[i] = make_int4(end, 0, beg, len);
                     }
                 }
-                int ctot;
-                const int off = block_scan1024(len, &ctot, S.ws);
-                S.s_beg[tid] = beg;
-                S.s_off[tid] = off;
-                __syncthreads();
-                const int nk = min(KC, na - c0);
-                for (int jb = tid; jb < ctot; jb += HEAVY_THREADS * 4) {
-                    int c[4];
-                    #pragma unroll
-                    for (int r = 0; r < 4; ++r) {
-                        const int jj = jb + r * HEAVY_THREADS;
-                        c[r] = -1;
-                        if (jj < ctot) {
-                            const int kk = find_k(S.s_off, nk, jj);
-                            c[r] = __ldg(B.col + S.s_beg[kk] + (jj - S.s_off[kk]));
-                        }
-                    }
-                    #pragma unroll
-                    for (int r = 0; r < 4; ++r)
-                        if (c[r] >= 0) {
-                            const uint32_t d = (uint32_t)(c[r] - lo);
-                            atomicOr(&S.bm[d >> 5], 1u << (d & 31));
-                        }
-                }
-                tot += ctot;
+                int nk;
+                const int ctot = chunk_compact<int32_t>(len, beg, a, S.s_beg, S.s_off, S.s_a, &nk, S.wsll);
+                mark(2);
+                warp_slice<false, VT, int32_t>(S.s_beg, S.s_off, nullptr, nk, ctot, B, [&](int32_t c, double) {
+                    warp_set_bit(S.bm, c >= 0 ? (int)(c - lo) : -1);
+                });
+                tot1 = ctot;
+                nk1 = nk;
                 if (!single) __syncthreads();
             }
             __syncthreads();
-            // ---- rank prefix over the range's words (8 consecutive words per thread) ----
+            mark(3);
+            // ---- rank prefix over the range's words: warp w owns words [256w, 256w+256) in a
+            // lane-strided (bank-conflict-free) layout; 8 warp scans + one scan over the warps ----
             {
-                const int w0 = tid * 8;
-                int cw[8], loc = 0;
+                const int wb = wid * 256;
+                int x[8], inc[8], rowbase[8], acc = 0;
                 #pragma unroll
-                for (int q = 0; q < 8; ++q) { cw[q] = w0 + q < nwords ? __popc(S.bm[w0 + q]) : 0; loc += cw[q]; }
-                int t2;
-                int pre = block_scan1024(loc, &t2, S.ws);
+                for (int q = 0; q < 8; ++q) {
+                    const int wd = wb + 32 * q + lane;
+                    x[q] = wd < nwords ? __popc(S.bm[wd]) : 0;
+                    inc[q] = warp_incl_scan(x[q]);
+                    rowbase[q] = acc;
+                    acc += __shfl_sync(FULL, inc[q], 31);
+                }
+                if (lane == 0) S.ws[wid] = acc;
+                __syncthreads();
+                if (wid == 0) {
+                    const int y = S.ws[lane];
+                    const int yi = warp_incl_scan(y);
+                    S.ws[lane] = yi - y;
+                }
+                __syncthreads();
+                const int wpre = S.ws[wid];
                 #pragma unroll
-                for (int q = 0; q < 8; ++q) { if (w0 + q < nwords) S.pref[w0 + q] = (uint16_t)pre; pre += cw[q]; }
+                for (int q = 0; q < 8; ++q) {
+                    const int wd = wb + 32 * q + lane;
+                    if (wd < nwords) S.pref[wd] = (uint16_t)(wpre + rowbase[q] + inc[q] - x[q]);
+                }
             }
             __syncthreads();
+            mark(4);
             // ---- pass 2: accumulate into the compact array at rank(c) ----
-            for (int c0 = 0; c0 < na; c0 += KC) {
-                const int nk = min(KC, na - c0);
-                int ctot;
-                if (single) {
-                    ctot = tot;  // segments of pass 1 are still in S.s_beg / S.s_off
-                } else {
+            auto acc = [&](int32_t c, double v) {
+                if (c < 0) return;
+                const uint32_t d = (uint32_t)(c - lo);
+                const uint32_t wv = S.bm[d >> 5];
+                const int rank = S.pref[d >> 5] + __popc(wv & ((1u << (d & 31)) - 1u));
+                atomicAdd(&S.vals[rank], v);
+            };
+            if (single) {
+                warp_slice<true, VT, int32_t>(S.s_beg, S.s_off, S.s_a, nk1, tot1, B, acc);  // pass-1 packing kept
+            } else {
+                for (int c0 = 0; c0 < na; c0 += KC) {
                     const int i = c0 + tid;
                     int len = 0, beg = 0;
-                    if (i < na) { const int4 g = gs[i]; beg = g.z; len = g.w; S.s_a[tid] = ldv<VT>(A.val, s0 + i); }
-                    const int off = block_scan1024(len, &ctot, S.ws);
-                    S.s_beg[tid] = beg;
-                    S.s_off[tid] = off;
+                    double a = 0.0;
+                    if (i < na) {
+                        const int4 g = gs[i];
+                        beg = g.z; len = g.w;
+                        if (len > 0) a = ldv<VT>(A.val, s0 + i);
+                    }
+                    int nk;
+                    const int ctot = chunk_compact<int32_t>(len, beg, a, S.s_beg, S.s_off, S.s_a, &nk, S.wsll);
+                    warp_slice<true, VT, int32_t>(S.s_beg, S.s_off, S.s_a, nk, ctot, B, acc);
                     __syncthreads();
                 }
-                for (int jb = tid; jb < ctot; jb += HEAVY_THREADS * 4) {
-                    int c[4];
-                    double v[4];
-                    #pragma unroll
-                    for (int r = 0; r < 4; ++r) {
-                        const int jj = jb + r * HEAVY_THREADS;
-                        c[r] = -1;
-                        if (jj < ctot) {
-                            const int kk = find_k(S.s_off, nk, jj);
-                            const int64_t q = S.s_beg[kk] + (jj - S.s_off[kk]);
-                            c[r] = __ldg(B.col + q);
-                            v[r] = S.s_a[kk] * ldv<VT>(B.val, q);
-                        }
-                    }
-                    #pragma unroll
-                    for (int r = 0; r < 4; ++r)
-                        if (c[r] >= 0) {
-                            const uint32_t d = (uint32_t)(c[r] - lo);
-                            const uint32_t wv = S.bm[d >> 5];
-                            const int rank = S.pref[d >> 5] + __popc(wv & ((1u << (d & 31)) - 1u));
-                            atomicAdd(&S.vals[rank], v[r]);
-                        }
-                }
-                if (!single) __syncthreads();
             }
             __syncthreads();
-            // ---- emission: columns from the bitmap, values from the compact array ----
+            mark(5);
+            // ---- emission: values by rank (coalesced); columns word by word, one lane per bit, so
+            // each non-empty word becomes one coalesced run of C.col ----
             const int64_t base = crow + R.off;
+            const int cnt = R.cnt;
+            for (int e = tid; e < cnt; e += HEAVY_THREADS) {
+                C_val[base + e] = (VT)S.vals[e];
+                S.vals[e] = 0.0;
+            }
             for (int wd = tid; wd < nwords; wd += HEAVY_THREADS) {
                 uint32_t bits = S.bm[wd];
                 if (!bits) continue;
-                int o = S.pref[wd];
+                int64_t o = base + S.pref[wd];
                 S.bm[wd] = 0u;
                 while (bits) {
                     const int b = __ffs(bits) - 1;
                     bits &= bits - 1;
-                    C_col[base + o++] = (int32_t)(lo + wd * 32 + b);
+                    C_col[o++] = (int32_t)(lo + wd * 32 + b);
                 }
             }
-            for (int e = tid; e < R.cnt; e += HEAVY_THREADS) {
-                C_val[base + e] = (VT)S.vals[e];
-                S.vals[e] = 0.0;
-            }
             __syncthreads();
+            mark(6);
         }
     }
+    if (dbg && threadIdx.x == 0)
+        for (int k = 0; k < 8; ++k) atomicAdd(&dbg[k], tph[k]);
 }
 
 cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, int64_t nheavy, int64_t rb,
                              const int64_t* range_off, const int32_t* nranges, const RangeRec* ranges,
                              const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
-                             void* C_val, unsigned long long* counter, int4* gscr, int64_t amax, cudaStream_t s) {
+                             void* C_val, unsigned long long* counter, int4* gscr, int64_t amax, cudaStream_t s,
+                             unsigned long long* dbg) {
     if (nheavy <= 0) return cudaSuccess;
     const int smem = (int)sizeof(HeavySmem);
     cudaError_t e = cudaMemsetAsync(counter, 0, sizeof(unsigned long long), s);
@@ -529,12 +656,12 @@ cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, i
         if ((e = cudaFuncSetAttribute(k_num_heavy<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
         SG_LAUNCH("k_num_heavy", s, (k_num_heavy<double><<<grid, HEAVY_THREADS, smem, s>>>(
                                         A, B, heavy, nheavy, rb, range_off, nranges, ranges, long_id, tp, T, C_rp, C_col,
-                                        (double*)C_val, counter, gscr, amax)));
+                                        (double*)C_val, counter, gscr, amax, dbg)));
     } else {
         if ((e = cudaFuncSetAttribute(k_num_heavy<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
         SG_LAUNCH("k_num_heavy", s, (k_num_heavy<float><<<grid, HEAVY_THREADS, smem, s>>>(
                                         A, B, heavy, nheavy, rb, range_off, nranges, ranges, long_id, tp, T, C_rp, C_col,
-                                        (float*)C_val, counter, gscr, amax)));
+                                        (float*)C_val, counter, gscr, amax, dbg)));
     }
     return cudaGetLastError();
 }

@@ -86,7 +86,8 @@ cudaError_t launch_sym_heavy(const Mat& A, const Mat& B, const int32_t* list, in
 cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, int64_t nheavy, int64_t rb,
                              const int64_t* range_off, const int32_t* nranges, const RangeRec* ranges,
                              const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
-                             void* C_val, unsigned long long* counter, int4* gscr, int64_t amax, cudaStream_t s);
+                             void* C_val, unsigned long long* counter, int4* gscr, int64_t amax, cudaStream_t s,
+                             unsigned long long* dbg = nullptr);
 cudaError_t launch_max_a(const Mat& A, const int32_t* list, int64_t cnt, int64_t rb, unsigned long long* out,
                          cudaStream_t s);
 int heavy_kc();
