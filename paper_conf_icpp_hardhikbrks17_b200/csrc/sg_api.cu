@@ -488,7 +488,7 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
         pl->tp = (uint32_t*)palloc(pl, 4 * (size_t)(pl->nlong > 0 ? pl->nlong : 1) * (size_t)(pl->T + 1));
         if (!pl->ranges || !pl->tp) return fail(SG_ERR_OOM);
         if (pl->amax > heavy_kc()) {
-            pl->gscr = (int4*)palloc(pl, sizeof(int4) * 148 * (size_t)pl->amax);
+            pl->gscr = (int4*)palloc(pl, sizeof(int4) * (size_t)heavy_grid() * (size_t)pl->amax);
             if (!pl->gscr) return fail(SG_ERR_OOM);
         }
         if (pl->nlong > 0) CKF(launch_build_tp(b, pl->long_id, pl->T, pl->tp, s));

@@ -17,11 +17,15 @@
 
 namespace sg {
 
-constexpr int KC = HEAVY_THREADS;  // k entries per chunk: one per thread
-constexpr int RW_TILES = 32;       // max tiles per numeric range -> 256K columns, 32 KB bitmap
-constexpr int RW_WORDS = RW_TILES * TW / 32;
-constexpr int RCAP = 16384;        // max entries per numeric range (fp64 accumulator 128 KB)
-constexpr int RHALF = RCAP / 2;    // range key granularity (a range = run of tiles with equal key)
+constexpr int SYM_T = HEAVY_THREADS;  // symbolic: one CTA of 1024 threads per SM (128 KB bitmap window)
+constexpr int NUM_T = 1024;           // numeric: threads per CTA
+constexpr int NUM_OCC = 1;            // numeric CTAs per SM (smem-bound)
+constexpr int KC = NUM_T;             // numeric k entries per chunk: one per thread
+constexpr int KCS = SYM_T;            // symbolic k entries per chunk
+constexpr int RW_TILES = NUM_T / 32;  // max tiles per numeric range (16 -> 128K columns, 16 KB bitmap)
+constexpr int RW_WORDS = RW_TILES * TW / 32;   // = 256 words per warp in the rank prefix
+constexpr int RCAP = 16384;           // max entries per numeric range (fp64 accumulator 128 KB)
+constexpr int RHALF = RCAP / 2;       // range key granularity (a range = run of tiles with equal key)
 
 __device__ __forceinline__ int64_t lower_bound_col(const int32_t* __restrict__ col, int64_t lo, int64_t hi, int64_t x) {
     while (lo < hi) {
@@ -32,13 +36,14 @@ __device__ __forceinline__ int64_t lower_bound_col(const int32_t* __restrict__ c
 }
 
 // exclusive scan of one int per thread over a 1024-thread block; *total for everyone
-__device__ __forceinline__ int block_scan1024(int v, int* total, int* ws) {
+template <int NT>
+__device__ __forceinline__ int block_scan(int v, int* total, int* ws) {
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     int inc = warp_incl_scan(v);
     if (lane == 31) ws[wid] = inc;
     __syncthreads();
     if (wid == 0) {
-        int x = ws[lane];
+        int x = lane < NT / 32 ? ws[lane] : 0;
         int xi = warp_incl_scan(x);
         ws[lane] = xi - x;
         if (lane == 31) ws[32] = xi;
@@ -60,13 +65,14 @@ __device__ __forceinline__ int find_k(const int* off, int nk, int j) {
     return lo;
 }
 
-__device__ __forceinline__ long long block_scan1024_ll(long long v, long long* total, long long* ws) {
+template <int NT>
+__device__ __forceinline__ long long block_scan_ll(long long v, long long* total, long long* ws) {
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     long long inc = warp_incl_scan(v);
     if (lane == 31) ws[wid] = inc;
     __syncthreads();
     if (wid == 0) {
-        long long x = ws[lane];
+        long long x = lane < NT / 32 ? ws[lane] : 0;
         long long xi = warp_incl_scan(x);
         ws[lane] = xi - x;
         if (lane == 31) ws[32] = xi;
@@ -80,11 +86,11 @@ __device__ __forceinline__ long long block_scan1024_ll(long long v, long long* t
 
 // One chunk of k entries (one per thread): pack the entries with len > 0, in order, into
 // s_beg / s_off (exclusive prefix of len) / s_a; returns the chunk's product count, *nk = packed.
-template <class BEG>
+template <int NT, class BEG>
 __device__ __forceinline__ int chunk_compact(int len, BEG beg, double a, BEG* s_beg, int* s_off, double* s_a, int* nk,
                                              long long* wsll) {
     long long tot;
-    const long long ex = block_scan1024_ll(((long long)len << 16) | (len > 0 ? 1 : 0), &tot, wsll);
+    const long long ex = block_scan_ll<NT>(((long long)len << 16) | (len > 0 ? 1 : 0), &tot, wsll);
     if (len > 0) {
         const int ci = (int)(ex & 0xFFFF);
         s_beg[ci] = beg;
@@ -100,10 +106,10 @@ __device__ __forceinline__ int chunk_compact(int len, BEG beg, double a, BEG* s_
 // batch of 32 consecutive products lies in at most 32 consecutive packed entries (each has len >= 1),
 // so every lane finds its entry with a 5-step shuffle search; the next batch's gathers are issued
 // before the current batch is consumed (two batches in flight per warp).
-template <bool VAL, class VT, class BEG, class F>
+template <int NT, bool VAL, class VT, class BEG, class F>
 __device__ __forceinline__ void warp_slice(const BEG* s_beg, const int* s_off, const double* s_a, int nk, int tot,
                                            const Mat& B, F&& f) {
-    constexpr int NW = HEAVY_THREADS / 32;
+    constexpr int NW = NT / 32;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const int per = (((tot + NW - 1) / NW) + 31) & ~31;
     const int j_lo = wid * per, j_hi = min(tot, j_lo + per);
@@ -306,8 +312,8 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_sym_heavy(Mat A, Mat B, co
                                                                  int32_t* __restrict__ nranges,
                                                                  unsigned long long* counter) {
     extern __shared__ uint32_t bm[];  // WIN/32 words
-    __shared__ int64_t s_beg[KC];
-    __shared__ int s_off[KC];
+    __shared__ int64_t s_beg[KCS];
+    __shared__ int s_off[KCS];
     __shared__ int tcnt[WIN / TW];
     __shared__ int Ps[WIN / TW];
     __shared__ unsigned char st[WIN / TW];
@@ -331,7 +337,7 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_sym_heavy(Mat A, Mat B, co
             const int64_t wlo = win * WIN, whi = min(p, wlo + WIN);
             const int nwords = (int)((whi - wlo + 31) / 32);
             for (int q = tid; q < nwords; q += HEAVY_THREADS) bm[q] = 0u;
-            for (int64_t c0 = s0; c0 < s1; c0 += KC) {
+            for (int64_t c0 = s0; c0 < s1; c0 += KCS) {
                 const int64_t i = c0 + tid;
                 int len = 0;
                 int64_t beg = 0;
@@ -346,9 +352,9 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_sym_heavy(Mat A, Mat B, co
                     len = (int)(q1 - q0);
                 }
                 int nk;
-                const int tot = chunk_compact<int64_t>(len, beg, 0.0, s_beg, s_off, nullptr, &nk, wsll);
-                warp_slice<false, double, int64_t>(s_beg, s_off, nullptr, nk, tot, B, [&](int32_t c, double) {
-                    warp_set_bit(bm, c >= 0 ? (int)(c - wlo) : -1);
+                const int tot = chunk_compact<SYM_T, int64_t>(len, beg, 0.0, s_beg, s_off, nullptr, &nk, wsll);
+                warp_slice<SYM_T, false, double, int64_t>(s_beg, s_off, nullptr, nk, tot, B, [&](int32_t c, double) {
+                    if (c >= 0) { const uint32_t d = (uint32_t)(c - wlo); atomicOr(&bm[d >> 5], 1u << (d & 31)); }
                 });
                 __syncthreads();
             }
@@ -467,7 +473,7 @@ __device__ __forceinline__ int seg_end(const Mat& B, int cur, int e1, int q0, bo
 }
 
 template <class VT>
-__global__ void __launch_bounds__(HEAVY_THREADS, 1) k_num_heavy(
+__global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
     Mat A, Mat B, const int32_t* __restrict__ heavy, int64_t nheavy, int64_t rb, const int64_t* __restrict__ range_off,
     const int32_t* __restrict__ nranges, const RangeRec* __restrict__ ranges, const int32_t* __restrict__ long_id,
     const uint32_t* __restrict__ tp, int T, const int64_t* __restrict__ C_rp, int32_t* __restrict__ C_col,
@@ -482,8 +488,8 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_num_heavy(
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
     const int64_t p = B.ncols;
     int4* gs = gscr + (int64_t)blockIdx.x * amax;  // multi-chunk rows: per-k (cur, -, beg, len)
-    for (int q = tid; q < RW_WORDS; q += HEAVY_THREADS) S.bm[q] = 0u;
-    for (int q = tid; q < RCAP; q += HEAVY_THREADS) S.vals[q] = 0.0;
+    for (int q = tid; q < RW_WORDS; q += NUM_T) S.bm[q] = 0u;
+    for (int q = tid; q < RCAP; q += NUM_T) S.vals[q] = 0.0;
     while (true) {
         if (tid == 0) s_j = (long long)atomicAdd(counter, 1ull);
         __syncthreads();
@@ -501,7 +507,7 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_num_heavy(
         const int64_t crow = C_rp[li];
         // per-k cursor state; single-chunk rows keep it in shared memory, one k per thread
         uint32_t tpv = 0;  // prefetched tile pointer of this thread's k for the next range
-        for (int i = tid; i < na; i += HEAVY_THREADS) {
+        for (int i = tid; i < na; i += NUM_T) {
             const int k = __ldg(A.col + s0 + i);
             const int32_t q0 = (int32_t)__ldg(B.rp + k), q1 = (int32_t)__ldg(B.rp + k + 1);
             if (single) {
@@ -546,10 +552,10 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_num_heavy(
                     }
                 }
                 int nk;
-                const int ctot = chunk_compact<int32_t>(len, beg, a, S.s_beg, S.s_off, S.s_a, &nk, S.wsll);
+                const int ctot = chunk_compact<NUM_T, int32_t>(len, beg, a, S.s_beg, S.s_off, S.s_a, &nk, S.wsll);
                 mark(2);
-                warp_slice<false, VT, int32_t>(S.s_beg, S.s_off, nullptr, nk, ctot, B, [&](int32_t c, double) {
-                    warp_set_bit(S.bm, c >= 0 ? (int)(c - lo) : -1);
+                warp_slice<NUM_T, false, VT, int32_t>(S.s_beg, S.s_off, nullptr, nk, ctot, B, [&](int32_t c, double) {
+                    if (c >= 0) { const uint32_t d = (uint32_t)(c - lo); atomicOr(&S.bm[d >> 5], 1u << (d & 31)); }
                 });
                 tot1 = ctot;
                 nk1 = nk;
@@ -573,7 +579,7 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_num_heavy(
                 if (lane == 0) S.ws[wid] = acc;
                 __syncthreads();
                 if (wid == 0) {
-                    const int y = S.ws[lane];
+                    const int y = lane < NUM_T / 32 ? S.ws[lane] : 0;
                     const int yi = warp_incl_scan(y);
                     S.ws[lane] = yi - y;
                 }
@@ -596,7 +602,7 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_num_heavy(
                 atomicAdd(&S.vals[rank], v);
             };
             if (single) {
-                warp_slice<true, VT, int32_t>(S.s_beg, S.s_off, S.s_a, nk1, tot1, B, acc);  // pass-1 packing kept
+                warp_slice<NUM_T, true, VT, int32_t>(S.s_beg, S.s_off, S.s_a, nk1, tot1, B, acc);  // pass-1 packing kept
             } else {
                 for (int c0 = 0; c0 < na; c0 += KC) {
                     const int i = c0 + tid;
@@ -608,8 +614,8 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_num_heavy(
                         if (len > 0) a = ldv<VT>(A.val, s0 + i);
                     }
                     int nk;
-                    const int ctot = chunk_compact<int32_t>(len, beg, a, S.s_beg, S.s_off, S.s_a, &nk, S.wsll);
-                    warp_slice<true, VT, int32_t>(S.s_beg, S.s_off, S.s_a, nk, ctot, B, acc);
+                    const int ctot = chunk_compact<NUM_T, int32_t>(len, beg, a, S.s_beg, S.s_off, S.s_a, &nk, S.wsll);
+                    warp_slice<NUM_T, true, VT, int32_t>(S.s_beg, S.s_off, S.s_a, nk, ctot, B, acc);
                     __syncthreads();
                 }
             }
@@ -619,11 +625,11 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_num_heavy(
             // each non-empty word becomes one coalesced run of C.col ----
             const int64_t base = crow + R.off;
             const int cnt = R.cnt;
-            for (int e = tid; e < cnt; e += HEAVY_THREADS) {
+            for (int e = tid; e < cnt; e += NUM_T) {
                 C_val[base + e] = (VT)S.vals[e];
                 S.vals[e] = 0.0;
             }
-            for (int wd = tid; wd < nwords; wd += HEAVY_THREADS) {
+            for (int wd = tid; wd < nwords; wd += NUM_T) {
                 uint32_t bits = S.bm[wd];
                 if (!bits) continue;
                 int64_t o = base + S.pref[wd];
@@ -651,15 +657,15 @@ cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, i
     const int smem = (int)sizeof(HeavySmem);
     cudaError_t e = cudaMemsetAsync(counter, 0, sizeof(unsigned long long), s);
     if (e != cudaSuccess) return e;
-    const int grid = (int)(nheavy < 148 ? nheavy : 148);
+    const int grid = (int)(nheavy < NUM_OCC * 148 ? nheavy : NUM_OCC * 148);
     if (A.dt == 0) {
         if ((e = cudaFuncSetAttribute(k_num_heavy<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
-        SG_LAUNCH("k_num_heavy", s, (k_num_heavy<double><<<grid, HEAVY_THREADS, smem, s>>>(
+        SG_LAUNCH("k_num_heavy", s, (k_num_heavy<double><<<grid, NUM_T, smem, s>>>(
                                         A, B, heavy, nheavy, rb, range_off, nranges, ranges, long_id, tp, T, C_rp, C_col,
                                         (double*)C_val, counter, gscr, amax, dbg)));
     } else {
         if ((e = cudaFuncSetAttribute(k_num_heavy<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
-        SG_LAUNCH("k_num_heavy", s, (k_num_heavy<float><<<grid, HEAVY_THREADS, smem, s>>>(
+        SG_LAUNCH("k_num_heavy", s, (k_num_heavy<float><<<grid, NUM_T, smem, s>>>(
                                         A, B, heavy, nheavy, rb, range_off, nranges, ranges, long_id, tp, T, C_rp, C_col,
                                         (float*)C_val, counter, gscr, amax, dbg)));
     }
@@ -667,6 +673,7 @@ cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, i
 }
 
 int heavy_kc() { return KC; }
+int heavy_grid() { return NUM_OCC * 148; }
 
 }  // namespace sg
 

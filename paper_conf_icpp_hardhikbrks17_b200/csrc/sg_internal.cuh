@@ -91,6 +91,7 @@ cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, i
 cudaError_t launch_max_a(const Mat& A, const int32_t* list, int64_t cnt, int64_t rb, unsigned long long* out,
                          cudaStream_t s);
 int heavy_kc();
+int heavy_grid();
 // threshold: cost histogram over rows then argmin over t in [0, cap_L]
 struct ThrResult { long long thr, Jmin, base, W_L, W_all, nonempty; };
 cudaError_t launch_cost_hist(const CostModelD& cm, const int64_t* w, const int64_t* a, const int64_t* u, int64_t nr,
