@@ -146,9 +146,11 @@ CostModelD cm_of(const sg_cost_model* c) {
 }
 
 // Default model: calibrated from the measured kernels (profiles/).
+// Fitted by tools/sweep.py (non-negative least squares of per-class kernel times over the
+// threshold grid on ER 2^18 and R-MAT 18; profiles/r01_sweep_calibration.json), in ps of SM time.
 const sg_cost_model kDefaultModel = {
-    /*kappa_L*/ 3000, /*lambda_L*/ 120, /*sigma_L*/ 0, /*rho_L*/ 150,
-    /*kappa_H*/ 250000, /*lambda_H*/ 60, /*tau_H*/ 400, /*mu_H*/ 120,
+    /*kappa_L*/ 0, /*lambda_L*/ 19273, /*sigma_L*/ 0, /*rho_L*/ 0,
+    /*kappa_H*/ 14832686, /*lambda_H*/ 1043, /*tau_H*/ 87934, /*mu_H*/ 0,
     /*tiles_fixed*/ 1, /*capu*/ 12288, /*cap_L*/ SG_CAP_L_MAX};
 
 // Identify over a row list (rows == nullptr: rows [0, nr)). Computes w, a, u of those rows on the
