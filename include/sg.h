@@ -160,6 +160,13 @@ sg_status sg_gather(sg_plan* plan, void* nccl_comm, int gather_values,
                     int64_t* C_row_ptr_global, int32_t* C_col_global /*nullable*/, void* C_val_global /*nullable*/,
                     int64_t* nnz_total_out /*host*/, void* stream);
 
+/* The host-only arithmetic of sg_gather (no device work, usable without a GPU): lay holds the
+ * per-rank (row_begin, row_end, nnz) triples in rank order. Checks that the blocks are contiguous
+ * from row 0 (SHAPE otherwise) and writes begin[r] (first row of rank r, nranks entries), off[r]
+ * (first C entry of rank r; nranks+1 entries, off[nranks] = total), the row count n and the total. */
+sg_status sg_gather_layout(const int64_t* lay /*host, 3*nranks*/, int nranks, int64_t* begin /*host*/,
+                           int64_t* off /*host*/, int64_t* n_out /*host*/, int64_t* total_out /*host*/);
+
 /* Plan introspection for tests and reports. */
 sg_status sg_plan_get_info(const sg_plan* plan, sg_plan_info* out /*host*/);
 /* Row classes of the plan's rows: 0 EMPTY, 1 LIGHT, 2 HEAVY (device int8, row_end-row_begin). */

@@ -36,7 +36,8 @@ _STATUS = ["SG_OK", "SG_ERR_INVALID_ARG", "SG_ERR_SHAPE", "SG_ERR_DTYPE", "SG_ER
 EXPORTS = ["sg_status_string", "sg_version", "sg_default_cost_model", "sg_row_work", "sg_sample_threshold",
            "sg_exhaustive_threshold", "sg_cost_curve", "sg_partition", "sg_symbolic", "sg_numeric", "sg_gather",
            "sg_plan_get_info", "sg_plan_get_classes", "sg_plan_get_work", "sg_plan_destroy", "sg_sample_rows",
-           "sg_profile_enable", "sg_launch_count", "sg_profile_count", "sg_profile_read", "sg_profile_reset"]
+           "sg_profile_enable", "sg_launch_count", "sg_profile_count", "sg_profile_read", "sg_profile_reset",
+           "sg_gather_layout"]
 
 
 class SgError(RuntimeError):
@@ -121,6 +122,7 @@ def load(build_if_missing: bool = True):
         "sg_profile_count": (i64, []),
         "sg_profile_read": (i64, [P, P, i64]),
         "sg_profile_reset": (None, []),
+        "sg_gather_layout": (st, [P, ctypes.c_int, P, P, pi64, pi64]),
     }
     for name, (res, args) in sigs.items():
         f = getattr(L, name)
@@ -379,6 +381,21 @@ class profile:
 
 def launch_count() -> int:
     return int(lib().sg_launch_count())
+
+
+def sg_gather_layout(layouts):
+    """Host-only assembly arithmetic of sg_gather: layouts = [(row_begin, row_end, nnz)] in rank
+    order -> (begin[nranks], off[nranks+1], n, total). Raises SgError(SHAPE) if not contiguous."""
+    import numpy as np
+    lay = np.ascontiguousarray(np.asarray(layouts, dtype=np.int64).reshape(-1))
+    G = lay.shape[0] // 3
+    begin = np.zeros(G, dtype=np.int64)
+    off = np.zeros(G + 1, dtype=np.int64)
+    n, tot = ctypes.c_int64(0), ctypes.c_int64(0)
+    _check(lib().sg_gather_layout(lay.ctypes.data_as(ctypes.c_void_p), G, begin.ctypes.data_as(ctypes.c_void_p),
+                                  off.ctypes.data_as(ctypes.c_void_p), ctypes.byref(n), ctypes.byref(tot)),
+           "sg_gather_layout")
+    return begin, off, int(n.value), int(tot.value)
 
 
 def spgemm(A: DeviceCSR, B: DeviceCSR, sample_frac: float = 0.01, seed: int = 1, cm: CostModel | None = None,

@@ -31,6 +31,24 @@ __global__ void k_fix_offsets(int64_t* rp, const int64_t* __restrict__ seg_begin
 }
 }  // namespace
 
+// Host-only assembly arithmetic (no CUDA, no NCCL): validates that the per-rank row blocks are
+// contiguous in rank order from row 0, and derives each rank's first row and first C entry.
+extern "C" sg_status sg_gather_layout(const int64_t* lay, int nranks, int64_t* begin, int64_t* off, int64_t* n_out,
+                                      int64_t* total_out) {
+    if (!lay || nranks < 1 || !begin || !off || !n_out || !total_out) return SG_ERR_INVALID_ARG;
+    if (lay[0] != 0) return SG_ERR_SHAPE;
+    off[0] = 0;
+    for (int r = 0; r < nranks; ++r) {
+        if (lay[3 * r + 1] < lay[3 * r] || lay[3 * r + 2] < 0) return SG_ERR_SHAPE;
+        if (r > 0 && lay[3 * r] != lay[3 * (r - 1) + 1]) return SG_ERR_SHAPE;
+        begin[r] = lay[3 * r];
+        off[r + 1] = off[r] + lay[3 * r + 2];
+    }
+    *n_out = lay[3 * (nranks - 1) + 1];
+    *total_out = off[nranks];
+    return SG_OK;
+}
+
 extern "C" sg_status sg_gather(sg_plan* plan, void* nccl_comm, int gather_values, const int64_t* local_row_ptr,
                                const int32_t* local_col, const void* local_val, int64_t* C_row_ptr_global,
                                int32_t* C_col_global, void* C_val_global, int64_t* nnz_total_out, void* stream) {
@@ -56,17 +74,10 @@ extern "C" sg_status sg_gather(sg_plan* plan, void* nccl_comm, int gather_values
         if (ncclAllGather(dlay, dlay + 3, 3, ncclInt64, comm, s) != ncclSuccess) { st = SG_ERR_NCCL; break; }
         if (cudaMemcpyAsync(lay.data(), dlay + 3, sizeof(int64_t) * 3 * nranks, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
             cudaStreamSynchronize(s) != cudaSuccess) { st = SG_ERR_CUDA; break; }
-        // contiguity: rank order, covering [0, n)
+        // contiguity: rank order, covering [0, n); entry offsets of every rank's C rows
         std::vector<int64_t> off(nranks + 1, 0), begin(nranks);
-        if (lay[0] != 0) { st = SG_ERR_SHAPE; break; }
-        for (int r = 0; r < nranks; ++r) {
-            if (r > 0 && lay[3 * r] != lay[3 * (r - 1) + 1]) { st = SG_ERR_SHAPE; break; }
-            begin[r] = lay[3 * r];
-            off[r + 1] = off[r] + lay[3 * r + 2];
-        }
-        if (st != SG_OK) break;
-        const int64_t n = lay[3 * (nranks - 1) + 1];
-        const int64_t total = off[nranks];
+        int64_t n = 0, total = 0;
+        if ((st = sg_gather_layout(lay.data(), nranks, begin.data(), off.data(), &n, &total)) != SG_OK) break;
         // 2. allgatherv of the local prefixes (rows_r entries each, excluding the trailing total)
         if (ncclGroupStart() != ncclSuccess) { st = SG_ERR_NCCL; break; }
         for (int r = 0; r < nranks; ++r) {

@@ -285,3 +285,35 @@ def test_errors():
     A32 = _dev(A.astype("f32"))
     with pytest.raises(sg.SgError, match="DTYPE"):
         sg.sg_symbolic(dA, A32, 10)
+
+
+def test_gather_single_rank_nccl():
+    """sg_gather through a real NCCL communicator (world size 1 on the one-GPU box): the global
+    row_ptr and the gathered col/val equal the local result."""
+    import os
+    import socket
+    import torch.distributed as dist
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dev = torch.device("cuda", 0)
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=dev)
+    try:
+        dist.barrier()
+        comm = dist.group.WORLD._get_backend(dev)._comm_ptr()
+        A = gen.config("rmat12")
+        dA = _dev(A)
+        plan = sg.sg_symbolic(dA, dA, 256)
+        col, val = sg.sg_numeric(plan, dA, dA)
+        rp, gcol, gval, tot = sg.sg_gather(plan, comm, col, val, gather_values=True, n_global=A.nrows,
+                                           nnz_global=plan.nnz)
+        torch.cuda.synchronize()
+        assert tot == plan.nnz
+        assert torch.equal(rp, plan.row_ptr)
+        assert torch.equal(gcol, col) and torch.equal(gval, val)
+        plan.destroy()
+    finally:
+        dist.destroy_process_group()
