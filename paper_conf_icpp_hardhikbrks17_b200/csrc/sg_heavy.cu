@@ -563,33 +563,24 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
             }
             __syncthreads();
             mark(3);
-            // ---- rank prefix over the range's words: warp w owns words [256w, 256w+256) in a
-            // lane-strided (bank-conflict-free) layout; 8 warp scans + one scan over the warps ----
+            // ---- rank prefix over the range's words: thread t owns words [8t, 8t+8) (two 128-bit
+            // loads, a sequential local prefix, one block scan, one 128-bit store of 8 uint16) ----
             {
-                const int wb = wid * 256;
-                int x[8], inc[8], rowbase[8], acc = 0;
-                #pragma unroll
-                for (int q = 0; q < 8; ++q) {
-                    const int wd = wb + 32 * q + lane;
-                    x[q] = wd < nwords ? __popc(S.bm[wd]) : 0;
-                    inc[q] = warp_incl_scan(x[q]);
-                    rowbase[q] = acc;
-                    acc += __shfl_sync(FULL, inc[q], 31);
-                }
-                if (lane == 0) S.ws[wid] = acc;
-                __syncthreads();
-                if (wid == 0) {
-                    const int y = lane < NUM_T / 32 ? S.ws[lane] : 0;
-                    const int yi = warp_incl_scan(y);
-                    S.ws[lane] = yi - y;
-                }
-                __syncthreads();
-                const int wpre = S.ws[wid];
-                #pragma unroll
-                for (int q = 0; q < 8; ++q) {
-                    const int wd = wb + 32 * q + lane;
-                    if (wd < nwords) S.pref[wd] = (uint16_t)(wpre + rowbase[q] + inc[q] - x[q]);
-                }
+                static_assert(RW_WORDS == 8 * NUM_T, "prefix layout: 8 words per thread");
+                const uint4 q0 = reinterpret_cast<const uint4*>(S.bm)[2 * tid];
+                const uint4 q1 = reinterpret_cast<const uint4*>(S.bm)[2 * tid + 1];
+                const int c0 = __popc(q0.x), c1 = __popc(q0.y), c2 = __popc(q0.z), c3 = __popc(q0.w);
+                const int c4 = __popc(q1.x), c5 = __popc(q1.y), c6 = __popc(q1.z), c7 = __popc(q1.w);
+                int t2;
+                const int p0 = block_scan<NUM_T>(c0 + c1 + c2 + c3 + c4 + c5 + c6 + c7, &t2, S.ws);
+                const int p1 = p0 + c0, p2 = p1 + c1, p3 = p2 + c2, p4 = p3 + c3, p5 = p4 + c4, p6 = p5 + c5,
+                          p7 = p6 + c6;
+                uint4 o;
+                o.x = (uint32_t)p0 | ((uint32_t)p1 << 16);
+                o.y = (uint32_t)p2 | ((uint32_t)p3 << 16);
+                o.z = (uint32_t)p4 | ((uint32_t)p5 << 16);
+                o.w = (uint32_t)p6 | ((uint32_t)p7 << 16);
+                reinterpret_cast<uint4*>(S.pref)[tid] = o;  // words >= nwords are zero: harmless prefixes
             }
             __syncthreads();
             mark(4);
@@ -629,15 +620,30 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 C_val[base + e] = (VT)S.vals[e];
                 S.vals[e] = 0.0;
             }
-            for (int wd = tid; wd < nwords; wd += NUM_T) {
-                uint32_t bits = S.bm[wd];
-                if (!bits) continue;
-                int64_t o = base + S.pref[wd];
-                S.bm[wd] = 0u;
-                while (bits) {
-                    const int b = __ffs(bits) - 1;
-                    bits &= bits - 1;
-                    C_col[o++] = (int32_t)(lo + wd * 32 + b);
+            // columns: a warp takes 32 consecutive words; entry e of the group is found by a shuffle
+            // search over the lanes' popcount prefix and __fns (n-th set bit): one lane per entry,
+            // consecutive lanes write consecutive positions (no per-bit divergent loops)
+            for (int wb = wid * 32; wb < nwords; wb += NUM_T) {
+                const int wd = wb + lane;
+                const uint32_t bits = wd < nwords ? S.bm[wd] : 0u;
+                if (bits) S.bm[wd] = 0u;
+                const int pc = __popc(bits);
+                const int inc = warp_incl_scan(pc);
+                const int gtot = __shfl_sync(FULL, inc, 31);
+                if (gtot == 0) continue;
+                const int ex = inc - pc;
+                const int64_t gbase = base + S.pref[wb];
+                for (int e0 = 0; e0 < gtot; e0 += 32) {
+                    const int e = e0 + lane;
+                    int s = 0;
+                    #pragma unroll
+                    for (int b = 16; b; b >>= 1) {
+                        const int eb = __shfl_sync(FULL, ex, s + b);
+                        if (eb <= e) s += b;
+                    }
+                    const uint32_t wbits = __shfl_sync(FULL, bits, s);
+                    const int k = e - __shfl_sync(FULL, ex, s);
+                    if (e < gtot) C_col[gbase + e] = (int32_t)(lo + (int64_t)(wb + s) * 32 + __fns(wbits, 0, k + 1));
                 }
             }
             __syncthreads();

@@ -317,3 +317,24 @@ def test_gather_single_rank_nccl():
         plan.destroy()
     finally:
         dist.destroy_process_group()
+
+
+def test_rmat22_multi_window_row_subset():
+    """p = 2^22 columns: four 2^20-column symbolic windows, T = 512 column tiles (config 4's
+    matrix). Rows [0, n/256) at the sampled threshold: structure bit-exact on every row of the
+    subset (row_ptr vs oracle counts), values on a seeded sample plus the heaviest rows."""
+    A = gen.config("C4")
+    dA = _dev(A)
+    thr, _ = sg.sg_sample_threshold(dA, dA, 0.002, 1)
+    re = A.nrows // 256
+    plan = sg.sg_symbolic(dA, dA, thr, 0, re)
+    col, val = sg.sg_numeric(plan, dA, dA)
+    torch.cuda.synchronize()
+    rp = plan.row_ptr.cpu().numpy()
+    rows = np.arange(re, dtype=np.int64)
+    assert np.array_equal(np.diff(rp), oracle.counts(A, A, rows))
+    w = oracle.row_work(A, A)[:re]
+    pick = np.union1d(oracle.sample_rows(re, 5, 0.01), np.argsort(w)[-16:]).astype(np.int64)
+    R = oracle.spgemm(A, A, rows=pick, with_absmag=True)
+    compare_rows(rp, col.cpu().numpy(), val.cpu().numpy(), R, "f64")
+    plan.destroy()
