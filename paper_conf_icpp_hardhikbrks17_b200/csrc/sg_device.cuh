@@ -134,26 +134,13 @@ __device__ __forceinline__ int acc_insert(int32_t* keys, double* vals, int32_t c
     return (int)h;
 }
 
-// sort the occupied run starting at slot s (insertion sort; runs are short at load <= 1/2)
-__device__ __forceinline__ void sort_run(int32_t* keys, double* vals, int s, int nslots) {
-    int e = s + 1;
-    while (e < nslots && keys[e] != EMPTY_KEY) ++e;
-    for (int i = s + 1; i < e; ++i) {
-        const int32_t k = keys[i];
-        const double v = vals[i];
-        int q = i - 1;
-        while (q >= s && keys[q] > k) { keys[q + 1] = keys[q]; vals[q + 1] = vals[q]; --q; }
-        keys[q + 1] = k;
-        vals[q + 1] = v;
-    }
-}
-
 // Group-wide emission of slots [0, nslots) in slot order into C at `base`, clearing each slot.
 // Each warp of the group owns a contiguous chunk of slots; one group-level exclusive scan of the
 // per-warp counts places the chunks (ws: >= G/32 ints of shared memory per group).
 template <int G, int BLK, class VT>
 __device__ __forceinline__ void emit_slots(int32_t* keys, double* vals, int nslots, int64_t base,
-                                           int32_t* __restrict__ C_col, VT* __restrict__ C_val, int* ws) {
+                                           int32_t* __restrict__ C_col, VT* __restrict__ C_val, int* ws,
+                                           bool ranked) {
     constexpr int NW = G / 32;
     const int lane = threadIdx.x & 31;
     const int w = (threadIdx.x % G) / 32;
@@ -171,19 +158,49 @@ __device__ __forceinline__ void emit_slots(int32_t* keys, double* vals, int nslo
         for (int q = 0; q < w; ++q) pos += ws[q];
         group_bar<G, BLK>();
     }
+    if (!ranked) {  // slot order is column order (identity map or runs already sorted)
+        for (int s0 = s_lo; s0 < s_hi; s0 += 32) {
+            const int s = s0 + lane;
+            const int32_t k = s < s_hi ? keys[s] : EMPTY_KEY;
+            const unsigned m = __ballot_sync(FULL, k != EMPTY_KEY);
+            if (k != EMPTY_KEY) {
+                const int64_t o = pos + __popc(m & lanemask_lt());
+                C_col[o] = k;
+                C_val[o] = (VT)vals[s];
+                keys[s] = EMPTY_KEY;
+                vals[s] = 0.0;
+            }
+            pos += __popc(m);
+        }
+        return;
+    }
+    // Order-preserving hash: runs (maximal occupied stretches) are mutually ordered but not sorted
+    // inside. The entry in slot s goes to (#occupied slots before its run) + (its rank inside the
+    // run): found from the occupancy ballot plus a short scan of the run's keys — no data movement.
     for (int s0 = s_lo; s0 < s_hi; s0 += 32) {
         const int s = s0 + lane;
         const int32_t k = s < s_hi ? keys[s] : EMPTY_KEY;
         const unsigned m = __ballot_sync(FULL, k != EMPTY_KEY);
         if (k != EMPTY_KEY) {
-            const int64_t o = pos + __popc(m & lanemask_lt());
+            const unsigned below = ~m & lanemask_lt();
+            int rs;
+            if (below) rs = s0 + 31 - __clz(below) + 1;
+            else { rs = s0; while (rs > 0 && keys[rs - 1] != EMPTY_KEY) --rs; }
+            const unsigned above = lane == 31 ? 0u : (~m & (~0u << (lane + 1)));
+            int re;
+            if (above) re = s0 + __ffs(above) - 1;
+            else { re = s0 + 32; while (re < nslots && keys[re] != EMPTY_KEY) ++re; }
+            int rank = 0;
+            for (int j = rs; j < re; ++j) rank += keys[j] < k;
+            const int64_t o = pos + __popc(m & lanemask_lt()) - (s - rs) + rank;
             C_col[o] = k;
             C_val[o] = (VT)vals[s];
-            keys[s] = EMPTY_KEY;
-            vals[s] = 0.0;
         }
         pos += __popc(m);
     }
+    group_bar<G, BLK>();  // every rank computed before any slot is cleared
+    for (int s = s_lo + lane; s < s_hi; s += 32)
+        if (keys[s] != EMPTY_KEY) { keys[s] = EMPTY_KEY; vals[s] = 0.0; }
 }
 
 }  // namespace sg

@@ -144,11 +144,7 @@ __global__ void __launch_bounds__(G * R) k_num_light(Mat A, Mat B, const int32_t
         }
         group_bar<G, BLK>();
         const int nslots = hmax + 1;
-        if (!ident)
-            for (int s = t; s < nslots; s += G)
-                if (keys[s] != EMPTY_KEY && (s == 0 || keys[s - 1] == EMPTY_KEY)) sort_run(keys, vals, s, nslots);
-        group_bar<G, BLK>();
-        emit_slots<G, BLK, VT>(keys, vals, nslots, C_rp[li], C_col, C_val, gws);
+        emit_slots<G, BLK, VT>(keys, vals, nslots, C_rp[li], C_col, C_val, gws, !ident);
         group_bar<G, BLK>();
     }
 }
