@@ -149,8 +149,8 @@ CostModelD cm_of(const sg_cost_model* c) {
 // Fitted by tools/sweep.py (non-negative least squares of per-class kernel times over the
 // threshold grid on ER 2^18 and R-MAT 18; profiles/r01_sweep_calibration.json), in ps of SM time.
 const sg_cost_model kDefaultModel = {
-    /*kappa_L*/ 0, /*lambda_L*/ 19273, /*sigma_L*/ 0, /*rho_L*/ 0,
-    /*kappa_H*/ 14832686, /*lambda_H*/ 1043, /*tau_H*/ 87934, /*mu_H*/ 0,
+    /*kappa_L*/ 33399, /*lambda_L*/ 7915, /*sigma_L*/ 0, /*rho_L*/ 0,
+    /*kappa_H*/ 17907513, /*lambda_H*/ 1102, /*tau_H*/ 68338, /*mu_H*/ 209,
     /*tiles_fixed*/ 1, /*capu*/ 12288, /*cap_L*/ SG_CAP_L_MAX};
 
 // Identify over a row list (rows == nullptr: rows [0, nr)). Computes w, a, u of those rows on the
@@ -528,8 +528,11 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
         const char* dbe = getenv("SG_DEBUG_HEAVY");
         unsigned long long* dbg = nullptr;
         if (dbe && dbe[0] == '1') {
-            CKP(pl, cudaMallocAsync((void**)&dbg, 8 * sizeof(unsigned long long), s));
-            CKP(pl, cudaMemsetAsync(dbg, 0, 8 * sizeof(unsigned long long), s));
+            CKP(pl, cudaMallocAsync((void**)&dbg, 9 * sizeof(unsigned long long), s));
+            CKP(pl, cudaMemsetAsync(dbg, 0, 9 * sizeof(unsigned long long), s));
+            const char* blk = getenv("SG_DEBUG_BLOCKS");  // results invalid: profiling experiments only
+            unsigned long long nb = blk ? strtoull(blk, nullptr, 10) : 0ull;
+            CKP(pl, cudaMemcpyAsync(dbg + 8, &nb, sizeof(nb), cudaMemcpyHostToDevice, s));
         }
         CKP(pl, launch_num_heavy(a, b, pl->heavy, pl->nheavy, pl->rb, pl->range_off, pl->nranges, pl->ranges,
                                  pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter, pl->gscr, pl->amax, s,

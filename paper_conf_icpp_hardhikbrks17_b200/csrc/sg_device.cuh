@@ -203,4 +203,146 @@ __device__ __forceinline__ void emit_slots(int32_t* keys, double* vals, int nslo
         if (keys[s] != EMPTY_KEY) { keys[s] = EMPTY_KEY; vals[s] = 0.0; }
 }
 
+// ---- block-level product flattening (heavy path; light rows with U >= 1024) ----------------------
+__device__ __forceinline__ int64_t lower_bound_col(const int32_t* __restrict__ col, int64_t lo, int64_t hi, int64_t x) {
+    while (lo < hi) {
+        int64_t mid = (lo + hi) >> 1;
+        if ((int64_t)__ldg(col + mid) < x) lo = mid + 1; else hi = mid;
+    }
+    return lo;
+}
+
+// exclusive scan of one int per thread over a 1024-thread block; *total for everyone
+template <int NT>
+__device__ __forceinline__ int block_scan(int v, int* total, int* ws) {
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    int inc = warp_incl_scan(v);
+    if (lane == 31) ws[wid] = inc;
+    __syncthreads();
+    if (wid == 0) {
+        int x = lane < NT / 32 ? ws[lane] : 0;
+        int xi = warp_incl_scan(x);
+        ws[lane] = xi - x;
+        if (lane == 31) ws[32] = xi;
+    }
+    __syncthreads();
+    int r = ws[wid] + inc - v;
+    *total = ws[32];
+    __syncthreads();
+    return r;
+}
+
+// largest i in [0, nk) with off[i] <= j (that entry has len > 0)
+__device__ __forceinline__ int find_k(const int* off, int nk, int j) {
+    int lo = 0, hi = nk - 1;
+    while (lo < hi) {
+        int mid = (lo + hi + 1) >> 1;
+        if (off[mid] <= j) lo = mid; else hi = mid - 1;
+    }
+    return lo;
+}
+
+template <int NT>
+__device__ __forceinline__ long long block_scan_ll(long long v, long long* total, long long* ws) {
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    long long inc = warp_incl_scan(v);
+    if (lane == 31) ws[wid] = inc;
+    __syncthreads();
+    if (wid == 0) {
+        long long x = lane < NT / 32 ? ws[lane] : 0;
+        long long xi = warp_incl_scan(x);
+        ws[lane] = xi - x;
+        if (lane == 31) ws[32] = xi;
+    }
+    __syncthreads();
+    long long r = ws[wid] + inc - v;
+    *total = ws[32];
+    __syncthreads();
+    return r;
+}
+
+// One chunk of k entries (one per thread): pack the entries with len > 0, in order, into
+// s_beg / s_off (exclusive prefix of len) / s_a; returns the chunk's product count, *nk = packed.
+template <int NT, class BEG>
+__device__ __forceinline__ int chunk_compact(int len, BEG beg, double a, BEG* s_beg, int* s_off, double* s_a, int* nk,
+                                             long long* wsll) {
+    long long tot;
+    const long long ex = block_scan_ll<NT>(((long long)len << 16) | (len > 0 ? 1 : 0), &tot, wsll);
+    if (len > 0) {
+        const int ci = (int)(ex & 0xFFFF);
+        s_beg[ci] = beg;
+        s_off[ci] = (int)(ex >> 16);
+        if (s_a) s_a[ci] = a;
+    }
+    *nk = (int)(tot & 0xFFFF);
+    __syncthreads();
+    return (int)(tot >> 16);
+}
+
+// Products [0, tot) of a packed chunk, split into one contiguous slice per warp. Within a slice a
+// batch of 32 consecutive products lies in at most 32 consecutive packed entries (each has len >= 1),
+// so every lane finds its entry with a 5-step shuffle search; the next batch's gathers are issued
+// before the current batch is consumed (two batches in flight per warp).
+template <int NT, bool VAL, class VT, class BEG, class F>
+__device__ __forceinline__ void warp_slice(const BEG* s_beg, const int* s_off, const double* s_a, int nk, int tot,
+                                           const Mat& B, F&& f) {
+    constexpr int NW = NT / 32;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int per = (((tot + NW - 1) / NW) + 31) & ~31;
+    const int j_lo = wid * per, j_hi = min(tot, j_lo + per);
+    if (j_lo >= j_hi) return;
+    int i0 = find_k(s_off, nk, j_lo);
+    auto fetch = [&](int j0, int& c, double& v) {
+        // fast path: the whole batch lies inside entry i0 (long B segments: hub rows of B)
+        const int e0 = i0 + 1 < nk ? s_off[i0 + 1] : tot;
+        if (j0 + 31 < e0) {
+            const int j = j0 + lane;
+            c = -1;
+            v = 0.0;
+            if (j < j_hi) {
+                const int64_t q = (int64_t)s_beg[i0] + (j - s_off[i0]);
+                c = __ldg(B.col + q);
+                if (VAL) v = s_a[i0] * ldv<VT>(B.val, q);
+            }
+            return;
+        }
+        const int ii = i0 + lane;
+        const int o = ii < nk ? s_off[ii] : INT_MAX;
+        const int j = j0 + lane;
+        int s = 0;
+        #pragma unroll
+        for (int b = 16; b; b >>= 1) {
+            const int ob = __shfl_sync(FULL, o, s + b);
+            if (ob <= j) s += b;
+        }
+        const int kk = i0 + s;
+        const int os = __shfl_sync(FULL, o, s);
+        c = -1;
+        v = 0.0;
+        if (j < j_hi) {
+            const int64_t q = (int64_t)s_beg[kk] + (j - os);
+            c = __ldg(B.col + q);
+            if (VAL) v = s_a[kk] * ldv<VT>(B.val, q);
+        }
+        i0 = __shfl_sync(FULL, kk, 31);
+    };
+    // four batches in flight: fetch(j + 96) is issued before batch j is consumed
+    int c0, c1, c2, c3;
+    double v0, v1, v2, v3;
+    fetch(j_lo, c0, v0);
+    fetch(j_lo + 32, c1, v1);
+    fetch(j_lo + 64, c2, v2);
+    for (int j0 = j_lo; j0 < j_hi; j0 += 128) {
+        fetch(j0 + 96, c3, v3);
+        f(c0, v0);  // f is called by every lane (c < 0: no product) so it may use warp collectives
+        if (j0 + 128 >= j_hi) { f(c1, v1); f(c2, v2); f(c3, v3); break; }
+        fetch(j0 + 128, c0, v0);
+        f(c1, v1);
+        fetch(j0 + 160, c1, v1);
+        f(c2, v2);
+        fetch(j0 + 192, c2, v2);
+        f(c3, v3);
+    }
+}
+
 }  // namespace sg
