@@ -90,7 +90,7 @@ def load(build_if_missing: bool = True):
     global _lib
     if _lib is not None:
         return _lib
-    so = _build.SO
+    so = os.environ.get("SG_LIB_PATH", _build.SO)  # A/B experiments may point at another build
     if not os.path.exists(so):
         if not build_if_missing:
             raise ImportError(f"{so} is missing; run __graft_entry__.build()")

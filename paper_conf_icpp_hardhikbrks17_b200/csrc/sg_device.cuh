@@ -279,23 +279,30 @@ __device__ __forceinline__ int chunk_compact(int len, BEG beg, double a, BEG* s_
     return (int)(tot >> 16);
 }
 
-// Products [0, tot) of a packed chunk, split into one contiguous slice per warp. Within a slice a
-// batch of 32 consecutive products lies in at most 32 consecutive packed entries (each has len >= 1),
-// so every lane finds its entry with a 5-step shuffle search; the next batch's gathers are issued
-// before the current batch is consumed (two batches in flight per warp).
-template <int NT, bool VAL, class VT, class BEG, class F>
-__device__ __forceinline__ void warp_slice(const BEG* s_beg, const int* s_off, const double* s_a, int nk, int tot,
-                                           const Mat& B, F&& f) {
-    constexpr int NW = NT / 32;
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    const int per = (((tot + NW - 1) / NW) + 31) & ~31;
-    const int j_lo = wid * per, j_hi = min(tot, j_lo + per);
-    if (j_lo >= j_hi) return;
-    int i0 = find_k(s_off, nk, j_lo);
-    auto fetch = [&](int j0, int& c, double& v) {
-        // fast path: the whole batch lies inside entry i0 (long B segments: hub rows of B)
+// Products [0, tot) of a packed chunk, split into one contiguous slice per warp (a multiple of 32).
+// Within a slice a batch of 32 consecutive products lies in at most 32 consecutive packed entries
+// (each has len >= 1), so every lane finds its entry with a 5-step shuffle search (or none: the
+// fast path when the batch lies inside one long B segment).
+template <int NT, bool VAL, class VT, class BEG>
+struct SliceCursor {
+    const BEG* s_beg;
+    const int* s_off;
+    const double* s_a;
+    int nk, tot, j_lo, j_hi, i0;
+    __device__ __forceinline__ SliceCursor(const BEG* sb, const int* so, const double* sa, int nk_, int tot_)
+        : s_beg(sb), s_off(so), s_a(sa), nk(nk_), tot(tot_) {
+        constexpr int NW = NT / 32;
+        const int wid = threadIdx.x >> 5;
+        const int per = (((tot + NW - 1) / NW) + 31) & ~31;
+        j_lo = wid * per;
+        j_hi = min(tot, j_lo + per);
+        i0 = j_lo < j_hi ? find_k(s_off, nk, j_lo) : 0;
+    }
+    // batch [j0, j0 + 32): lane's (column, a_ik * b_kj), c = -1 beyond the slice
+    __device__ __forceinline__ void fetch(const Mat& B, int j0, int& c, double& v) {
+        const int lane = threadIdx.x & 31;
         const int e0 = i0 + 1 < nk ? s_off[i0 + 1] : tot;
-        if (j0 + 31 < e0) {
+        if (j0 + 31 < e0) {  // fast path: the whole batch lies inside entry i0 (hub rows of B)
             const int j = j0 + lane;
             c = -1;
             v = 0.0;
@@ -325,24 +332,50 @@ __device__ __forceinline__ void warp_slice(const BEG* s_beg, const int* s_off, c
             if (VAL) v = s_a[kk] * ldv<VT>(B.val, q);
         }
         i0 = __shfl_sync(FULL, kk, 31);
-    };
-    // four batches in flight: fetch(j + 96) is issued before batch j is consumed
+    }
+};
+
+// Streams the warp's slice through f, four batches in flight (fetch(j + 96) is issued before batch
+// j is consumed). f is called by every lane (c < 0: no product) so it may use warp collectives.
+template <int NT, bool VAL, class VT, class BEG, class F>
+__device__ __forceinline__ void warp_slice(const BEG* s_beg, const int* s_off, const double* s_a, int nk, int tot,
+                                           const Mat& B, F&& f) {
+    SliceCursor<NT, VAL, VT, BEG> sc(s_beg, s_off, s_a, nk, tot);
+    const int j_lo = sc.j_lo, j_hi = sc.j_hi;
+    if (j_lo >= j_hi) return;
     int c0, c1, c2, c3;
     double v0, v1, v2, v3;
-    fetch(j_lo, c0, v0);
-    fetch(j_lo + 32, c1, v1);
-    fetch(j_lo + 64, c2, v2);
+    sc.fetch(B, j_lo, c0, v0);
+    sc.fetch(B, j_lo + 32, c1, v1);
+    sc.fetch(B, j_lo + 64, c2, v2);
     for (int j0 = j_lo; j0 < j_hi; j0 += 128) {
-        fetch(j0 + 96, c3, v3);
-        f(c0, v0);  // f is called by every lane (c < 0: no product) so it may use warp collectives
+        sc.fetch(B, j0 + 96, c3, v3);
+        f(c0, v0);
         if (j0 + 128 >= j_hi) { f(c1, v1); f(c2, v2); f(c3, v3); break; }
-        fetch(j0 + 128, c0, v0);
+        sc.fetch(B, j0 + 128, c0, v0);
         f(c1, v1);
-        fetch(j0 + 160, c1, v1);
+        sc.fetch(B, j0 + 160, c1, v1);
         f(c2, v2);
-        fetch(j0 + 192, c2, v2);
+        sc.fetch(B, j0 + 192, c2, v2);
         f(c3, v3);
     }
+}
+
+// Small chunks (every warp slice <= 128 products, i.e. tot <= 4*NT): the warp's whole slice is
+// fetched once into registers (columns AND values), so a two-pass consumer (bitmap, then rank
+// accumulation) reads B once. Returns false (nothing fetched) when the chunk is too large.
+template <int NT, class VT, class BEG>
+__device__ __forceinline__ bool warp_slice_regs(const BEG* s_beg, const int* s_off, const double* s_a, int nk, int tot,
+                                                const Mat& B, int (&c)[4], double (&v)[4]) {
+    if (tot > 4 * NT) return false;
+    SliceCursor<NT, true, VT, BEG> sc(s_beg, s_off, s_a, nk, tot);
+    #pragma unroll
+    for (int r = 0; r < 4; ++r) {
+        c[r] = -1;
+        v[r] = 0.0;
+        if (sc.j_lo + 32 * r < sc.j_hi) sc.fetch(B, sc.j_lo + 32 * r, c[r], v[r]);
+    }
+    return true;
 }
 
 }  // namespace sg

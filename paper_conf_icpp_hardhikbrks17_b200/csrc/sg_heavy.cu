@@ -17,6 +17,9 @@
 
 namespace sg {
 
+#ifndef SG_INREG
+#define SG_INREG 1
+#endif
 constexpr int SYM_T = HEAVY_THREADS;  // symbolic: one CTA of 1024 threads per SM (128 KB bitmap window)
 constexpr int NUM_T = 1024;           // numeric: threads per CTA
 constexpr int NUM_OCC = 1;            // numeric CTAs per SM (smem-bound)
@@ -365,6 +368,9 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
             const int64_t lo = (int64_t)R.t0 * TW, hi = min(p, (int64_t)R.t1 * TW);
             const int nwords = (int)((hi - lo + 31) / 32);
             int tot1 = 0, nk1 = 0;
+            bool inreg = false;
+            int rc[4];
+            double rv[4];
             // ---- pass 1: segments (advance cursors) + bitmap of the range ----
             for (int c0 = 0; c0 < na; c0 += KC) {
                 const int i = c0 + tid;
@@ -392,9 +398,17 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 int nk;
                 const int ctot = chunk_compact<NUM_T, int32_t>(len, beg, a, S.s_beg, S.s_off, S.s_a, &nk, S.wsll);
                 mark(2);
-                warp_slice<NUM_T, false, VT, int32_t>(S.s_beg, S.s_off, nullptr, nk, ctot, B, [&](int32_t c, double) {
+                auto setbit = [&](int32_t c, double) {
                     if (c >= 0) { const uint32_t d = (uint32_t)(c - lo); atomicOr(&S.bm[d >> 5], 1u << (d & 31)); }
-                });
+                };
+                // small ranges: the products stay in registers from pass 1 to pass 2 (B read once)
+                inreg = SG_INREG && single && warp_slice_regs<NUM_T, VT, int32_t>(S.s_beg, S.s_off, S.s_a, nk, ctot, B, rc, rv);
+                if (inreg) {
+                    #pragma unroll
+                    for (int r = 0; r < 4; ++r) setbit(rc[r], 0.0);
+                } else {
+                    warp_slice<NUM_T, false, VT, int32_t>(S.s_beg, S.s_off, nullptr, nk, ctot, B, setbit);
+                }
                 tot1 = ctot;
                 nk1 = nk;
                 if (!single) __syncthreads();
@@ -430,7 +444,10 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 const int rank = S.pref[d >> 5] + __popc(wv & ((1u << (d & 31)) - 1u));
                 atomicAdd(&S.vals[rank], v);
             };
-            if (single) {
+            if (inreg) {
+                #pragma unroll
+                for (int r = 0; r < 4; ++r) acc(rc[r], rv[r]);
+            } else if (single) {
                 warp_slice<NUM_T, true, VT, int32_t>(S.s_beg, S.s_off, S.s_a, nk1, tot1, B, acc);  // pass-1 packing kept
             } else {
                 for (int c0 = 0; c0 < na; c0 += KC) {
