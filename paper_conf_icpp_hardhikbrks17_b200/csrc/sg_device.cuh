@@ -213,24 +213,22 @@ __device__ __forceinline__ int64_t lower_bound_col(const int32_t* __restrict__ c
 }
 
 // exclusive scan of one int per thread over a 1024-thread block; *total for everyone
-template <int NT>
-__device__ __forceinline__ int block_scan(int v, int* total, int* ws) {
+// Exclusive scan of one value per thread over an NT-thread block with ONE barrier: warp totals go
+// to ws, then every warp re-scans the (<= 32) warp totals itself. ws must not be rewritten until
+// the caller has passed another __syncthreads (call sites alternate between distinct ws arrays).
+template <int NT, class T>
+__device__ __forceinline__ T block_scan1(T v, T* total, T* ws) {
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    int inc = warp_incl_scan(v);
+    const T inc = warp_incl_scan(v);
     if (lane == 31) ws[wid] = inc;
     __syncthreads();
-    if (wid == 0) {
-        int x = lane < NT / 32 ? ws[lane] : 0;
-        int xi = warp_incl_scan(x);
-        ws[lane] = xi - x;
-        if (lane == 31) ws[32] = xi;
-    }
-    __syncthreads();
-    int r = ws[wid] + inc - v;
-    *total = ws[32];
-    __syncthreads();
-    return r;
+    const T x = lane < NT / 32 ? ws[lane] : T(0);
+    const T xi = warp_incl_scan(x);
+    *total = __shfl_sync(FULL, xi, 31);
+    return __shfl_sync(FULL, xi - x, wid) + inc - v;
 }
+template <int NT>
+__device__ __forceinline__ int block_scan(int v, int* total, int* ws) { return block_scan1<NT, int>(v, total, ws); }
 
 // largest i in [0, nk) with off[i] <= j (that entry has len > 0)
 __device__ __forceinline__ int find_k(const int* off, int nk, int j) {
@@ -244,21 +242,7 @@ __device__ __forceinline__ int find_k(const int* off, int nk, int j) {
 
 template <int NT>
 __device__ __forceinline__ long long block_scan_ll(long long v, long long* total, long long* ws) {
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    long long inc = warp_incl_scan(v);
-    if (lane == 31) ws[wid] = inc;
-    __syncthreads();
-    if (wid == 0) {
-        long long x = lane < NT / 32 ? ws[lane] : 0;
-        long long xi = warp_incl_scan(x);
-        ws[lane] = xi - x;
-        if (lane == 31) ws[32] = xi;
-    }
-    __syncthreads();
-    long long r = ws[wid] + inc - v;
-    *total = ws[32];
-    __syncthreads();
-    return r;
+    return block_scan1<NT, long long>(v, total, ws);
 }
 
 // One chunk of k entries (one per thread): pack the entries with len > 0, in order, into
