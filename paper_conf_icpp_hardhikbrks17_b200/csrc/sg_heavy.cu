@@ -324,7 +324,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
     auto mark = [&](int k) { if (dbg && threadIdx.x == 0) { long long t = clock64(); tph[k] += t - t_last; t_last = t; } };
     HeavySmem& S = *reinterpret_cast<HeavySmem*>(smem_raw);
     __shared__ long long s_j;
-    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+    const int tid = threadIdx.x;
     const int64_t p = B.ncols;
     int4* gs = gscr + (int64_t)blockIdx.x * amax;  // multi-chunk rows: per-k (cur, -, beg, len)
     for (int q = tid; q < RW_WORDS; q += NUM_T) S.bm[q] = 0u;
@@ -366,7 +366,6 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
             // debug (SG_DEBUG_BLOCKS=b): only the first b column blocks (later ranges never feed cursors)
             if (dbg && dbg[8] != 0 && (unsigned long long)(R.t0 / RW_TILES) >= dbg[8]) break;
             const int64_t lo = (int64_t)R.t0 * TW, hi = min(p, (int64_t)R.t1 * TW);
-            const int nwords = (int)((hi - lo + 31) / 32);
             int tot1 = 0, nk1 = 0;
             bool inreg = false;
             int rc[4];
@@ -467,38 +466,30 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
             }
             __syncthreads();
             mark(5);
-            // ---- emission: values by rank (coalesced); columns word by word, one lane per bit, so
-            // each non-empty word becomes one coalesced run of C.col ----
+            // ---- emission: values by rank (coalesced), then columns from the bitmap ----
             const int64_t base = crow + R.off;
             const int cnt = R.cnt;
             for (int e = tid; e < cnt; e += NUM_T) {
                 C_val[base + e] = (VT)S.vals[e];
                 S.vals[e] = 0.0;
             }
-            // columns: a warp takes 32 consecutive words; entry e of the group is found by a shuffle
-            // search over the lanes' popcount prefix and __fns (n-th set bit): one lane per entry,
-            // consecutive lanes write consecutive positions (no per-bit divergent loops)
-            for (int wb = wid * 32; wb < nwords; wb += NUM_T) {
-                const int wd = wb + lane;
-                const uint32_t bits = wd < nwords ? S.bm[wd] : 0u;
-                if (bits) S.bm[wd] = 0u;
-                const int pc = __popc(bits);
-                const int inc = warp_incl_scan(pc);
-                const int gtot = __shfl_sync(FULL, inc, 31);
-                if (gtot == 0) continue;
-                const int ex = inc - pc;
-                const int64_t gbase = base + S.pref[wb];
-                for (int e0 = 0; e0 < gtot; e0 += 32) {
-                    const int e = e0 + lane;
-                    int s = 0;
-                    #pragma unroll
-                    for (int b = 16; b; b >>= 1) {
-                        const int eb = __shfl_sync(FULL, ex, s + b);
-                        if (eb <= e) s += b;
+            // columns: thread t owns words [8t, 8t+8) (the prefix layout); its entries are consecutive
+            // ranks from pref[8t], emitted lowest bit first from four 64-bit registers (no shuffles)
+            {
+                uint4* bm4 = reinterpret_cast<uint4*>(S.bm);
+                const uint4 q0 = bm4[2 * tid], q1 = bm4[2 * tid + 1];
+                uint64_t d0 = q0.x | ((uint64_t)q0.y << 32), d1 = q0.z | ((uint64_t)q0.w << 32);
+                uint64_t d2 = q1.x | ((uint64_t)q1.y << 32), d3 = q1.z | ((uint64_t)q1.w << 32);
+                if (d0 | d1 | d2 | d3) {
+                    bm4[2 * tid] = make_uint4(0, 0, 0, 0);
+                    bm4[2 * tid + 1] = make_uint4(0, 0, 0, 0);
+                    int32_t* out = C_col + base + (S.pref[8 * tid]);
+                    int32_t cb = (int32_t)(lo + (int64_t)tid * 256);
+                    while (d0 | d1 | d2 | d3) {
+                        if (d0 == 0) { d0 = d1; d1 = d2; d2 = d3; d3 = 0; cb += 64; continue; }
+                        *out++ = cb + __ffsll((long long)d0) - 1;
+                        d0 &= d0 - 1;
                     }
-                    const uint32_t wbits = __shfl_sync(FULL, bits, s);
-                    const int k = e - __shfl_sync(FULL, ex, s);
-                    if (e < gtot) C_col[gbase + e] = (int32_t)(lo + (int64_t)(wb + s) * 32 + __fns(wbits, 0, k + 1));
                 }
             }
             __syncthreads();
