@@ -361,8 +361,11 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
         __syncthreads();
         mark(1);
         if (dbg && tid == 0) tph[7] += nr;
+        RangeRec Rn;  // next range's record, loaded one range ahead
+        if (nr > 0) Rn = rr[0];
         for (int ri = 0; ri < nr; ++ri) {
-            const RangeRec R = rr[ri];
+            const RangeRec R = Rn;
+            if (ri + 1 < nr) Rn = rr[ri + 1];
             // debug (SG_DEBUG_BLOCKS=b): only the first b column blocks (later ranges never feed cursors)
             if (dbg && dbg[8] != 0 && (unsigned long long)(R.t0 / RW_TILES) >= dbg[8]) break;
             const int64_t lo = (int64_t)R.t0 * TW, hi = min(p, (int64_t)R.t1 * TW);
@@ -382,7 +385,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                         beg = cur; len = end - cur; a = S.c_a[i];
                         S.c_cur[i] = end;
                         // prefetch the next range's tile pointer (its latency hides behind this range)
-                        if (lid >= 0 && ri + 1 < nr) tpv = __ldg(tp + (int64_t)lid * (T + 1) + rr[ri + 1].t1);
+                        if (lid >= 0 && ri + 1 < nr) tpv = __ldg(tp + (int64_t)lid * (T + 1) + Rn.t1);
                     } else {
                         const int4 g = gs[i];
                         const int k = __ldg(A.col + s0 + i);
@@ -435,7 +438,27 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
             }
             __syncthreads();
             mark(4);
-            // ---- pass 2: accumulate into the compact array at rank(c) ----
+            // ---- pass 2: columns of the range, then every product accumulated at rank(c) ----
+            const int64_t base = crow + R.off;
+            // columns first: thread t owns words [8t, 8t+8) (the prefix layout); its entries are the
+            // consecutive ranks from pref[8t], written lowest bit first from four 64-bit registers.
+            // The loop is instruction-bound and divergent; placed here it overlaps the gather
+            // latency of the other warps' products instead of ending in a barrier of its own.
+            {
+                const uint4* bm4 = reinterpret_cast<const uint4*>(S.bm);
+                const uint4 q0 = bm4[2 * tid], q1 = bm4[2 * tid + 1];
+                uint64_t d0 = q0.x | ((uint64_t)q0.y << 32), d1 = q0.z | ((uint64_t)q0.w << 32);
+                uint64_t d2 = q1.x | ((uint64_t)q1.y << 32), d3 = q1.z | ((uint64_t)q1.w << 32);
+                if (d0 | d1 | d2 | d3) {
+                    int32_t* out = C_col + base + S.pref[8 * tid];
+                    int32_t cb = (int32_t)(lo + (int64_t)tid * 256);
+                    while (d0 | d1 | d2 | d3) {
+                        if (d0 == 0) { d0 = d1; d1 = d2; d2 = d3; d3 = 0; cb += 64; continue; }
+                        *out++ = cb + __ffsll((long long)d0) - 1;
+                        d0 &= d0 - 1;
+                    }
+                }
+            }
             auto acc = [&](int32_t c, double v) {
                 if (c < 0) return;
                 const uint32_t d = (uint32_t)(c - lo);
@@ -466,31 +489,16 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
             }
             __syncthreads();
             mark(5);
-            // ---- emission: values by rank (coalesced), then columns from the bitmap ----
-            const int64_t base = crow + R.off;
+            // ---- values by rank (coalesced); accumulator and bitmap cleared for the next range ----
             const int cnt = R.cnt;
             for (int e = tid; e < cnt; e += NUM_T) {
                 C_val[base + e] = (VT)S.vals[e];
                 S.vals[e] = 0.0;
             }
-            // columns: thread t owns words [8t, 8t+8) (the prefix layout); its entries are consecutive
-            // ranks from pref[8t], emitted lowest bit first from four 64-bit registers (no shuffles)
             {
                 uint4* bm4 = reinterpret_cast<uint4*>(S.bm);
-                const uint4 q0 = bm4[2 * tid], q1 = bm4[2 * tid + 1];
-                uint64_t d0 = q0.x | ((uint64_t)q0.y << 32), d1 = q0.z | ((uint64_t)q0.w << 32);
-                uint64_t d2 = q1.x | ((uint64_t)q1.y << 32), d3 = q1.z | ((uint64_t)q1.w << 32);
-                if (d0 | d1 | d2 | d3) {
-                    bm4[2 * tid] = make_uint4(0, 0, 0, 0);
-                    bm4[2 * tid + 1] = make_uint4(0, 0, 0, 0);
-                    int32_t* out = C_col + base + (S.pref[8 * tid]);
-                    int32_t cb = (int32_t)(lo + (int64_t)tid * 256);
-                    while (d0 | d1 | d2 | d3) {
-                        if (d0 == 0) { d0 = d1; d1 = d2; d2 = d3; d3 = 0; cb += 64; continue; }
-                        *out++ = cb + __ffsll((long long)d0) - 1;
-                        d0 &= d0 - 1;
-                    }
-                }
+                bm4[2 * tid] = make_uint4(0, 0, 0, 0);
+                bm4[2 * tid + 1] = make_uint4(0, 0, 0, 0);
             }
             __syncthreads();
             mark(6);
