@@ -8,7 +8,8 @@
 // Numeric, per range [lo, hi): pass 1 rebuilds the range's bitmap, a block scan turns word
 // popcounts into a rank prefix, pass 2 accumulates every product into a COMPACT fp64 array at
 // rank(c) = prefix[word] + popc(word & below) — a rank-indexed dense accumulator: no hashing, no
-// probing, and the emission (bitmap scan + contiguous value copy) is sorted by construction.
+// probing, and the output is sorted by construction: C.col[rank] is written by the product that
+// finds the accumulator at 0.0 (the first arrival), C.val by a coalesced copy of the array.
 // Products are flattened over the whole block (one k per thread, block scan of segment lengths,
 // per-product binary search), so rows with few k (median 9 on R-MAT) still use every warp.
 // Per-k cursors advance monotonically across ranges; B rows longer than LONG_ROW locate their
@@ -438,33 +439,17 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
             }
             __syncthreads();
             mark(4);
-            // ---- pass 2: columns of the range, then every product accumulated at rank(c) ----
+            // ---- pass 2: every product accumulated at rank(c); the column is written on first arrival ----
             const int64_t base = crow + R.off;
-            // columns first: thread t owns words [8t, 8t+8) (the prefix layout); its entries are the
-            // consecutive ranks from pref[8t], written lowest bit first from four 64-bit registers.
-            // The loop is instruction-bound and divergent; placed here it overlaps the gather
-            // latency of the other warps' products instead of ending in a barrier of its own.
-            {
-                const uint4* bm4 = reinterpret_cast<const uint4*>(S.bm);
-                const uint4 q0 = bm4[2 * tid], q1 = bm4[2 * tid + 1];
-                uint64_t d0 = q0.x | ((uint64_t)q0.y << 32), d1 = q0.z | ((uint64_t)q0.w << 32);
-                uint64_t d2 = q1.x | ((uint64_t)q1.y << 32), d3 = q1.z | ((uint64_t)q1.w << 32);
-                if (d0 | d1 | d2 | d3) {
-                    int32_t* out = C_col + base + S.pref[8 * tid];
-                    int32_t cb = (int32_t)(lo + (int64_t)tid * 256);
-                    while (d0 | d1 | d2 | d3) {
-                        if (d0 == 0) { d0 = d1; d1 = d2; d2 = d3; d3 = 0; cb += 64; continue; }
-                        *out++ = cb + __ffsll((long long)d0) - 1;
-                        d0 &= d0 - 1;
-                    }
-                }
-            }
             auto acc = [&](int32_t c, double v) {
                 if (c < 0) return;
                 const uint32_t d = (uint32_t)(c - lo);
                 const uint32_t wv = S.bm[d >> 5];
                 const int rank = S.pref[d >> 5] + __popc(wv & ((1u << (d & 31)) - 1u));
-                atomicAdd(&S.vals[rank], v);
+                // the product that finds the accumulator at exactly 0.0 writes the column: the first
+                // product of every column does (accumulators start at 0.0); a later one only when the
+                // partial sum is exactly 0.0, rewriting the same value
+                if (atomicAdd(&S.vals[rank], v) == 0.0) C_col[base + rank] = c;
             };
             if (inreg) {
                 #pragma unroll
