@@ -528,23 +528,24 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
         const char* dbe = getenv("SG_DEBUG_HEAVY");
         unsigned long long* dbg = nullptr;
         if (dbe && dbe[0] == '1') {
-            CKP(pl, cudaMallocAsync((void**)&dbg, 9 * sizeof(unsigned long long), s));
-            CKP(pl, cudaMemsetAsync(dbg, 0, 9 * sizeof(unsigned long long), s));
+            CKP(pl, cudaMallocAsync((void**)&dbg, 17 * sizeof(unsigned long long), s));
+            CKP(pl, cudaMemsetAsync(dbg, 0, 17 * sizeof(unsigned long long), s));
             const char* blk = getenv("SG_DEBUG_BLOCKS");  // results invalid: profiling experiments only
             unsigned long long nb = blk ? strtoull(blk, nullptr, 10) : 0ull;
-            CKP(pl, cudaMemcpyAsync(dbg + 8, &nb, sizeof(nb), cudaMemcpyHostToDevice, s));
+            CKP(pl, cudaMemcpyAsync(dbg + 16, &nb, sizeof(nb), cudaMemcpyHostToDevice, s));
         }
         CKP(pl, launch_num_heavy(a, b, pl->heavy, pl->nheavy, pl->rb, pl->range_off, pl->nranges, pl->ranges,
                                  pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter, pl->gscr, pl->amax, s,
                                  dbg));
         if (dbg) {
-            unsigned long long h[8];
+            unsigned long long h[16];
             CKP(pl, cudaMemcpyAsync(h, dbg, sizeof(h), cudaMemcpyDeviceToHost, s));
             CKP(pl, cudaStreamSynchronize(s));
             cudaFreeAsync(dbg, s);
             fprintf(stderr, "[sg heavy] Mcycles (sum over CTAs): fetch %.1f init %.1f seg+compact %.1f pass1 %.1f "
-                            "prefix %.1f pass2 %.1f emit %.1f | ranges %llu\n",
-                    h[0] / 1e6, h[1] / 1e6, h[2] / 1e6, h[3] / 1e6, h[4] / 1e6, h[5] / 1e6, h[6] / 1e6, h[7]);
+                            "prefix %.1f pass2 %.1f emit %.1f | ranges %llu | extra %.1f %.1f %.1f %.1f\n",
+                    h[0] / 1e6, h[1] / 1e6, h[2] / 1e6, h[3] / 1e6, h[4] / 1e6, h[5] / 1e6, h[6] / 1e6, h[7],
+                    h[8] / 1e6, h[9] / 1e6, h[10] / 1e6, h[11] / 1e6);
         }
     }
     return SG_OK;

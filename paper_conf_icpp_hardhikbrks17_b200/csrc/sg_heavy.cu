@@ -286,7 +286,7 @@ cudaError_t launch_sym_heavy(const Mat& A, const Mat& B, const int32_t* list, in
 // ------------------------------------------------------------------------------------------------
 struct HeavySmem {
     uint32_t bm[RW_WORDS];       // 32 KB  range bitmap
-    double vals[RCAP];           // 128 KB compact accumulator (by rank); int32 column staging at emission
+    double vals[RCAP + 2];       // 128 KB compact accumulator: rank r at vals[r + sh], sh = C offset parity
     uint16_t pref[RW_WORDS];     // 16 KB  rank prefix per bitmap word
     int32_t s_beg[KC];           // packed chunk entries: segment begin (B position)
     int32_t s_off[KC];           //                       exclusive prefix of segment lengths
@@ -299,6 +299,16 @@ struct HeavySmem {
     long long wsll[33];
     int ws[33];
 };
+
+// fp64 values leave shared memory by a bulk async copy (TMA engine, no LSU traffic)
+__device__ __forceinline__ void bulk_s2g(void* gdst, const void* ssrc, uint32_t bytes) {
+    const uint32_t sa = (uint32_t)__cvta_generic_to_shared(ssrc);
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(gdst), "r"(sa), "r"(bytes) : "memory");
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 
 // Segment of one k entry for tiles [.., t1) starting at its cursor: long B rows read the tile
 // pointer (prefetched `tpv`), short rows (<= LONG_ROW entries) count their entries below hi with
@@ -320,7 +330,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
     VT* __restrict__ C_val, unsigned long long* counter, int4* __restrict__ gscr, int64_t amax,
     unsigned long long* __restrict__ dbg) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    unsigned long long tph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    unsigned long long tph[12] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
     long long t_last = clock64();
     auto mark = [&](int k) { if (dbg && threadIdx.x == 0) { long long t = clock64(); tph[k] += t - t_last; t_last = t; } };
     HeavySmem& S = *reinterpret_cast<HeavySmem*>(smem_raw);
@@ -329,7 +339,9 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
     const int64_t p = B.ncols;
     int4* gs = gscr + (int64_t)blockIdx.x * amax;  // multi-chunk rows: per-k (cur, -, beg, len)
     for (int q = tid; q < RW_WORDS; q += NUM_T) S.bm[q] = 0u;
-    for (int q = tid; q < RCAP; q += NUM_T) S.vals[q] = 0.0;
+    for (int q = tid; q < RCAP + 2; q += NUM_T) S.vals[q] = 0.0;
+    constexpr bool kBulk = sizeof(VT) == 8;  // fp64 output: accumulator copied out by bulk async copy
+    int clear_n = 0;                          // accumulator entries still to be cleared (bulk path)
     while (true) {
         if (tid == 0) s_j = (long long)atomicAdd(counter, 1ull);
         __syncthreads();
@@ -368,7 +380,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
             const RangeRec R = Rn;
             if (ri + 1 < nr) Rn = rr[ri + 1];
             // debug (SG_DEBUG_BLOCKS=b): only the first b column blocks (later ranges never feed cursors)
-            if (dbg && dbg[8] != 0 && (unsigned long long)(R.t0 / RW_TILES) >= dbg[8]) break;
+            if (dbg && dbg[16] != 0 && (unsigned long long)(R.t0 / RW_TILES) >= dbg[16]) break;
             const int64_t lo = (int64_t)R.t0 * TW, hi = min(p, (int64_t)R.t1 * TW);
             int tot1 = 0, nk1 = 0;
             bool inreg = false;
@@ -427,7 +439,12 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 const int c0 = __popc(q0.x), c1 = __popc(q0.y), c2 = __popc(q0.z), c3 = __popc(q0.w);
                 const int c4 = __popc(q1.x), c5 = __popc(q1.y), c6 = __popc(q1.z), c7 = __popc(q1.w);
                 int t2;
+                if (kBulk && tid == 0) bulk_wait_read();  // previous range's values have left shared memory
                 const int p0 = block_scan<NUM_T>(c0 + c1 + c2 + c3 + c4 + c5 + c6 + c7, &t2, S.ws);
+                if (kBulk) {
+                    for (int e = tid; e < clear_n; e += NUM_T) S.vals[e] = 0.0;
+                    clear_n = 0;
+                }
                 const int p1 = p0 + c0, p2 = p1 + c1, p3 = p2 + c2, p4 = p3 + c3, p5 = p4 + c4, p6 = p5 + c5,
                           p7 = p6 + c6;
                 uint4 o;
@@ -441,6 +458,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
             mark(4);
             // ---- pass 2: every product accumulated at rank(c); the column is written on first arrival ----
             const int64_t base = crow + R.off;
+            const int sh = kBulk ? (int)(base & 1) : 0;  // vals[e + sh] and C_val[base + e] share 16 B alignment
             auto acc = [&](int32_t c, double v) {
                 if (c < 0) return;
                 const uint32_t d = (uint32_t)(c - lo);
@@ -449,7 +467,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 // the product that finds the accumulator at exactly 0.0 writes the column: the first
                 // product of every column does (accumulators start at 0.0); a later one only when the
                 // partial sum is exactly 0.0, rewriting the same value
-                if (atomicAdd(&S.vals[rank], v) == 0.0) C_col[base + rank] = c;
+                if (atomicAdd(&S.vals[rank + sh], v) == 0.0) C_col[base + rank] = c;
             };
             if (inreg) {
                 #pragma unroll
@@ -472,13 +490,26 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                     __syncthreads();
                 }
             }
+            if (kBulk) fence_proxy_async_smem();  // accumulator writes visible to the bulk copy
             __syncthreads();
             mark(5);
-            // ---- values by rank (coalesced); accumulator and bitmap cleared for the next range ----
+            // ---- values by rank; bitmap cleared for the next range ----
             const int cnt = R.cnt;
-            for (int e = tid; e < cnt; e += NUM_T) {
-                C_val[base + e] = (VT)S.vals[e];
-                S.vals[e] = 0.0;
+            if constexpr (kBulk) {
+                // one bulk copy of the 16 B-aligned body; head / tail doubles by plain stores. The
+                // accumulator is cleared in the next range's prefix phase, after the copy has read it.
+                const int e0 = sh, n2 = (cnt - e0) & ~1;
+                if (tid == 0 && n2 > 0) bulk_s2g(C_val + base + e0, &S.vals[e0 + sh], (uint32_t)n2 * 8u);
+                if (tid == 32) {
+                    if (sh && cnt > 0) C_val[base] = S.vals[sh];
+                    if (e0 + n2 < cnt) C_val[base + e0 + n2] = S.vals[e0 + n2 + sh];
+                }
+                clear_n = cnt + 1;
+            } else {
+                for (int e = tid; e < cnt; e += NUM_T) {
+                    C_val[base + e] = (VT)S.vals[e];
+                    S.vals[e] = 0.0;
+                }
             }
             {
                 uint4* bm4 = reinterpret_cast<uint4*>(S.bm);
@@ -489,8 +520,9 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
             mark(6);
         }
     }
+    if (kBulk && tid == 0) bulk_wait_all();
     if (dbg && threadIdx.x == 0)
-        for (int k = 0; k < 8; ++k) atomicAdd(&dbg[k], tph[k]);
+        for (int k = 0; k < 12; ++k) atomicAdd(&dbg[k], tph[k]);
 }
 
 cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, int64_t nheavy, int64_t rb,
