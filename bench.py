@@ -248,6 +248,7 @@ def main():
         thr, rep, cuts, W, plan, col, val, _g = step(A)
         info = plan.info()
         cls = plan.classes()
+        wrow = plan.work()
         rp_local = plan.row_ptr
         plan.destroy()
         del col, val
@@ -260,7 +261,12 @@ def main():
     nnzA_heavy = int(a_rows[cls == 2].sum().item())
     nnzA_light = int(a_rows[cls == 1].sum().item())
     nheavy = int((cls == 2).sum().item())
-    del cls, u, a_rows
+    # heavy rows split between the dense-window kernel (w >= 2^dense_log2) and the rank kernel
+    dmask = (cls == 2) & (wrow >= (1 << min(int(info["dense_log2"]), 62)))
+    ndense = int(dmask.sum().item())
+    nnzC_dense = int(u[dmask].sum().item())
+    nnzA_dense = int(a_rows[dmask].sum().item())
+    del cls, u, a_rows, wrow, dmask
     nnzC_total = nnz_local
     if world > 1:
         t = torch.tensor([nnz_local], device=dev, dtype=torch.int64)
@@ -306,7 +312,9 @@ def main():
     Bbytes = csr_bytes(H.nrows, H.nnz, vbytes)
     alg = {
         # compulsory bytes of one launch: its A rows, B once, its C entries
-        "k_num_heavy": 12 * nnzA_heavy + 8 * nheavy + Bbytes + (4 + vbytes) * nnzC_heavy,
+        "k_num_heavy": 12 * (nnzA_heavy - nnzA_dense) + 8 * (nheavy - ndense) + Bbytes
+                       + (4 + vbytes) * (nnzC_heavy - nnzC_dense),
+        "k_num_dense": 12 * nnzA_dense + 8 * ndense + Bbytes + (4 + vbytes) * nnzC_dense,
         "k_sym_heavy": 4 * nnzA_heavy + 8 * nheavy + 8 * (H.nrows + 1) + 4 * H.nnz,
     }
     dom = max(bk.items(), key=lambda kv: kv[1][1])[0] if bk else None
@@ -367,7 +375,7 @@ def main():
             "roofline": roof, "compulsory": compulsory, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": launches, "clocks": ck, "threshold_gap": gap,
             "kernel_share": {k: round(v, 4) for k, v in sorted(share.items(), key=lambda kv: -kv[1])},
-            "plan": {k: info[k] for k in ("n_empty", "n_light", "n_heavy", "n_ranges")},
+            "plan": {k: info[k] for k in ("n_empty", "n_light", "n_heavy", "n_ranges", "n_dense", "dense_log2")},
         }
         print(json.dumps(line), flush=True)
         if args.profile_out:

@@ -89,6 +89,8 @@ typedef struct {
     int64_t flops;            /* W = sum of w_i over the plan's rows (multiply-adds) */
     int64_t n_ranges;         /* heavy column ranges (numeric work items of the heavy path) */
     int64_t light_bins[13];   /* light rows per bin b: 2^(b-1) < w <= 2^b (b = 0: w == 1) */
+    int64_t n_dense;          /* heavy rows on the dense-window kernel (w >= 2^dense_log2) */
+    int64_t dense_log2;       /* that row-work bound (SG_DW_LOG2 overrides; >= 62: path disabled) */
 } sg_plan_info;
 
 typedef struct sg_plan sg_plan;   /* opaque; owns only its workspace */

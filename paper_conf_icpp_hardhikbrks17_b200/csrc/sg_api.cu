@@ -28,6 +28,8 @@ struct sg_plan {
     int32_t* nranges = nullptr;
     RangeRec* ranges = nullptr;
     int64_t nslots = 0, amax = 0;
+    int64_t ndw = 0;                // heavy[0, ndw): dense-window rows (w >= 2^dw_log2), sg_dense.cu
+    int dw_log2 = 0;
     int2* span = nullptr;           // light rows: [cmin, cmax] of the output columns
     int4* gscr = nullptr;           // heavy rows with more than KC entries: per-k cursor scratch
     int32_t* long_id = nullptr;
@@ -198,7 +200,7 @@ sg_status row_stats(const Mat& A, const Mat& B, const int64_t* rows, int64_t nr,
     unsigned long long* counter = (unsigned long long*)sc.get(sizeof(unsigned long long));
     if (!counter) return SG_ERR_OOM;
     CK(launch_sym_heavy(A, B, lists + off[BIN_HEAVY], cnt[BIN_HEAVY], rows, 0, rs.u, nullptr, nullptr, nullptr,
-                        counter, s));
+                        0, counter, s));
     return SG_OK;
 }
 
@@ -476,14 +478,22 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
         void* t2 = palloc(pl, scan_tmp_bytes(pl->nheavy));
         if (!pl->heavy || !hist || !pl->range_bounds || !pl->range_off || !pl->nranges || !t2) return fail(SG_ERR_OOM);
         CKF(launch_heavy_order(pl->lists + pl->bin_off[BIN_HEAVY], pl->nheavy, pl->w, hist, pl->heavy, s));
-        CKF(launch_range_bounds(pl->heavy, pl->nheavy, pl->w, pl->p, pl->range_bounds, s));
+        // dense-window rows: w >= 2^dw_log2, a prefix of the heaviest-first order
+        pl->dw_log2 = dense_window_log2(pl->p);
+        const int64_t dw_min_w = pl->dw_log2 >= 62 ? INT64_MAX : ((int64_t)1 << pl->dw_log2);
+        CKF(launch_range_bounds(pl->heavy, pl->nheavy, pl->w, pl->p, dw_min_w, pl->range_bounds, s));
         CKF(scan_exclusive(pl->range_bounds, pl->range_off, pl->nheavy, t2, s));
         CKF(cudaMemsetAsync(pl->counter + 1, 0, sizeof(unsigned long long), s));
         CKF(launch_max_a(a, pl->heavy, pl->nheavy, row_begin, pl->counter + 1, s));
         int64_t hb[2];
+        unsigned int hh[64];
         CKF(cudaMemcpyAsync(&hb[0], pl->range_off + pl->nheavy, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
         CKF(cudaMemcpyAsync(&hb[1], pl->counter + 1, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        CKF(cudaMemcpyAsync(hh, hist, sizeof(hh), cudaMemcpyDeviceToHost, s));
         CKF(cudaStreamSynchronize(s));
+        // heavy order bucket b = 62 - floor(log2 w) (ascending = heaviest first): w >= 2^m <=> b <= 62 - m
+        pl->ndw = 0;
+        for (int hb2 = 0; hb2 <= 62 - pl->dw_log2 && hb2 < 64; ++hb2) pl->ndw += hh[hb2];
         pl->nslots = hb[0];
         pl->amax = hb[1];
         pl->ranges = (RangeRec*)palloc(pl, sizeof(RangeRec) * (size_t)(pl->nslots > 0 ? pl->nslots : 1));
@@ -499,7 +509,7 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
     for (int k = 0; k < NBIN_LIGHT; ++k)
         CKF(launch_sym_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], nullptr, row_begin, pl->u, pl->span, s));
     CKF(launch_sym_heavy(a, b, pl->heavy, pl->nheavy, nullptr, row_begin, pl->u, pl->range_off, pl->ranges,
-                         pl->nranges, pl->counter, s));
+                         pl->nranges, pl->ndw, pl->counter, s));
     CKF(scan_exclusive(pl->u, C_row_ptr, nr, stmp, s));
     CKF(cudaMemcpyAsync(&pl->nnz_c, C_row_ptr + nr, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     CKF(cudaStreamSynchronize(s));
@@ -534,7 +544,24 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
             unsigned long long nb = blk ? strtoull(blk, nullptr, 10) : 0ull;
             CKP(pl, cudaMemcpyAsync(dbg + 16, &nb, sizeof(nb), cudaMemcpyHostToDevice, s));
         }
-        CKP(pl, launch_num_heavy(a, b, pl->heavy, pl->nheavy, pl->rb, pl->range_off, pl->nranges, pl->ranges,
+        if (dbg) {
+            unsigned long long* dd = nullptr;
+            CKP(pl, cudaMallocAsync((void**)&dd, 8 * sizeof(unsigned long long), s));
+            CKP(pl, cudaMemsetAsync(dd, 0, 8 * sizeof(unsigned long long), s));
+            CKP(pl, launch_num_dense(a, b, pl->heavy, pl->ndw, pl->rb, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
+                                     C_val, pl->counter, pl->gscr, pl->amax, s, dd));
+            unsigned long long h[8];
+            CKP(pl, cudaMemcpyAsync(h, dd, sizeof(h), cudaMemcpyDeviceToHost, s));
+            CKP(pl, cudaStreamSynchronize(s));
+            cudaFreeAsync(dd, s);
+            fprintf(stderr, "[sg dense] rows %lld Mcycles (sum over CTAs): fetch %.1f setup %.1f seg+compact %.1f "
+                            "products %.1f emit %.1f | windows %llu\n", (long long)pl->ndw,
+                    h[0] / 1e6, h[1] / 1e6, h[2] / 1e6, h[3] / 1e6, h[4] / 1e6, h[6]);
+        } else {
+            CKP(pl, launch_num_dense(a, b, pl->heavy, pl->ndw, pl->rb, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
+                                     C_val, pl->counter, pl->gscr, pl->amax, s));
+        }
+        CKP(pl, launch_num_heavy(a, b, pl->heavy, pl->ndw, pl->nheavy, pl->rb, pl->range_off, pl->nranges, pl->ranges,
                                  pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter, pl->gscr, pl->amax, s,
                                  dbg));
         if (dbg) {
@@ -561,6 +588,8 @@ sg_status sg_plan_get_info(const sg_plan* pl, sg_plan_info* out) {
     for (int k = 0; k < NBIN_LIGHT; ++k) { out->light_bins[k] = pl->bin_cnt[k]; out->n_light += pl->bin_cnt[k]; }
     out->nnz_c = pl->nnz_c;
     out->n_ranges = pl->nslots;
+    out->n_dense = pl->ndw;
+    out->dense_log2 = pl->dw_log2;
     // flops on demand
     if (pl->nr > 0) {
         cudaStream_t s = pl->s;

@@ -1,0 +1,219 @@
+// sg_dense.cu — the densest HEAVY rows (w_i >= 2^dw_log2 > thr; PAPER L272-L274 routes them to the
+// heavy path): a single-pass DENSE-WINDOW numeric.
+//
+// One CTA (1024 threads) per row, rows heaviest-first from a dynamic counter. The row's column
+// space is swept in windows of WD = 16384 columns; the accumulator is a dense fp64 array indexed by
+// column (vals[c - lo]): no bitmap pre-pass and no rank lookup per product (the rank-mode kernel in
+// sg_heavy.cu needs both). The product that finds vals[c - lo] at exactly 0.0 (the first arrival)
+// marks bit (c - lo) of a 512-word occupancy bitmap; the window's entries are then emitted in column
+// order (sorted by construction): one block scan of half-word popcounts, each thread writing its own
+// set bits; only the emitted slots are cleared.
+//
+// Per-k cursors advance monotonically window by window: B rows longer than LONG_ROW read their end
+// from the tile-pointer table tp (prefetched one window ahead), short rows keep their <= LONG_ROW
+// columns in shared memory (one load per entry per row, not per window).
+#include "sg_device.cuh"
+#include <cstdlib>
+
+namespace sg {
+
+constexpr int DW_T = 1024;              // threads per CTA, one CTA per SM
+constexpr int DW_TILES = 2;             // TW tiles per window
+constexpr int WD = DW_TILES * TW;       // 16384 columns per window (128 KB fp64 accumulator)
+constexpr int DW_WORDS = WD / 32;       // 512 occupancy words
+constexpr int DKC = DW_T;               // k entries per chunk (one per thread)
+static_assert(DW_WORDS * 2 == DW_T, "emission: one half occupancy word per thread");
+
+struct DenseSmem {
+    double vals[WD];                // dense accumulator of the window
+    uint32_t bm[DW_WORDS];          // occupancy (set by the first arrival)
+    int32_t s_beg[DKC];             // packed chunk entries: segment begin (B position)
+    int32_t s_off[DKC];             //                       exclusive prefix of segment lengths
+    double s_a[DKC];                //                       a_ik
+    int32_t sc[LONG_ROW][DKC];      // short B rows of single-chunk rows: their columns ([q][k], INT_MAX pad)
+    long long wsll[33];
+    int ws[33];
+};
+
+template <class VT>
+__global__ void __launch_bounds__(DW_T, 1) k_num_dense(
+    Mat A, Mat B, const int32_t* __restrict__ heavy, int64_t ndw, int64_t rb, const int32_t* __restrict__ long_id,
+    const uint32_t* __restrict__ tp, int T, const int64_t* __restrict__ C_rp, int32_t* __restrict__ C_col,
+    VT* __restrict__ C_val, unsigned long long* counter, int4* __restrict__ gscr, int64_t amax,
+    unsigned long long* __restrict__ dbg) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    unsigned long long tph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    long long t_last = clock64();
+    auto mark = [&](int k) { if (dbg && threadIdx.x == 0) { long long t = clock64(); tph[k] += t - t_last; t_last = t; } };
+    DenseSmem& S = *reinterpret_cast<DenseSmem*>(smem_raw);
+    __shared__ long long s_j;
+    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+    const int64_t p = B.ncols;
+    const int nwin = (int)((p + WD - 1) / WD);
+    int4* gs = gscr + (int64_t)blockIdx.x * amax;  // multi-chunk rows: per-k cursor
+    for (int q = tid; q < WD; q += DW_T) S.vals[q] = 0.0;
+    for (int q = tid; q < DW_WORDS; q += DW_T) S.bm[q] = 0u;
+    while (true) {
+        if (tid == 0) s_j = (long long)atomicAdd(counter, 1ull);
+        __syncthreads();
+        const int64_t h = s_j;
+        __syncthreads();
+        if (h >= ndw) break;
+        mark(0);
+        const int64_t li = heavy[h];
+        const int64_t row = rb + li;
+        const int64_t s0 = __ldg(A.rp + row), s1 = __ldg(A.rp + row + 1);
+        const int na = (int)(s1 - s0);
+        const bool single = na <= DKC;
+        int64_t pos = C_rp[li];
+        // per-k state of single-chunk rows: thread tid owns k entry tid
+        int cur = 0, q0 = 0, lid = -1;
+        uint32_t tpv = 0;
+        double a = 0.0;
+        if (single) {
+            if (tid < na) {
+                const int k = __ldg(A.col + s0 + tid);
+                q0 = (int)__ldg(B.rp + k);
+                const int len = (int)(__ldg(B.rp + k + 1) - q0);
+                cur = q0;
+                a = ldv<VT>(A.val, s0 + tid);
+                if (len > LONG_ROW) {
+                    lid = __ldg(long_id + k);
+                    tpv = __ldg(tp + (int64_t)lid * (T + 1) + min(DW_TILES, T));
+                } else {
+                    #pragma unroll
+                    for (int q = 0; q < LONG_ROW; ++q) S.sc[q][tid] = q < len ? __ldg(B.col + q0 + q) : INT_MAX;
+                }
+            }
+        } else {
+            for (int i = tid; i < na; i += DW_T) {
+                const int k = __ldg(A.col + s0 + i);
+                gs[i] = make_int4((int)__ldg(B.rp + k), 0, 0, 0);
+            }
+        }
+        mark(1);
+        for (int t = 0; t < nwin; ++t) {
+            const int64_t lo = (int64_t)t * WD, hi = min(p, lo + WD);
+            const int th = min((t + 1) * DW_TILES, T);  // tile index of hi
+            auto acc = [&](int32_t c, double v) {
+                if (c < 0) return;
+                const uint32_t d = (uint32_t)(c - lo);
+                // first arrival (accumulator at exactly 0.0) marks the column; a later product that finds
+                // an exact 0.0 partial sum re-marks it (idempotent)
+                if (atomicAdd(&S.vals[d], v) == 0.0) atomicOr(&S.bm[d >> 5], 1u << (d & 31));
+            };
+            int any = 0;
+            if (single) {
+                int len = 0;
+                const int beg = cur;
+                if (tid < na) {
+                    int end;
+                    if (lid >= 0) {
+                        end = q0 + (int)tpv;
+                        if (t + 1 < nwin) tpv = __ldg(tp + (int64_t)lid * (T + 1) + min((t + 2) * DW_TILES, T));
+                    } else {
+                        int n = 0;
+                        #pragma unroll
+                        for (int q = 0; q < LONG_ROW; ++q) n += S.sc[q][tid] < hi;
+                        end = q0 + n;
+                    }
+                    len = end - cur;
+                    cur = end;
+                }
+                int nk;
+                any = chunk_compact<DW_T, int32_t>(len, beg, a, S.s_beg, S.s_off, S.s_a, &nk, S.wsll);
+                mark(2);
+                if (any == 0) continue;  // block-uniform: nothing in this window
+                warp_slice<DW_T, true, VT, int32_t>(S.s_beg, S.s_off, S.s_a, nk, any, B, acc);
+            } else {
+                for (int c0 = 0; c0 < na; c0 += DKC) {
+                    const int i = c0 + tid;
+                    int len = 0, beg = 0;
+                    double ai = 0.0;
+                    if (i < na) {
+                        const int4 g = gs[i];
+                        const int k = __ldg(A.col + s0 + i);
+                        const int32_t kq0 = (int32_t)__ldg(B.rp + k), e1 = (int32_t)__ldg(B.rp + k + 1);
+                        const bool lng = e1 - kq0 > LONG_ROW;
+                        const uint32_t tv = lng ? __ldg(tp + (int64_t)__ldg(long_id + k) * (T + 1) + th) : 0u;
+                        const int end = seg_end(B, g.x, e1, kq0, lng, tv, hi);
+                        beg = g.x;
+                        len = end - g.x;
+                        if (len > 0) ai = ldv<VT>(A.val, s0 + i);
+                        gs[i] = make_int4(end, 0, 0, 0);
+                    }
+                    int nk;
+                    const int ctot = chunk_compact<DW_T, int32_t>(len, beg, ai, S.s_beg, S.s_off, S.s_a, &nk, S.wsll);
+                    if (ctot > 0) warp_slice<DW_T, true, VT, int32_t>(S.s_beg, S.s_off, S.s_a, nk, ctot, B, acc);
+                    any += ctot;
+                }
+                if (any == 0) continue;
+            }
+            if (dbg && tid == 0) tph[6] += 1;
+            __syncthreads();  // every product of the window accumulated
+            mark(3);
+            // ---- emission: thread tid owns 16 columns (half of occupancy word tid/2); one block scan
+            // of the half-word popcounts places every run; each thread writes its set bits in order ----
+            const uint32_t hw = (S.bm[tid >> 1] >> ((tid & 1) * 16)) & 0xFFFFu;
+            int wtot;
+            const int ex = block_scan1<DW_T, int>(__popc(hw), &wtot, S.ws);
+            if ((tid & 1) == 0) S.bm[tid >> 1] = 0u;  // both halves were read before the scan's barrier
+            {
+                uint32_t m = hw;
+                int64_t at = pos + ex;
+                const int ebase = tid * 16;
+                while (m) {
+                    const int e = ebase + __ffs(m) - 1;
+                    m &= m - 1u;
+                    C_col[at] = (int32_t)(lo + e);
+                    C_val[at] = (VT)S.vals[e];
+                    S.vals[e] = 0.0;
+                    ++at;
+                }
+            }
+            pos += wtot;
+            mark(4);
+            // the next window's chunk_compact barriers order these clears before its products
+        }
+    }
+    if (dbg && threadIdx.x == 0)
+        for (int k = 0; k < 8; ++k) atomicAdd(&dbg[k], tph[k]);
+}
+
+cudaError_t launch_num_dense(const Mat& A, const Mat& B, const int32_t* heavy, int64_t ndw, int64_t rb,
+                             const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
+                             void* C_val, unsigned long long* counter, int4* gscr, int64_t amax, cudaStream_t s,
+                             unsigned long long* dbg) {
+    if (ndw <= 0) return cudaSuccess;
+    const int smem = (int)sizeof(DenseSmem);
+    cudaError_t e = cudaMemsetAsync(counter, 0, sizeof(unsigned long long), s);
+    if (e != cudaSuccess) return e;
+    const int grid = (int)(ndw < 148 ? ndw : 148);
+    if (A.dt == 0) {
+        if ((e = cudaFuncSetAttribute(k_num_dense<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
+        SG_LAUNCH("k_num_dense", s, (k_num_dense<double><<<grid, DW_T, smem, s>>>(A, B, heavy, ndw, rb, long_id, tp, T, C_rp,
+                                                                                  C_col, (double*)C_val, counter, gscr, amax, dbg)));
+    } else {
+        if ((e = cudaFuncSetAttribute(k_num_dense<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
+        SG_LAUNCH("k_num_dense", s, (k_num_dense<float><<<grid, DW_T, smem, s>>>(A, B, heavy, ndw, rb, long_id, tp, T, C_rp,
+                                                                                 C_col, (float*)C_val, counter, gscr, amax, dbg)));
+    }
+    return cudaGetLastError();
+}
+
+int dense_window_cols() { return WD; }
+
+}  // namespace sg
+
+namespace sg {
+// Rows with w >= 2^m take the dense-window kernel. Its fixed cost grows with the number of windows
+// (p / WD) while its saving over the rank kernel grows with w, so m tracks log2 p: 2^18 at p = 2^20 (measured best of 2^16..2^20 on R-MAT 20).
+int dense_window_log2(int64_t p) {
+    const char* e = getenv("SG_DW_LOG2");
+    if (e && *e) return atoi(e);
+    int lp = 0;
+    while (lp < 62 && ((int64_t)1 << lp) < p) ++lp;
+    const int m = lp - 2;
+    return m < 4 ? 4 : m;
+}
+}  // namespace sg

@@ -362,4 +362,16 @@ __device__ __forceinline__ bool warp_slice_regs(const BEG* s_beg, const int* s_o
     return true;
 }
 
+// Segment of one k entry for tiles [.., t1) starting at its cursor: long B rows read the tile
+// pointer (prefetched `tpv`), short rows (<= LONG_ROW entries) count their entries below hi with
+// independent loads. Returns the new cursor.
+__device__ __forceinline__ int seg_end(const Mat& B, int cur, int e1, int q0, bool is_long, uint32_t tpv, int64_t hi) {
+    if (is_long) return q0 + (int)tpv;
+    int n = 0;
+    #pragma unroll
+    for (int q = 0; q < LONG_ROW; ++q)
+        if (cur + q < e1 && __ldg(B.col + cur + q) < hi) ++n;
+    return cur + n;
+}
+
 }  // namespace sg

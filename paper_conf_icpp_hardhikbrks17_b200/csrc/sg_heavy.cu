@@ -122,10 +122,11 @@ cudaError_t launch_heavy_order(const int32_t* heavy, int64_t nh, const int64_t* 
 
 // per heavy row: an upper bound on its range count
 __global__ void k_range_bounds(const int32_t* __restrict__ heavy, int64_t nh, const int64_t* __restrict__ w,
-                               int64_t p, int64_t* __restrict__ bounds) {
+                               int64_t p, int64_t dw_min_w, int64_t* __restrict__ bounds) {
     int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (j >= nh) return;
     int64_t wi = w[heavy[j]];
+    if (wi >= dw_min_w) { bounds[j] = 0; return; }  // dense-window row (sg_dense.cu): no range plan
     int64_t mu = wi < p ? wi : p;
     int64_t T = (p + TW - 1) / TW;
     int64_t nwin = (p + WIN - 1) / WIN;
@@ -134,10 +135,10 @@ __global__ void k_range_bounds(const int32_t* __restrict__ heavy, int64_t nh, co
     bounds[j] = b < T ? b : T;
 }
 
-cudaError_t launch_range_bounds(const int32_t* heavy, int64_t nh, const int64_t* w, int64_t p, int64_t* bounds,
-                                cudaStream_t s) {
+cudaError_t launch_range_bounds(const int32_t* heavy, int64_t nh, const int64_t* w, int64_t p, int64_t dw_min_w,
+                                int64_t* bounds, cudaStream_t s) {
     if (nh <= 0) return cudaSuccess;
-    SG_LAUNCH("k_range_bounds", s, (k_range_bounds<<<(unsigned)((nh + 255) / 256), 256, 0, s>>>(heavy, nh, w, p, bounds)));
+    SG_LAUNCH("k_range_bounds", s, (k_range_bounds<<<(unsigned)((nh + 255) / 256), 256, 0, s>>>(heavy, nh, w, p, dw_min_w, bounds)));
     return cudaGetLastError();
 }
 
@@ -149,7 +150,7 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_sym_heavy(Mat A, Mat B, co
                                                                  int64_t rb, int64_t* __restrict__ u,
                                                                  const int64_t* __restrict__ range_off,
                                                                  RangeRec* __restrict__ ranges,
-                                                                 int32_t* __restrict__ nranges,
+                                                                 int32_t* __restrict__ nranges, int64_t ndw,
                                                                  unsigned long long* counter) {
     extern __shared__ uint32_t bm[];  // WIN/32 words
     __shared__ int64_t s_beg[KCS];
@@ -210,7 +211,12 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_sym_heavy(Mat A, Mat B, co
             __syncthreads();
             // range plan (warp 0): key(t) = (ceil(P_t / RHALF) - 1, t / RW_TILES); a range is a run of
             // equal keys -> count <= RHALF + cnt(first tile) <= RCAP, width <= RW_TILES tiles.
-            if (wid == 0) {
+            if (wid == 0 && j < ndw) {  // dense-window row (sg_dense.cu): u only, no range plan
+                int c = 0;
+                for (int t = lane; t < nt; t += 32) c += tcnt[t];
+                c = warp_sum(c);
+                if (lane == 0) { s_nr = nr; s_u = utot + c; }
+            } else if (wid == 0) {
                 int c4[4], loc = 0;
                 #pragma unroll
                 for (int q = 0; q < 4; ++q) { const int t = 4 * lane + q; c4[q] = t < nt ? tcnt[t] : 0; loc += c4[q]; }
@@ -269,7 +275,7 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_sym_heavy(Mat A, Mat B, co
 
 cudaError_t launch_sym_heavy(const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, const int64_t* rowmap,
                              int64_t rb, int64_t* u, const int64_t* range_off, RangeRec* ranges, int32_t* nranges,
-                             unsigned long long* counter, cudaStream_t s) {
+                             int64_t ndw, unsigned long long* counter, cudaStream_t s) {
     if (cnt <= 0) return cudaSuccess;
     const int smem = (WIN / 32) * 4;
     cudaError_t e = cudaFuncSetAttribute(k_sym_heavy, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
@@ -277,7 +283,7 @@ cudaError_t launch_sym_heavy(const Mat& A, const Mat& B, const int32_t* list, in
     if ((e = cudaMemsetAsync(counter, 0, sizeof(unsigned long long), s)) != cudaSuccess) return e;
     const int grid = (int)(cnt < 148 ? cnt : 148);
     SG_LAUNCH("k_sym_heavy", s, (k_sym_heavy<<<grid, HEAVY_THREADS, smem, s>>>(A, B, list, cnt, rowmap, rb, u, range_off,
-                                                                                ranges, nranges, counter)));
+                                                                                ranges, nranges, ndw, counter)));
     return cudaGetLastError();
 }
 
@@ -310,21 +316,9 @@ __device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.w
 __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 __device__ __forceinline__ void fence_proxy_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 
-// Segment of one k entry for tiles [.., t1) starting at its cursor: long B rows read the tile
-// pointer (prefetched `tpv`), short rows (<= LONG_ROW entries) count their entries below hi with
-// independent loads. Returns the new cursor.
-__device__ __forceinline__ int seg_end(const Mat& B, int cur, int e1, int q0, bool is_long, uint32_t tpv, int64_t hi) {
-    if (is_long) return q0 + (int)tpv;
-    int n = 0;
-    #pragma unroll
-    for (int q = 0; q < LONG_ROW; ++q)
-        if (cur + q < e1 && __ldg(B.col + cur + q) < hi) ++n;
-    return cur + n;
-}
-
 template <class VT>
 __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
-    Mat A, Mat B, const int32_t* __restrict__ heavy, int64_t nheavy, int64_t rb, const int64_t* __restrict__ range_off,
+    Mat A, Mat B, const int32_t* __restrict__ heavy, int64_t h0, int64_t nheavy, int64_t rb, const int64_t* __restrict__ range_off,
     const int32_t* __restrict__ nranges, const RangeRec* __restrict__ ranges, const int32_t* __restrict__ long_id,
     const uint32_t* __restrict__ tp, int T, const int64_t* __restrict__ C_rp, int32_t* __restrict__ C_col,
     VT* __restrict__ C_val, unsigned long long* counter, int4* __restrict__ gscr, int64_t amax,
@@ -343,7 +337,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
     constexpr bool kBulk = sizeof(VT) == 8;  // fp64 output: accumulator copied out by bulk async copy
     int clear_n = 0;                          // accumulator entries still to be cleared (bulk path)
     while (true) {
-        if (tid == 0) s_j = (long long)atomicAdd(counter, 1ull);
+        if (tid == 0) s_j = h0 + (long long)atomicAdd(counter, 1ull);
         __syncthreads();
         const int64_t h = s_j;
         __syncthreads();
@@ -525,25 +519,26 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
         for (int k = 0; k < 12; ++k) atomicAdd(&dbg[k], tph[k]);
 }
 
-cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, int64_t nheavy, int64_t rb,
+cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, int64_t h0, int64_t nheavy, int64_t rb,
                              const int64_t* range_off, const int32_t* nranges, const RangeRec* ranges,
                              const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
                              void* C_val, unsigned long long* counter, int4* gscr, int64_t amax, cudaStream_t s,
                              unsigned long long* dbg) {
-    if (nheavy <= 0) return cudaSuccess;
+    if (nheavy - h0 <= 0) return cudaSuccess;
     const int smem = (int)sizeof(HeavySmem);
     cudaError_t e = cudaMemsetAsync(counter, 0, sizeof(unsigned long long), s);
     if (e != cudaSuccess) return e;
-    const int grid = (int)(nheavy < NUM_OCC * 148 ? nheavy : NUM_OCC * 148);
+    const int64_t nh = nheavy - h0;
+    const int grid = (int)(nh < NUM_OCC * 148 ? nh : NUM_OCC * 148);
     if (A.dt == 0) {
         if ((e = cudaFuncSetAttribute(k_num_heavy<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
         SG_LAUNCH("k_num_heavy", s, (k_num_heavy<double><<<grid, NUM_T, smem, s>>>(
-                                        A, B, heavy, nheavy, rb, range_off, nranges, ranges, long_id, tp, T, C_rp, C_col,
+                                        A, B, heavy, h0, nheavy, rb, range_off, nranges, ranges, long_id, tp, T, C_rp, C_col,
                                         (double*)C_val, counter, gscr, amax, dbg)));
     } else {
         if ((e = cudaFuncSetAttribute(k_num_heavy<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
         SG_LAUNCH("k_num_heavy", s, (k_num_heavy<float><<<grid, NUM_T, smem, s>>>(
-                                        A, B, heavy, nheavy, rb, range_off, nranges, ranges, long_id, tp, T, C_rp, C_col,
+                                        A, B, heavy, h0, nheavy, rb, range_off, nranges, ranges, long_id, tp, T, C_rp, C_col,
                                         (float*)C_val, counter, gscr, amax, dbg)));
     }
     return cudaGetLastError();

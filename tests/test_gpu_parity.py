@@ -338,3 +338,29 @@ def test_rmat22_multi_window_row_subset():
     R = oracle.spgemm(A, A, rows=pick, with_absmag=True)
     compare_rows(rp, col.cpu().numpy(), val.cpu().numpy(), R, "f64")
     plan.destroy()
+
+
+@pytest.mark.parametrize("dw", ["0", "99"])
+@pytest.mark.parametrize("name,thr", [("rmat12", 0), ("rmat16", 2048), ("C1", 16)])
+def test_dense_window_path_forced(monkeypatch, name, thr, dw):
+    """Every heavy row on the dense-window kernel (SG_DW_LOG2=0) or none (99): same C either way."""
+    monkeypatch.setenv("SG_DW_LOG2", dw)
+    A = gen.config(name)
+    (rp, col, val), info, _ = _full_product(A, A, thr)
+    R = oracle.spgemm(A, A, with_absmag=True)
+    assert np.array_equal(rp, R.row_ptr)
+    compare_rows(rp, col, val, R, "f64")
+    assert info["n_dense"] == (info["n_heavy"] if dw == "0" else 0)
+
+
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+def test_dense_window_integer_values_exact(monkeypatch, dtype):
+    """Dense-window accumulation in integer-value mode: values bit-exact (R11); includes
+    rows with more than 1024 k entries (multi-chunk) at R-MAT 16."""
+    monkeypatch.setenv("SG_DW_LOG2", "0")
+    A = gen.config("rmat16", mode="int", dtype=dtype)
+    (rp, col, val), info, _ = _full_product(A, A, 1024)
+    assert int(np.diff(A.row_ptr).max()) > 1024
+    R = oracle.spgemm(A, A, with_absmag=True)
+    compare_rows(rp, col, val, R, dtype, exact_values=True)
+    assert info["n_dense"] == info["n_heavy"] > 0
