@@ -119,6 +119,15 @@ sg_status sg_sample_threshold(const sg_csr_view* A, const sg_csr_view* B, double
                               const sg_cost_model* cm, int64_t* thr_out /*host*/,
                               sg_sample_report* rep /*host, nullable*/, void* stream);
 
+/* Identify on an EXPLICIT row sample (PAPER L87-L89 with a caller-chosen I_s): rows (device int64,
+ * nrows entries, each in [0, A.nrows); duplicates count twice) -> thr = the smallest minimiser of
+ * J(t; rows), exactly as sg_sample_threshold computes it on its Bernoulli sample. For the paper's
+ * sample-shape experiments: a predetermined sub-matrix vs a random one (L250, Fig. 7), sqrt(n) rows
+ * (L139, L287). Synchronises. Errors: INVALID_ARG (row id out of range), EMPTY_SAMPLE, SHAPE, DTYPE. */
+sg_status sg_threshold_on_rows(const sg_csr_view* A, const sg_csr_view* B, const int64_t* rows, int64_t nrows,
+                               const sg_cost_model* cm, int64_t* thr_out /*host*/, sg_sample_report* rep /*host, nullable*/,
+                               void* stream);
+
 /* The exhaustive threshold thr* = thr over ALL rows (needs u_i for every row, i.e. a full
  * symbolic pass — what the paper calls "not practical", L198, L246). Used for the gap report. */
 sg_status sg_exhaustive_threshold(const sg_csr_view* A, const sg_csr_view* B, const sg_cost_model* cm,

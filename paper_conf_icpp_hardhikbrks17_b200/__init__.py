@@ -23,7 +23,8 @@ from . import _build
 
 __all__ = [
     "DeviceCSR", "CostModel", "SampleReport", "PlanInfo", "SgError", "Plan", "lib", "load",
-    "sg_row_work", "sg_sample_rows", "sg_sample_threshold", "sg_exhaustive_threshold", "sg_cost_curve",
+    "sg_row_work", "sg_sample_rows", "sg_sample_threshold", "sg_threshold_on_rows", "sg_exhaustive_threshold",
+    "sg_cost_curve",
     "sg_partition", "sg_symbolic", "sg_numeric", "sg_gather", "sg_default_cost_model", "spgemm",
     "SG_CAP_L_MAX",
 ]
@@ -37,7 +38,7 @@ EXPORTS = ["sg_status_string", "sg_version", "sg_default_cost_model", "sg_row_wo
            "sg_exhaustive_threshold", "sg_cost_curve", "sg_partition", "sg_symbolic", "sg_numeric", "sg_gather",
            "sg_plan_get_info", "sg_plan_get_classes", "sg_plan_get_work", "sg_plan_destroy", "sg_sample_rows",
            "sg_profile_enable", "sg_launch_count", "sg_profile_count", "sg_profile_read", "sg_profile_reset",
-           "sg_gather_layout"]
+           "sg_gather_layout", "sg_threshold_on_rows"]
 
 
 class SgError(RuntimeError):
@@ -107,6 +108,7 @@ def load(build_if_missing: bool = True):
         "sg_row_work": (st, [V, V, i64, i64, P, pi64, P]),
         "sg_sample_rows": (st, [i64, i64, ctypes.c_double, u64, P, i64, pi64, P]),
         "sg_sample_threshold": (st, [V, V, ctypes.c_double, u64, CM, pi64, ctypes.POINTER(SampleReport), P]),
+        "sg_threshold_on_rows": (st, [V, V, P, i64, CM, pi64, ctypes.POINTER(SampleReport), P]),
         "sg_exhaustive_threshold": (st, [V, V, CM, pi64, pi64, P]),
         "sg_cost_curve": (st, [V, V, CM, i64, P, P, P]),
         "sg_partition": (st, [V, V, ctypes.c_int, P, pi64, P]),
@@ -228,6 +230,18 @@ def sg_sample_threshold(A: DeviceCSR, B: DeviceCSR, sample_frac: float, seed: in
     rep = SampleReport()
     _check(lib().sg_sample_threshold(ctypes.byref(A.view()), ctypes.byref(B.view()), sample_frac, seed, _cmref(cm),
                                      ctypes.byref(thr), ctypes.byref(rep), _stream()), "sg_sample_threshold")
+    return int(thr.value), rep.as_dict()
+
+
+def sg_threshold_on_rows(A: DeviceCSR, B: DeviceCSR, rows, cm: CostModel | None = None):
+    """Identify on an explicit row sample (device or host int64 row ids). Returns (thr, SampleReport dict)."""
+    _require_cuda()
+    r = torch.as_tensor(rows, dtype=torch.int64, device=A.row_ptr.device).contiguous()
+    thr = ctypes.c_int64(0)
+    rep = SampleReport()
+    _check(lib().sg_threshold_on_rows(ctypes.byref(A.view()), ctypes.byref(B.view()), ctypes.c_void_p(r.data_ptr()),
+                                      r.numel(), _cmref(cm), ctypes.byref(thr), ctypes.byref(rep), _stream()),
+           "sg_threshold_on_rows")
     return int(thr.value), rep.as_dict()
 
 

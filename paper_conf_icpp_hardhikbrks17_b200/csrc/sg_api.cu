@@ -29,6 +29,7 @@ struct sg_plan {
     RangeRec* ranges = nullptr;
     int64_t nslots = 0, amax = 0;
     int64_t ndw = 0;                // heavy[0, ndw): dense-window rows (w >= 2^dw_log2), sg_dense.cu
+    int32_t* dtc = nullptr;         // their per-tile output counts (ndw x T), from the symbolic pass
     int dw_log2 = 0;
     int2* span = nullptr;           // light rows: [cmin, cmax] of the output columns
     int4* gscr = nullptr;           // heavy rows with more than KC entries: per-k cursor scratch
@@ -200,7 +201,7 @@ sg_status row_stats(const Mat& A, const Mat& B, const int64_t* rows, int64_t nr,
     unsigned long long* counter = (unsigned long long*)sc.get(sizeof(unsigned long long));
     if (!counter) return SG_ERR_OOM;
     CK(launch_sym_heavy(A, B, lists + off[BIN_HEAVY], cnt[BIN_HEAVY], rows, 0, rs.u, nullptr, nullptr, nullptr,
-                        0, counter, s));
+                        0, nullptr, counter, s));
     return SG_OK;
 }
 
@@ -342,6 +343,43 @@ sg_status sg_sample_threshold(const sg_csr_view* A, const sg_csr_view* B, double
     *thr_out = r.thr;
     if (rep) {
         rep->sample_rows = ns;
+        rep->sample_nonempty = r.nonempty;
+        rep->thr = r.thr;
+        rep->W_est_L = r.W_L;
+        rep->W_est_H = r.W_all - r.W_L;
+        rep->J_min = r.Jmin;
+    }
+    return SG_OK;
+}
+
+sg_status sg_threshold_on_rows(const sg_csr_view* A, const sg_csr_view* B, const int64_t* rows, int64_t nrows,
+                               const sg_cost_model* cm, int64_t* thr_out, sg_sample_report* rep, void* stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    init_pool();
+    if (!thr_out || nrows < 0 || (nrows > 0 && !rows)) return SG_ERR_INVALID_ARG;
+    sg_status st = validate_pair(A, B, s);
+    if (st != SG_OK) return st;
+    const sg_cost_model* c = cm ? cm : &kDefaultModel;
+    if ((st = check_model(c)) != SG_OK) return st;
+    if (nrows == 0) return SG_ERR_EMPTY_SAMPLE;
+    {
+        Scratch sc(s);
+        unsigned long long* bad = (unsigned long long*)sc.get(sizeof(unsigned long long));
+        if (!bad) return SG_ERR_OOM;
+        unsigned long long hb = 0;
+        CK(cudaMemsetAsync(bad, 0, sizeof(unsigned long long), s));
+        CK(launch_check_rows(rows, nrows, A->nrows, bad, s));
+        CK(cudaMemcpyAsync(&hb, bad, sizeof(hb), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (hb) return SG_ERR_INVALID_ARG;
+    }
+    ThrResult r;
+    st = identify(mat_of(A), mat_of(B), rows, nrows, c, &r, s);
+    if (st != SG_OK) return st;
+    if (r.nonempty == 0) return SG_ERR_EMPTY_SAMPLE;
+    *thr_out = r.thr;
+    if (rep) {
+        rep->sample_rows = nrows;
         rep->sample_nonempty = r.nonempty;
         rep->thr = r.thr;
         rep->W_est_L = r.W_L;
@@ -494,6 +532,10 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
         // heavy order bucket b = 62 - floor(log2 w) (ascending = heaviest first): w >= 2^m <=> b <= 62 - m
         pl->ndw = 0;
         for (int hb2 = 0; hb2 <= 62 - pl->dw_log2 && hb2 < 64; ++hb2) pl->ndw += hh[hb2];
+        if (pl->ndw > 0) {
+            pl->dtc = (int32_t*)palloc(pl, sizeof(int32_t) * (size_t)pl->ndw * (size_t)pl->T);
+            if (!pl->dtc) return fail(SG_ERR_OOM);
+        }
         pl->nslots = hb[0];
         pl->amax = hb[1];
         pl->ranges = (RangeRec*)palloc(pl, sizeof(RangeRec) * (size_t)(pl->nslots > 0 ? pl->nslots : 1));
@@ -509,7 +551,7 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
     for (int k = 0; k < NBIN_LIGHT; ++k)
         CKF(launch_sym_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], nullptr, row_begin, pl->u, pl->span, s));
     CKF(launch_sym_heavy(a, b, pl->heavy, pl->nheavy, nullptr, row_begin, pl->u, pl->range_off, pl->ranges,
-                         pl->nranges, pl->ndw, pl->counter, s));
+                         pl->nranges, pl->ndw, pl->dtc, pl->counter, s));
     CKF(scan_exclusive(pl->u, C_row_ptr, nr, stmp, s));
     CKF(cudaMemcpyAsync(&pl->nnz_c, C_row_ptr + nr, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     CKF(cudaStreamSynchronize(s));
@@ -540,16 +582,13 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
         if (dbe && dbe[0] == '1') {
             CKP(pl, cudaMallocAsync((void**)&dbg, 17 * sizeof(unsigned long long), s));
             CKP(pl, cudaMemsetAsync(dbg, 0, 17 * sizeof(unsigned long long), s));
-            const char* blk = getenv("SG_DEBUG_BLOCKS");  // results invalid: profiling experiments only
-            unsigned long long nb = blk ? strtoull(blk, nullptr, 10) : 0ull;
-            CKP(pl, cudaMemcpyAsync(dbg + 16, &nb, sizeof(nb), cudaMemcpyHostToDevice, s));
         }
         if (dbg) {
             unsigned long long* dd = nullptr;
             CKP(pl, cudaMallocAsync((void**)&dd, 8 * sizeof(unsigned long long), s));
             CKP(pl, cudaMemsetAsync(dd, 0, 8 * sizeof(unsigned long long), s));
             CKP(pl, launch_num_dense(a, b, pl->heavy, pl->ndw, pl->rb, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
-                                     C_val, pl->counter, pl->gscr, pl->amax, s, dd));
+                                     C_val, pl->counter, pl->gscr, pl->amax, pl->dtc, s, dd));
             unsigned long long h[8];
             CKP(pl, cudaMemcpyAsync(h, dd, sizeof(h), cudaMemcpyDeviceToHost, s));
             CKP(pl, cudaStreamSynchronize(s));
@@ -559,7 +598,7 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
                     h[0] / 1e6, h[1] / 1e6, h[2] / 1e6, h[3] / 1e6, h[4] / 1e6, h[6]);
         } else {
             CKP(pl, launch_num_dense(a, b, pl->heavy, pl->ndw, pl->rb, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
-                                     C_val, pl->counter, pl->gscr, pl->amax, s));
+                                     C_val, pl->counter, pl->gscr, pl->amax, pl->dtc, s));
         }
         CKP(pl, launch_num_heavy(a, b, pl->heavy, pl->ndw, pl->nheavy, pl->rb, pl->range_off, pl->nranges, pl->ranges,
                                  pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter, pl->gscr, pl->amax, s,

@@ -40,14 +40,15 @@ __global__ void __launch_bounds__(DW_T, 1) k_num_dense(
     Mat A, Mat B, const int32_t* __restrict__ heavy, int64_t ndw, int64_t rb, const int32_t* __restrict__ long_id,
     const uint32_t* __restrict__ tp, int T, const int64_t* __restrict__ C_rp, int32_t* __restrict__ C_col,
     VT* __restrict__ C_val, unsigned long long* counter, int4* __restrict__ gscr, int64_t amax,
-    unsigned long long* __restrict__ dbg) {
+    const int32_t* __restrict__ dtc, unsigned long long* gclock, unsigned long long* __restrict__ dbg) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     unsigned long long tph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
     long long t_last = clock64();
     auto mark = [&](int k) { if (dbg && threadIdx.x == 0) { long long t = clock64(); tph[k] += t - t_last; t_last = t; } };
     DenseSmem& S = *reinterpret_cast<DenseSmem*>(smem_raw);
     __shared__ long long s_j;
-    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+    __shared__ int s_t0;
+    const int tid = threadIdx.x;
     const int64_t p = B.ncols;
     const int nwin = (int)((p + WD - 1) / WD);
     int4* gs = gscr + (int64_t)blockIdx.x * amax;  // multi-chunk rows: per-k cursor
@@ -65,8 +66,27 @@ __global__ void __launch_bounds__(DW_T, 1) k_num_dense(
         const int64_t s0 = __ldg(A.rp + row), s1 = __ldg(A.rp + row + 1);
         const int na = (int)(s1 - s0);
         const bool single = na <= DKC;
-        int64_t pos = C_rp[li];
-        // per-k state of single-chunk rows: thread tid owns k entry tid
+        // Phase-synchronised sweep: the row starts at the window the CTAs are currently at on average
+        // (windows completed by all CTAs / CTAs, mod nwin) and wraps around, so that concurrently
+        // running rows read the same column slice of B and it stays in L2 (B > L2 at R-MAT 20).
+        if (tid == 0) s_t0 = (int)((*(volatile unsigned long long*)gclock / gridDim.x) % (unsigned long long)nwin);
+        __syncthreads();
+        const int t0 = s_t0;
+        const int64_t lo0 = (int64_t)t0 * WD;
+        // output offset of window t0 inside the row: the row's tile counts below tile t0*DW_TILES
+        int64_t off0 = 0;
+        if (t0 > 0) {
+            long long c = 0;
+            const int te = min(t0 * DW_TILES, T);
+            for (int q = tid; q < te; q += DW_T) c += dtc[h * (int64_t)T + q];
+            long long tot;
+            block_scan_ll<DW_T>(c, &tot, S.wsll);
+            off0 = tot;
+            __syncthreads();  // every warp has read wsll before chunk_compact rewrites it
+        }
+        const int64_t rowbase = C_rp[li];
+        int64_t pos = rowbase + off0;
+        // per-k state of single-chunk rows: thread tid owns k entry tid; cursor at column lo0
         int cur = 0, q0 = 0, lid = -1;
         uint32_t tpv = 0;
         double a = 0.0;
@@ -75,24 +95,42 @@ __global__ void __launch_bounds__(DW_T, 1) k_num_dense(
                 const int k = __ldg(A.col + s0 + tid);
                 q0 = (int)__ldg(B.rp + k);
                 const int len = (int)(__ldg(B.rp + k + 1) - q0);
-                cur = q0;
                 a = ldv<VT>(A.val, s0 + tid);
                 if (len > LONG_ROW) {
                     lid = __ldg(long_id + k);
-                    tpv = __ldg(tp + (int64_t)lid * (T + 1) + min(DW_TILES, T));
+                    const uint32_t* tr = tp + (int64_t)lid * (T + 1);
+                    cur = q0 + (int)__ldg(tr + min(t0 * DW_TILES, T));
+                    tpv = __ldg(tr + min((t0 + 1) * DW_TILES, T));
                 } else {
+                    int n0 = 0;
                     #pragma unroll
-                    for (int q = 0; q < LONG_ROW; ++q) S.sc[q][tid] = q < len ? __ldg(B.col + q0 + q) : INT_MAX;
+                    for (int q = 0; q < LONG_ROW; ++q) {
+                        const int c = q < len ? __ldg(B.col + q0 + q) : INT_MAX;
+                        S.sc[q][tid] = c;
+                        n0 += c < lo0;
+                    }
+                    cur = q0 + n0;
                 }
             }
         } else {
             for (int i = tid; i < na; i += DW_T) {
                 const int k = __ldg(A.col + s0 + i);
-                gs[i] = make_int4((int)__ldg(B.rp + k), 0, 0, 0);
+                const int32_t kq0 = (int32_t)__ldg(B.rp + k), e1 = (int32_t)__ldg(B.rp + k + 1);
+                int c0 = kq0;
+                if (t0 > 0) {
+                    const bool lng = e1 - kq0 > LONG_ROW;
+                    const uint32_t tv = lng ? __ldg(tp + (int64_t)__ldg(long_id + k) * (T + 1) + min(t0 * DW_TILES, T)) : 0u;
+                    c0 = seg_end(B, kq0, e1, kq0, lng, tv, lo0);
+                }
+                gs[i] = make_int4(c0, 0, 0, 0);
             }
         }
         mark(1);
-        for (int t = 0; t < nwin; ++t) {
+        for (int j = 0; j < nwin; ++j) {
+            const int t = t0 + j < nwin ? t0 + j : t0 + j - nwin;
+            const int tn = t + 1 < nwin ? t + 1 : 0;  // next window in sweep order
+            if (tid == 0) atomicAdd(gclock, 1ull);
+            if (t == 0) pos = rowbase;                 // wrapped to the row's first window
             const int64_t lo = (int64_t)t * WD, hi = min(p, lo + WD);
             const int th = min((t + 1) * DW_TILES, T);  // tile index of hi
             auto acc = [&](int32_t c, double v) {
@@ -110,7 +148,7 @@ __global__ void __launch_bounds__(DW_T, 1) k_num_dense(
                     int end;
                     if (lid >= 0) {
                         end = q0 + (int)tpv;
-                        if (t + 1 < nwin) tpv = __ldg(tp + (int64_t)lid * (T + 1) + min((t + 2) * DW_TILES, T));
+                        if (j + 1 < nwin) tpv = __ldg(tp + (int64_t)lid * (T + 1) + min((tn + 1) * DW_TILES, T));
                     } else {
                         int n = 0;
                         #pragma unroll
@@ -118,7 +156,7 @@ __global__ void __launch_bounds__(DW_T, 1) k_num_dense(
                         end = q0 + n;
                     }
                     len = end - cur;
-                    cur = end;
+                    cur = tn == 0 ? q0 : end;
                 }
                 int nk;
                 any = chunk_compact<DW_T, int32_t>(len, beg, a, S.s_beg, S.s_off, S.s_a, &nk, S.wsll);
@@ -140,7 +178,7 @@ __global__ void __launch_bounds__(DW_T, 1) k_num_dense(
                         beg = g.x;
                         len = end - g.x;
                         if (len > 0) ai = ldv<VT>(A.val, s0 + i);
-                        gs[i] = make_int4(end, 0, 0, 0);
+                        gs[i] = make_int4(tn == 0 ? kq0 : end, 0, 0, 0);
                     }
                     int nk;
                     const int ctot = chunk_compact<DW_T, int32_t>(len, beg, ai, S.s_beg, S.s_off, S.s_a, &nk, S.wsll);
@@ -165,8 +203,8 @@ __global__ void __launch_bounds__(DW_T, 1) k_num_dense(
                 while (m) {
                     const int e = ebase + __ffs(m) - 1;
                     m &= m - 1u;
-                    C_col[at] = (int32_t)(lo + e);
-                    C_val[at] = (VT)S.vals[e];
+                    st_out(C_col + at, (int32_t)(lo + e));
+                    st_out(C_val + at, (VT)S.vals[e]);
                     S.vals[e] = 0.0;
                     ++at;
                 }
@@ -182,21 +220,21 @@ __global__ void __launch_bounds__(DW_T, 1) k_num_dense(
 
 cudaError_t launch_num_dense(const Mat& A, const Mat& B, const int32_t* heavy, int64_t ndw, int64_t rb,
                              const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
-                             void* C_val, unsigned long long* counter, int4* gscr, int64_t amax, cudaStream_t s,
-                             unsigned long long* dbg) {
+                             void* C_val, unsigned long long* counter, int4* gscr, int64_t amax,
+                             const int32_t* dtc, cudaStream_t s, unsigned long long* dbg) {
     if (ndw <= 0) return cudaSuccess;
     const int smem = (int)sizeof(DenseSmem);
-    cudaError_t e = cudaMemsetAsync(counter, 0, sizeof(unsigned long long), s);
+    cudaError_t e = cudaMemsetAsync(counter, 0, 2 * sizeof(unsigned long long), s);  // row counter, window clock
     if (e != cudaSuccess) return e;
     const int grid = (int)(ndw < 148 ? ndw : 148);
     if (A.dt == 0) {
         if ((e = cudaFuncSetAttribute(k_num_dense<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
         SG_LAUNCH("k_num_dense", s, (k_num_dense<double><<<grid, DW_T, smem, s>>>(A, B, heavy, ndw, rb, long_id, tp, T, C_rp,
-                                                                                  C_col, (double*)C_val, counter, gscr, amax, dbg)));
+                                                                                  C_col, (double*)C_val, counter, gscr, amax, dtc, counter + 1, dbg)));
     } else {
         if ((e = cudaFuncSetAttribute(k_num_dense<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
         SG_LAUNCH("k_num_dense", s, (k_num_dense<float><<<grid, DW_T, smem, s>>>(A, B, heavy, ndw, rb, long_id, tp, T, C_rp,
-                                                                                 C_col, (float*)C_val, counter, gscr, amax, dbg)));
+                                                                                 C_col, (float*)C_val, counter, gscr, amax, dtc, counter + 1, dbg)));
     }
     return cudaGetLastError();
 }

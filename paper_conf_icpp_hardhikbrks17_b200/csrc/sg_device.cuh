@@ -38,6 +38,19 @@ __device__ __forceinline__ unsigned lanemask_lt() {
     return m;
 }
 
+// C is written once and never re-read by the kernels: streaming stores (st.global.cs, evict-first
+// in L2) keep the 116 GB output stream from evicting B, the operand every product gathers.
+#ifndef SG_STCS
+#define SG_STCS 1
+#endif
+template <class T> __device__ __forceinline__ void st_out(T* p, T v) {
+#if SG_STCS
+    __stcs(p, v);
+#else
+    *p = v;
+#endif
+}
+
 template <class VT> __device__ __forceinline__ double ldv(const void* v, int64_t q) {
     return (double)__ldg(reinterpret_cast<const VT*>(v) + q);
 }
@@ -165,8 +178,8 @@ __device__ __forceinline__ void emit_slots(int32_t* keys, double* vals, int nslo
             const unsigned m = __ballot_sync(FULL, k != EMPTY_KEY);
             if (k != EMPTY_KEY) {
                 const int64_t o = pos + __popc(m & lanemask_lt());
-                C_col[o] = k;
-                C_val[o] = (VT)vals[s];
+                st_out(C_col + o, k);
+                st_out(C_val + o, (VT)vals[s]);
                 keys[s] = EMPTY_KEY;
                 vals[s] = 0.0;
             }
@@ -193,8 +206,8 @@ __device__ __forceinline__ void emit_slots(int32_t* keys, double* vals, int nslo
             int rank = 0;
             for (int j = rs; j < re; ++j) rank += keys[j] < k;
             const int64_t o = pos + __popc(m & lanemask_lt()) - (s - rs) + rank;
-            C_col[o] = k;
-            C_val[o] = (VT)vals[s];
+            st_out(C_col + o, k);
+            st_out(C_val + o, (VT)vals[s]);
         }
         pos += __popc(m);
     }

@@ -151,7 +151,7 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_sym_heavy(Mat A, Mat B, co
                                                                  const int64_t* __restrict__ range_off,
                                                                  RangeRec* __restrict__ ranges,
                                                                  int32_t* __restrict__ nranges, int64_t ndw,
-                                                                 unsigned long long* counter) {
+                                                                 int32_t* __restrict__ dtc, unsigned long long* counter) {
     extern __shared__ uint32_t bm[];  // WIN/32 words
     __shared__ int64_t s_beg[KCS];
     __shared__ int s_off[KCS];
@@ -211,9 +211,13 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_sym_heavy(Mat A, Mat B, co
             __syncthreads();
             // range plan (warp 0): key(t) = (ceil(P_t / RHALF) - 1, t / RW_TILES); a range is a run of
             // equal keys -> count <= RHALF + cnt(first tile) <= RCAP, width <= RW_TILES tiles.
-            if (wid == 0 && j < ndw) {  // dense-window row (sg_dense.cu): u only, no range plan
+            if (wid == 0 && j < ndw) {  // dense-window row (sg_dense.cu): u and its tile counts, no range plan
                 int c = 0;
-                for (int t = lane; t < nt; t += 32) c += tcnt[t];
+                const int64_t Tall = (p + TW - 1) / TW;
+                for (int t = lane; t < nt; t += 32) {
+                    c += tcnt[t];
+                    if (dtc) dtc[j * Tall + wlo / TW + t] = tcnt[t];
+                }
                 c = warp_sum(c);
                 if (lane == 0) { s_nr = nr; s_u = utot + c; }
             } else if (wid == 0) {
@@ -275,7 +279,7 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_sym_heavy(Mat A, Mat B, co
 
 cudaError_t launch_sym_heavy(const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, const int64_t* rowmap,
                              int64_t rb, int64_t* u, const int64_t* range_off, RangeRec* ranges, int32_t* nranges,
-                             int64_t ndw, unsigned long long* counter, cudaStream_t s) {
+                             int64_t ndw, int32_t* dtc, unsigned long long* counter, cudaStream_t s) {
     if (cnt <= 0) return cudaSuccess;
     const int smem = (WIN / 32) * 4;
     cudaError_t e = cudaFuncSetAttribute(k_sym_heavy, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
@@ -283,7 +287,7 @@ cudaError_t launch_sym_heavy(const Mat& A, const Mat& B, const int32_t* list, in
     if ((e = cudaMemsetAsync(counter, 0, sizeof(unsigned long long), s)) != cudaSuccess) return e;
     const int grid = (int)(cnt < 148 ? cnt : 148);
     SG_LAUNCH("k_sym_heavy", s, (k_sym_heavy<<<grid, HEAVY_THREADS, smem, s>>>(A, B, list, cnt, rowmap, rb, u, range_off,
-                                                                                ranges, nranges, ndw, counter)));
+                                                                                ranges, nranges, ndw, dtc, counter)));
     return cudaGetLastError();
 }
 
@@ -309,7 +313,14 @@ struct HeavySmem {
 // fp64 values leave shared memory by a bulk async copy (TMA engine, no LSU traffic)
 __device__ __forceinline__ void bulk_s2g(void* gdst, const void* ssrc, uint32_t bytes) {
     const uint32_t sa = (uint32_t)__cvta_generic_to_shared(ssrc);
+#if SG_STCS
+    uint64_t pol;  // C values: evict-first in L2 (see st_out)
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group.L2::cache_hint [%0], [%1], %2, %3;" ::"l"(gdst), "r"(sa),
+                 "r"(bytes), "l"(pol) : "memory");
+#else
     asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(gdst), "r"(sa), "r"(bytes) : "memory");
+#endif
     asm volatile("cp.async.bulk.commit_group;" ::: "memory");
 }
 __device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
@@ -334,7 +345,10 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
     int4* gs = gscr + (int64_t)blockIdx.x * amax;  // multi-chunk rows: per-k (cur, -, beg, len)
     for (int q = tid; q < RW_WORDS; q += NUM_T) S.bm[q] = 0u;
     for (int q = tid; q < RCAP + 2; q += NUM_T) S.vals[q] = 0.0;
-    constexpr bool kBulk = sizeof(VT) == 8;  // fp64 output: accumulator copied out by bulk async copy
+#ifndef SG_BULK
+#define SG_BULK 1
+#endif
+    constexpr bool kBulk = SG_BULK && sizeof(VT) == 8;  // fp64 output: accumulator copied out by bulk async copy
     int clear_n = 0;                          // accumulator entries still to be cleared (bulk path)
     while (true) {
         if (tid == 0) s_j = h0 + (long long)atomicAdd(counter, 1ull);
@@ -373,8 +387,6 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
         for (int ri = 0; ri < nr; ++ri) {
             const RangeRec R = Rn;
             if (ri + 1 < nr) Rn = rr[ri + 1];
-            // debug (SG_DEBUG_BLOCKS=b): only the first b column blocks (later ranges never feed cursors)
-            if (dbg && dbg[16] != 0 && (unsigned long long)(R.t0 / RW_TILES) >= dbg[16]) break;
             const int64_t lo = (int64_t)R.t0 * TW, hi = min(p, (int64_t)R.t1 * TW);
             int tot1 = 0, nk1 = 0;
             bool inreg = false;
@@ -391,8 +403,6 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                         const int end = seg_end(B, cur, S.c_end[i], S.c_q0[i], lid >= 0, tpv, hi);
                         beg = cur; len = end - cur; a = S.c_a[i];
                         S.c_cur[i] = end;
-                        // prefetch the next range's tile pointer (its latency hides behind this range)
-                        if (lid >= 0 && ri + 1 < nr) tpv = __ldg(tp + (int64_t)lid * (T + 1) + Rn.t1);
                     } else {
                         const int4 g = gs[i];
                         const int k = __ldg(A.col + s0 + i);
@@ -405,6 +415,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                     }
                 }
                 int nk;
+                mark(8);
                 const int ctot = chunk_compact<NUM_T, int32_t>(len, beg, a, S.s_beg, S.s_off, S.s_a, &nk, S.wsll);
                 mark(2);
                 auto setbit = [&](int32_t c, double) {
@@ -417,6 +428,12 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                     for (int r = 0; r < 4; ++r) setbit(rc[r], 0.0);
                 } else {
                     warp_slice<NUM_T, false, VT, int32_t>(S.s_beg, S.s_off, nullptr, nk, ctot, B, setbit);
+                }
+                // prefetch the next range's tile pointer (its latency hides behind this range; issued
+                // after pass 1 so that the next range record Rn has arrived)
+                if (single && i < na && ri + 1 < nr) {
+                    const int lid = S.c_lid[i];
+                    if (lid >= 0) tpv = __ldg(tp + (int64_t)lid * (T + 1) + Rn.t1);
                 }
                 tot1 = ctot;
                 nk1 = nk;
@@ -434,6 +451,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 const int c4 = __popc(q1.x), c5 = __popc(q1.y), c6 = __popc(q1.z), c7 = __popc(q1.w);
                 int t2;
                 if (kBulk && tid == 0) bulk_wait_read();  // previous range's values have left shared memory
+                mark(9);
                 const int p0 = block_scan<NUM_T>(c0 + c1 + c2 + c3 + c4 + c5 + c6 + c7, &t2, S.ws);
                 if (kBulk) {
                     for (int e = tid; e < clear_n; e += NUM_T) S.vals[e] = 0.0;
@@ -461,7 +479,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 // the product that finds the accumulator at exactly 0.0 writes the column: the first
                 // product of every column does (accumulators start at 0.0); a later one only when the
                 // partial sum is exactly 0.0, rewriting the same value
-                if (atomicAdd(&S.vals[rank + sh], v) == 0.0) C_col[base + rank] = c;
+                if (atomicAdd(&S.vals[rank + sh], v) == 0.0) st_out(C_col + base + rank, c);
             };
             if (inreg) {
                 #pragma unroll
@@ -495,13 +513,13 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 const int e0 = sh, n2 = (cnt - e0) & ~1;
                 if (tid == 0 && n2 > 0) bulk_s2g(C_val + base + e0, &S.vals[e0 + sh], (uint32_t)n2 * 8u);
                 if (tid == 32) {
-                    if (sh && cnt > 0) C_val[base] = S.vals[sh];
-                    if (e0 + n2 < cnt) C_val[base + e0 + n2] = S.vals[e0 + n2 + sh];
+                    if (sh && cnt > 0) st_out(C_val + base, (VT)S.vals[sh]);
+                    if (e0 + n2 < cnt) st_out(C_val + base + e0 + n2, (VT)S.vals[e0 + n2 + sh]);
                 }
                 clear_n = cnt + 1;
             } else {
                 for (int e = tid; e < cnt; e += NUM_T) {
-                    C_val[base + e] = (VT)S.vals[e];
+                    st_out(C_val + base + e, (VT)S.vals[e]);
                     S.vals[e] = 0.0;
                 }
             }
@@ -510,6 +528,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 bm4[2 * tid] = make_uint4(0, 0, 0, 0);
                 bm4[2 * tid + 1] = make_uint4(0, 0, 0, 0);
             }
+            mark(10);
             __syncthreads();
             mark(6);
         }

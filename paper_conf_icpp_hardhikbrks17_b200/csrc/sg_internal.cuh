@@ -82,7 +82,8 @@ cudaError_t launch_range_bounds(const int32_t* heavy_list, int64_t nheavy, const
                                 int64_t dw_min_w, int64_t* bounds, cudaStream_t s);
 cudaError_t launch_sym_heavy(const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, const int64_t* rowmap,
                              int64_t rb, int64_t* u, const int64_t* range_off, RangeRec* ranges, int32_t* nranges,
-                             int64_t ndw, unsigned long long* counter, cudaStream_t s);
+                             int64_t ndw, int32_t* dtc /*ndw x T tile counts, nullable*/, unsigned long long* counter,
+                             cudaStream_t s);
 cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, int64_t h0, int64_t nheavy, int64_t rb,
                              const int64_t* range_off, const int32_t* nranges, const RangeRec* ranges,
                              const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
@@ -93,8 +94,8 @@ cudaError_t launch_max_a(const Mat& A, const int32_t* list, int64_t cnt, int64_t
 // dense-window heavy rows (sg_dense.cu): heavy[0, ndw), all with w >= 2^dense_window_log2(p)
 cudaError_t launch_num_dense(const Mat& A, const Mat& B, const int32_t* heavy, int64_t ndw, int64_t rb,
                              const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
-                             void* C_val, unsigned long long* counter, int4* gscr, int64_t amax, cudaStream_t s,
-                             unsigned long long* dbg = nullptr);
+                             void* C_val, unsigned long long* counter /*2 words*/, int4* gscr, int64_t amax,
+                             const int32_t* dtc, cudaStream_t s, unsigned long long* dbg = nullptr);
 int dense_window_cols();
 int dense_window_log2(int64_t p);  // SG_DW_LOG2 overrides (>= 62 disables the dense-window path)
 int heavy_kc();
@@ -111,5 +112,6 @@ cudaError_t launch_cost_curve(const CostModelD& cm, const int64_t* w, const int6
 cudaError_t launch_cuts(const int64_t* P, int64_t n, int G, int64_t* cuts, cudaStream_t s);
 cudaError_t launch_gather_rows(const int64_t* src, const int64_t* rows, int64_t nr, int64_t* dst, cudaStream_t s);
 cudaError_t launch_add_offset(int64_t* x, int64_t n, int64_t off, cudaStream_t s);
+cudaError_t launch_check_rows(const int64_t* rows, int64_t nr, int64_t n, unsigned long long* bad, cudaStream_t s);
 
 }  // namespace sg

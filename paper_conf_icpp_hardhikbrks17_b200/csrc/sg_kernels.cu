@@ -459,6 +459,18 @@ cudaError_t launch_gather_rows(const int64_t* src, const int64_t* rows, int64_t 
     return cudaGetLastError();
 }
 
+// count of row ids outside [0, n) (argument check of sg_threshold_on_rows)
+__global__ void k_check_rows(const int64_t* __restrict__ rows, int64_t nr, int64_t n, unsigned long long* bad) {
+    int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (j < nr && (rows[j] < 0 || rows[j] >= n)) atomicAdd(bad, 1ull);
+}
+
+cudaError_t launch_check_rows(const int64_t* rows, int64_t nr, int64_t n, unsigned long long* bad, cudaStream_t s) {
+    if (nr <= 0) return cudaSuccess;
+    SG_LAUNCH("k_check_rows", s, k_check_rows<<<(unsigned)((nr + 255) / 256), 256, 0, s>>>(rows, nr, n, bad));
+    return cudaGetLastError();
+}
+
 __global__ void k_add_offset(int64_t* x, int64_t n, int64_t off) {
     int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (j < n) x[j] += off;

@@ -114,6 +114,35 @@ def test_cost_curve_matches_plain_J():
     assert J == [oracle.J(_model_from(cm), w, a, u, t) for t in ts]
 
 
+@pytest.mark.parametrize("name,kind", [("C1", "first"), ("rmat12", "first"), ("rmat12", "random"),
+                                       ("rmat14_unperm", "first"), ("rmat14_unperm", "sqrt")])
+def test_threshold_on_explicit_rows_bit_exact(name, kind):
+    """Identify on a caller-chosen sample (predetermined first rows, random rows with repeats, sqrt(n)
+    rows): the GPU thr and J_min equal the oracle's argmin over exactly those rows."""
+    A = gen.rmat(14, permute=False) if name == "rmat14_unperm" else gen.config(name)
+    dA = _dev(A)
+    cm = sg.sg_default_cost_model()
+    n = A.nrows
+    rng = np.random.default_rng(3)
+    rows = {"first": np.arange(max(n // 50, 1)), "random": rng.integers(0, n, size=n // 20),
+            "sqrt": np.sort(rng.choice(n, size=int(np.sqrt(n)), replace=False))}[kind].astype(np.int64)
+    thr, rep = sg.sg_threshold_on_rows(dA, dA, rows, cm)
+    w = oracle.row_work(A, A)[rows]
+    a = np.diff(A.row_ptr)[rows]
+    u = oracle.counts(A, A, rows)
+    t_o, J_o = oracle.threshold(_model_from(cm), w, a, u)
+    assert (thr, rep["J_min"]) == (t_o, J_o)
+    assert rep["sample_rows"] == len(rows) and rep["sample_nonempty"] == int((w > 0).sum())
+
+
+def test_threshold_on_rows_rejects_bad_rows():
+    A = gen.config("C1")
+    dA = _dev(A)
+    with pytest.raises(sg.SgError) as e:
+        sg.sg_threshold_on_rows(dA, dA, np.array([0, 5, A.nrows], dtype=np.int64))
+    assert "INVALID_ARG" in str(e.value)
+
+
 def test_empty_sample_is_an_error():
     Z = gen.empty_rows(50, 50)
     dZ = _dev(Z)

@@ -89,7 +89,7 @@ def main():
             heavy = w > t
             arow = np.diff(H.row_ptr)
             kl = sum(v[1] for k, v in bk.items() if k in ("k_sym_light", "k_num_light"))
-            kh = sum(v[1] for k, v in bk.items() if k in ("k_sym_heavy", "k_num_heavy"))
+            kh = sum(v[1] for k, v in bk.items() if k in ("k_sym_heavy", "k_num_heavy", "k_num_dense"))
             rows.append({"t": t, "ms": ms, "ms_light": kl, "ms_heavy": kh, "r": r(t),
                          "L": [int(light.sum()), int(w[light].sum()), int(u[light].sum())],
                          "H": [int(heavy.sum()), int(w[heavy].sum()), int(u[heavy].sum()),
