@@ -2,35 +2,43 @@
 // heavy path): a single-pass DENSE-WINDOW numeric.
 //
 // One CTA (1024 threads) per row, rows heaviest-first from a dynamic counter. The row's column
-// space is swept in windows of WD = 16384 columns; the accumulator is a dense fp64 array indexed by
-// column (vals[c - lo]): no bitmap pre-pass and no rank lookup per product (the rank-mode kernel in
-// sg_heavy.cu needs both). The product that finds vals[c - lo] at exactly 0.0 (the first arrival)
-// marks bit (c - lo) of a 512-word occupancy bitmap; the window's entries are then emitted in column
-// order (sorted by construction): one block scan of half-word popcounts, each thread writing its own
-// set bits; only the emitted slots are cleared.
+// space is swept in windows of WD = 24576 columns (three tiles); the accumulator is a dense fp64
+// array indexed by column (vals[c - lo]): no bitmap pre-pass and no rank lookup per product (the
+// rank-mode kernel in sg_heavy.cu needs both). The product that finds vals[c - lo] at exactly 0.0
+// (the first arrival) marks bit (c - lo) of a 768-word occupancy bitmap; the window's entries are
+// then emitted in column order (sorted by construction): one block scan of per-thread popcounts
+// (24 columns each), each thread writing its own set bits; only the emitted slots are cleared.
 //
-// Per-k cursors advance monotonically window by window: B rows longer than LONG_ROW read their end
-// from the tile-pointer table tp (prefetched one window ahead), short rows keep their <= LONG_ROW
-// columns in shared memory (one load per entry per row, not per window).
+// The sweep is phase-synchronised: a row starts at the window the CTAs are at on average and wraps
+// around (output offsets from the symbolic pass's tile counts), so concurrent rows read the same
+// column slice of B, which then stays in L2 (DRAM reads of the kernel halved at R-MAT 20).
+// Per-k cursors advance window by window: B rows longer than LONG_ROW read their end from the
+// tile-pointer table tp (prefetched one window ahead), short rows count their entries below the
+// window end (cached in shared memory when two-tile windows leave room for it).
 #include "sg_device.cuh"
 #include <cstdlib>
 
 namespace sg {
 
 constexpr int DW_T = 1024;              // threads per CTA, one CTA per SM
-constexpr int DW_TILES = 2;             // TW tiles per window
-constexpr int WD = DW_TILES * TW;       // 16384 columns per window (128 KB fp64 accumulator)
-constexpr int DW_WORDS = WD / 32;       // 512 occupancy words
+#ifndef SG_DW_TILES
+#define SG_DW_TILES 3
+#endif
+constexpr int DW_TILES = SG_DW_TILES;   // TW tiles per window
+constexpr int WD = DW_TILES * TW;       // 24576 columns per window (192 KB fp64 accumulator)
+constexpr int DW_WORDS = WD / 32;       // 768 occupancy words
+constexpr int CPT = WD / 1024;          // columns per thread in the emission
+constexpr bool kShortCache = DW_TILES == 2;  // smem left for the short-row column cache
 constexpr int DKC = DW_T;               // k entries per chunk (one per thread)
-static_assert(DW_WORDS * 2 == DW_T, "emission: one half occupancy word per thread");
+static_assert(CPT * DW_T == WD && CPT <= 32, "emission: CPT columns per thread");
 
 struct DenseSmem {
     double vals[WD];                // dense accumulator of the window
-    uint32_t bm[DW_WORDS];          // occupancy (set by the first arrival)
+    uint32_t bm[DW_WORDS + 1];      // occupancy (set by the first arrival); +1 pad word
     int32_t s_beg[DKC];             // packed chunk entries: segment begin (B position)
     int32_t s_off[DKC];             //                       exclusive prefix of segment lengths
     double s_a[DKC];                //                       a_ik
-    int32_t sc[LONG_ROW][DKC];      // short B rows of single-chunk rows: their columns ([q][k], INT_MAX pad)
+    int32_t sc[kShortCache ? LONG_ROW : 1][DKC];  // short B rows of single-chunk rows: their columns ([q][k], INT_MAX pad)
     long long wsll[33];
     int ws[33];
 };
@@ -53,7 +61,7 @@ __global__ void __launch_bounds__(DW_T, 1) k_num_dense(
     const int nwin = (int)((p + WD - 1) / WD);
     int4* gs = gscr + (int64_t)blockIdx.x * amax;  // multi-chunk rows: per-k cursor
     for (int q = tid; q < WD; q += DW_T) S.vals[q] = 0.0;
-    for (int q = tid; q < DW_WORDS; q += DW_T) S.bm[q] = 0u;
+    for (int q = tid; q < DW_WORDS + 1; q += DW_T) S.bm[q] = 0u;
     while (true) {
         if (tid == 0) s_j = (long long)atomicAdd(counter, 1ull);
         __syncthreads();
@@ -87,7 +95,7 @@ __global__ void __launch_bounds__(DW_T, 1) k_num_dense(
         const int64_t rowbase = C_rp[li];
         int64_t pos = rowbase + off0;
         // per-k state of single-chunk rows: thread tid owns k entry tid; cursor at column lo0
-        int cur = 0, q0 = 0, lid = -1;
+        int cur = 0, q0 = 0, lid = -1, e1r = 0;
         uint32_t tpv = 0;
         double a = 0.0;
         if (single) {
@@ -101,7 +109,7 @@ __global__ void __launch_bounds__(DW_T, 1) k_num_dense(
                     const uint32_t* tr = tp + (int64_t)lid * (T + 1);
                     cur = q0 + (int)__ldg(tr + min(t0 * DW_TILES, T));
                     tpv = __ldg(tr + min((t0 + 1) * DW_TILES, T));
-                } else {
+                } else if constexpr (kShortCache) {
                     int n0 = 0;
                     #pragma unroll
                     for (int q = 0; q < LONG_ROW; ++q) {
@@ -110,6 +118,9 @@ __global__ void __launch_bounds__(DW_T, 1) k_num_dense(
                         n0 += c < lo0;
                     }
                     cur = q0 + n0;
+                } else {
+                    e1r = q0 + len;
+                    cur = t0 > 0 ? seg_end(B, q0, e1r, q0, false, 0u, lo0) : q0;
                 }
             }
         } else {
@@ -149,11 +160,13 @@ __global__ void __launch_bounds__(DW_T, 1) k_num_dense(
                     if (lid >= 0) {
                         end = q0 + (int)tpv;
                         if (j + 1 < nwin) tpv = __ldg(tp + (int64_t)lid * (T + 1) + min((tn + 1) * DW_TILES, T));
-                    } else {
+                    } else if constexpr (kShortCache) {
                         int n = 0;
                         #pragma unroll
                         for (int q = 0; q < LONG_ROW; ++q) n += S.sc[q][tid] < hi;
                         end = q0 + n;
+                    } else {
+                        end = seg_end(B, cur, e1r, q0, false, 0u, hi);
                     }
                     len = end - cur;
                     cur = tn == 0 ? q0 : end;
@@ -190,16 +203,21 @@ __global__ void __launch_bounds__(DW_T, 1) k_num_dense(
             if (dbg && tid == 0) tph[6] += 1;
             __syncthreads();  // every product of the window accumulated
             mark(3);
-            // ---- emission: thread tid owns 16 columns (half of occupancy word tid/2); one block scan
-            // of the half-word popcounts places every run; each thread writes its set bits in order ----
-            const uint32_t hw = (S.bm[tid >> 1] >> ((tid & 1) * 16)) & 0xFFFFu;
+            // ---- emission: thread tid owns columns [CPT*tid, CPT*tid + CPT) of the window; one block
+            // scan of their popcounts places every run; each thread writes its set bits in order ----
+            uint32_t hw;
+            {
+                const int b0 = CPT * tid, w0 = b0 >> 5, shv = b0 & 31;
+                const unsigned long long two = ((unsigned long long)S.bm[w0 + 1] << 32) | S.bm[w0];
+                hw = (uint32_t)(two >> shv) & (CPT == 32 ? 0xFFFFFFFFu : ((1u << CPT) - 1u));
+            }
             int wtot;
             const int ex = block_scan1<DW_T, int>(__popc(hw), &wtot, S.ws);
-            if ((tid & 1) == 0) S.bm[tid >> 1] = 0u;  // both halves were read before the scan's barrier
+            for (int q = tid; q < DW_WORDS; q += DW_T) S.bm[q] = 0u;  // all reads preceded the scan's barrier
             {
                 uint32_t m = hw;
                 int64_t at = pos + ex;
-                const int ebase = tid * 16;
+                const int ebase = tid * CPT;
                 while (m) {
                     const int e = ebase + __ffs(m) - 1;
                     m &= m - 1u;
