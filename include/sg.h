@@ -91,6 +91,7 @@ typedef struct {
     int64_t light_bins[13];   /* light rows per bin b: 2^(b-1) < w <= 2^b (b = 0: w == 1) */
     int64_t n_dense;          /* heavy rows on the dense-window kernel (w >= 2^dense_log2) */
     int64_t dense_log2;       /* that row-work bound (SG_DW_LOG2 overrides; >= 62: path disabled) */
+    int64_t n_light_sorted;   /* light rows whose columns cluster (hash homes crowded): uniform hash + sort */
 } sg_plan_info;
 
 typedef struct sg_plan sg_plan;   /* opaque; owns only its workspace */

@@ -75,7 +75,8 @@ class SampleReport(ctypes.Structure):
 class PlanInfo(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int64) for n in (
         "row_begin", "row_end", "thr", "n_empty", "n_light", "n_heavy", "nnz_c", "flops", "n_ranges")] + [
-        ("light_bins", ctypes.c_int64 * 13), ("n_dense", ctypes.c_int64), ("dense_log2", ctypes.c_int64)]
+        ("light_bins", ctypes.c_int64 * 13), ("n_dense", ctypes.c_int64), ("dense_log2", ctypes.c_int64),
+        ("n_light_sorted", ctypes.c_int64)]
 
     def as_dict(self):
         d = {n: int(getattr(self, n)) for n, _ in self._fields_ if n != "light_bins"}

@@ -30,6 +30,7 @@ struct sg_plan {
     int64_t nslots = 0, amax = 0;
     int64_t ndw = 0;                // heavy[0, ndw): dense-window rows (w >= 2^dw_log2), sg_dense.cu
     int32_t* dtc = nullptr;         // their per-tile output counts (ndw x T), from the symbolic pass
+    int64_t nskew = 0;              // light rows on the sorted path (column-skewed; sg_light.cu)
     int dw_log2 = 0;
     int2* span = nullptr;           // light rows: [cmin, cmax] of the output columns
     int4* gscr = nullptr;           // heavy rows with more than KC entries: per-k cursor scratch
@@ -197,7 +198,7 @@ sg_status row_stats(const Mat& A, const Mat& B, const int64_t* rows, int64_t nr,
     CK(cudaMemcpyAsync(dbin + NBINS, off, sizeof(int64_t) * NBINS, cudaMemcpyHostToDevice, s));
     CK(launch_bin_scatter(rs.w, nr, cap, dbin + NBINS, lists, s));
     for (int b = 0; b < NBIN_LIGHT; ++b)
-        CK(launch_sym_light(b, A, B, lists + off[b], cnt[b], rows, 0, rs.u, nullptr, s));
+        CK(launch_sym_light(b, A, B, lists + off[b], cnt[b], rows, 0, rs.u, nullptr, nullptr, s));
     unsigned long long* counter = (unsigned long long*)sc.get(sizeof(unsigned long long));
     if (!counter) return SG_ERR_OOM;
     CK(launch_sym_heavy(A, B, lists + off[BIN_HEAVY], cnt[BIN_HEAVY], rows, 0, rs.u, nullptr, nullptr, nullptr,
@@ -549,11 +550,13 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
     }
     // a6 symbolic
     for (int k = 0; k < NBIN_LIGHT; ++k)
-        CKF(launch_sym_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], nullptr, row_begin, pl->u, pl->span, s));
+        CKF(launch_sym_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], nullptr, row_begin, pl->u, pl->span,
+                             (unsigned long long*)(pl->dbin + 2 * NBINS + 1), s));
     CKF(launch_sym_heavy(a, b, pl->heavy, pl->nheavy, nullptr, row_begin, pl->u, pl->range_off, pl->ranges,
                          pl->nranges, pl->ndw, pl->dtc, pl->counter, s));
     CKF(scan_exclusive(pl->u, C_row_ptr, nr, stmp, s));
     CKF(cudaMemcpyAsync(&pl->nnz_c, C_row_ptr + nr, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    CKF(cudaMemcpyAsync(&pl->nskew, pl->dbin + 2 * NBINS + 1, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     CKF(cudaStreamSynchronize(s));
 #undef CKF
     *nnz_c_out = pl->nnz_c;
@@ -628,6 +631,7 @@ sg_status sg_plan_get_info(const sg_plan* pl, sg_plan_info* out) {
     out->nnz_c = pl->nnz_c;
     out->n_ranges = pl->nslots;
     out->n_dense = pl->ndw;
+    out->n_light_sorted = pl->nskew;
     out->dense_log2 = pl->dw_log2;
     // flops on demand
     if (pl->nr > 0) {

@@ -70,7 +70,8 @@ cudaError_t launch_bin_scatter(const int64_t* w, int64_t nr, int64_t thr, int64_
                                int32_t* lists, cudaStream_t s);
 // light path (sg_light.cu): bin b, rows = list entries (local index li); global row = rowmap ? rowmap[li] : rb + li
 cudaError_t launch_sym_light(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt,
-                             const int64_t* rowmap, int64_t rb, int64_t* u, int2* span, cudaStream_t s);
+                             const int64_t* rowmap, int64_t rb, int64_t* u, int2* span /*nullable*/,
+                             unsigned long long* nskew /*nullable: count of column-skewed rows*/, cudaStream_t s);
 cudaError_t launch_num_light(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, int64_t rb,
                              const int2* span, const int64_t* C_rp, int32_t* C_col, void* C_val, cudaStream_t s);
 // heavy path (sg_heavy.cu)

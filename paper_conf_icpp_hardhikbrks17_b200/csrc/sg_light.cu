@@ -46,19 +46,40 @@ __device__ __forceinline__ int set_insert(int32_t* T, int32_t c) {
     }
 }
 
+// ---- column-skew detection for the numeric pass's order-preserving hash -------------------------
+// The numeric pass homes column c at floor((c - cmin) * 2U / width). When a row's columns cluster far
+// below that resolution (R-MAT without the label permutation: hubs at low ids) the keys crowd some
+// stretches of homes and the probe runs grow with u. Rows with u > 64 keys in which some bucket of
+// 32 consecutive homes receives more than SKEW_BUCKET keys (local load > 1.25; a uniform row has
+// 16 on average) are flagged (span.x = -1 - cmin) and the numeric pass takes the SORTED path for
+// them: uniform hash, then a bitonic sort of the row's entries in shared memory.
+__device__ __forceinline__ uint32_t light_home(int32_t c, int cmin, uint64_t mult) {
+    return (uint32_t)(((uint64_t)(uint32_t)(c - cmin) * mult) >> 32);
+}
+template <int U> __device__ __forceinline__ uint64_t light_mult(int64_t width) {
+    return (((uint64_t)(2 * U)) << 32) / (uint64_t)width;
+}
+constexpr int SKEW_MIN_U = 64;
+constexpr int SKEW_BUCKET = 40;
+
 // ------------------------------------------------------------------------------------------------
 // symbolic, warp per row: u_i = |union of cols(B_k)| and the span [cmin, cmax] of those columns
 // ------------------------------------------------------------------------------------------------
 template <int U, int R>
 __global__ void __launch_bounds__(32 * R) k_sym_light(Mat A, Mat B, const int32_t* __restrict__ list, int64_t cnt,
                                                       const int64_t* __restrict__ rowmap, int64_t rb,
-                                                      int64_t* __restrict__ u, int2* __restrict__ span) {
+                                                      int64_t* __restrict__ u, int2* __restrict__ span,
+                                                      unsigned long long* nskew) {
     constexpr int P = 2 * U < 64 ? 64 : 2 * U;  // power of two, load <= 1/2
     constexpr int LOGP = __builtin_ctz(P);
+    constexpr int HBW = (2 * U + 31) / 32;      // key counts per 32 homes (skew detection)
     __shared__ int32_t tab[R * P];
+    __shared__ uint32_t hbits[R * HBW];
     const int g = threadIdx.x / 32, lane = threadIdx.x & 31;
     int32_t* T = tab + g * P;
+    uint32_t* hb = hbits + g * HBW;
     for (int s = lane; s < P; s += 32) T[s] = EMPTY_KEY;
+    for (int s = lane; s < HBW; s += 32) hb[s] = 0u;
     __syncwarp();
     for (int64_t j = (int64_t)blockIdx.x * R + g; j < cnt; j += (int64_t)gridDim.x * R) {
         const int64_t li = list[j];
@@ -76,9 +97,23 @@ __global__ void __launch_bounds__(32 * R) k_sym_light(Mat A, Mat B, const int32_
         ins = warp_sum(ins);
         cmn = warp_min(cmn);
         cmx = warp_max(cmx);
+        bool skew = false;
+        if (span && U > SKEW_MIN_U && ins > SKEW_MIN_U && (int64_t)cmx - cmn + 1 > 3 * U) {
+            __syncwarp();
+            const uint64_t mult = light_mult<U>((int64_t)cmx - cmn + 1);
+            for (int s = lane; s < P; s += 32) {
+                const int32_t c = T[s];
+                if (c != EMPTY_KEY) atomicAdd(&hb[light_home(c, cmn, mult) >> 5], 1u);  // keys per 32 homes
+            }
+            __syncwarp();
+            int d = 0;
+            for (int q = lane; q < HBW; q += 32) { d = max(d, (int)hb[q]); hb[q] = 0u; }
+            skew = warp_max(d) > SKEW_BUCKET;
+        }
         if (lane == 0) {
             u[li] = ins;
-            if (span) span[li] = make_int2(cmn, cmx);
+            if (span) span[li] = make_int2(skew ? -1 - cmn : cmn, cmx);
+            if (skew && nskew) atomicAdd(nskew, 1ull);
         }
         __syncwarp();
         for (int s = lane; s < P; s += 32) T[s] = EMPTY_KEY;
@@ -90,16 +125,21 @@ __global__ void __launch_bounds__(32 * R) k_sym_light(Mat A, Mat B, const int32_
 template <int U, int NT>
 __global__ void __launch_bounds__(NT) k_sym_light_blk(Mat A, Mat B, const int32_t* __restrict__ list, int64_t cnt,
                                                       const int64_t* __restrict__ rowmap, int64_t rb,
-                                                      int64_t* __restrict__ u, int2* __restrict__ span) {
+                                                      int64_t* __restrict__ u, int2* __restrict__ span,
+                                                      unsigned long long* nskew) {
     constexpr int P = 2 * U;
     constexpr int LOGP = __builtin_ctz(P);
+    constexpr int HBW = 2 * U / 32;
     __shared__ int32_t T[P];
+    __shared__ uint32_t hb[HBW];
+    __shared__ int s_d;
     __shared__ int64_t s_beg[NT];
     __shared__ int s_off[NT];
     __shared__ long long wsll[33];
     __shared__ int red[3][NT / 32];
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
     for (int s = tid; s < P; s += NT) T[s] = EMPTY_KEY;
+    for (int s = tid; s < HBW; s += NT) hb[s] = 0u;
     __syncthreads();
     for (int64_t j = blockIdx.x; j < cnt; j += gridDim.x) {
         const int64_t li = list[j];
@@ -130,32 +170,51 @@ __global__ void __launch_bounds__(NT) k_sym_light_blk(Mat A, Mat B, const int32_
         cmx = warp_max(cmx);
         if (lane == 0) { red[0][wid] = ins; red[1][wid] = cmn; red[2][wid] = cmx; }
         __syncthreads();
-        if (tid == 0) {
-            int a = 0, mn = INT_MAX, mx = -1;
-            for (int q = 0; q < NT / 32; ++q) { a += red[0][q]; mn = min(mn, red[1][q]); mx = max(mx, red[2][q]); }
-            u[li] = a;
-            if (span) span[li] = make_int2(mn, mx);
+        int a_ = 0, mn = INT_MAX, mx = -1;
+        for (int q = 0; q < NT / 32; ++q) { a_ += red[0][q]; mn = min(mn, red[1][q]); mx = max(mx, red[2][q]); }
+        bool skew = false;
+        if (span && a_ > SKEW_MIN_U && (int64_t)mx - mn + 1 > 3 * U) {  // block-uniform
+            const uint64_t mult = light_mult<U>((int64_t)mx - mn + 1);
+            for (int s = tid; s < P; s += NT) {
+                const int32_t c = T[s];
+                if (c != EMPTY_KEY) atomicAdd(&hb[light_home(c, mn, mult) >> 5], 1u);  // keys per 32 homes
+            }
+            if (tid == 0) s_d = 0;
+            __syncthreads();
+            int d = 0;
+            for (int q = tid; q < HBW; q += NT) { d = max(d, (int)hb[q]); hb[q] = 0u; }
+            d = warp_max(d);
+            if (lane == 0 && d) atomicMax(&s_d, d);
+            __syncthreads();
+            skew = s_d > SKEW_BUCKET;
         }
+        if (tid == 0) {
+            u[li] = a_;
+            if (span) span[li] = make_int2(skew ? -1 - mn : mn, mx);
+            if (skew && nskew) atomicAdd(nskew, 1ull);
+        }
+        __syncthreads();  // red[] and s_d read by everyone before the next row rewrites them
         for (int s = tid; s < P; s += NT) T[s] = EMPTY_KEY;
         __syncthreads();
     }
 }
 
 cudaError_t launch_sym_light(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt,
-                             const int64_t* rowmap, int64_t rb, int64_t* u, int2* span, cudaStream_t s) {
+                             const int64_t* rowmap, int64_t rb, int64_t* u, int2* span, unsigned long long* nskew,
+                             cudaStream_t s) {
     if (cnt <= 0) return cudaSuccess;
     switch (b) {
 #define X(B_, U_, R_)                                                                                     \
     case B_:                                                                                              \
         SG_LAUNCH("k_sym_light", s, (k_sym_light<U_, R_><<<grid_for(cnt, R_, 148 * 32), 32 * R_, 0, s>>>( \
-                                        A, B, list, cnt, rowmap, rb, u, span)));                           \
+                                        A, B, list, cnt, rowmap, rb, u, span, nskew)));                    \
         break;
         SG_LIGHT_WARP_BINS(X)
 #undef X
 #define X(B_, U_, NT_)                                                                                       \
     case B_:                                                                                                 \
         SG_LAUNCH("k_sym_light", s, (k_sym_light_blk<U_, NT_><<<grid_for(cnt, 1, 148 * 8), NT_, 0, s>>>(     \
-                                        A, B, list, cnt, rowmap, rb, u, span)));                              \
+                                        A, B, list, cnt, rowmap, rb, u, span, nskew)));                       \
         break;
         SG_LIGHT_BLOCK_BINS(X)
 #undef X
@@ -167,6 +226,79 @@ cudaError_t launch_sym_light(int b, const Mat& A, const Mat& B, const int32_t* l
 // ------------------------------------------------------------------------------------------------
 // numeric: order-preserving hash over [cmin, cmax] -> ascending row without a sort pass
 // ------------------------------------------------------------------------------------------------
+// ---- the SORTED path of column-skewed rows: uniform hash over [0, H), then the row's entries are
+// gathered into [H, H + u) (order irrelevant), bitonic-sorted by column and written out ----
+template <int H>
+__device__ __forceinline__ void uni_insert(int32_t* keys, double* vals, int32_t c, double v) {
+    constexpr int LOGH = __builtin_ctz(H);
+    uint32_t h = ((uint32_t)c * 0x9E3779B1u) >> (32 - LOGH);
+    while (true) {
+        int32_t old = keys[h];
+        if (old == c) break;
+        if (old == EMPTY_KEY) {
+            old = atomicCAS(&keys[h], EMPTY_KEY, c);
+            if (old == EMPTY_KEY || old == c) break;
+        }
+        h = (h + 1) & (H - 1);
+    }
+    atomicAdd(&vals[h], v);
+}
+
+// bitonic sort of n (a power of two) (key, value) pairs by key by the G threads of a group
+template <int G, int BLK>
+__device__ __forceinline__ void bitonic_pairs(int32_t* k, double* v, int n) {
+    const int t = threadIdx.x % G;
+    for (int kk = 2; kk <= n; kk <<= 1)
+        for (int j = kk >> 1; j > 0; j >>= 1) {
+            for (int i = t; i < n / 2; i += G) {
+                const int ix = ((i & ~(j - 1)) << 1) | (i & (j - 1));
+                const int iy = ix + j;
+                const int32_t a = k[ix], b = k[iy];
+                if ((a > b) == ((ix & kk) == 0)) {
+                    k[ix] = b;
+                    k[iy] = a;
+                    const double x = v[ix];
+                    v[ix] = v[iy];
+                    v[iy] = x;
+                }
+            }
+            group_bar<G, BLK>();
+        }
+}
+
+// Gather the occupied slots of [0, H) into [H, H + u), clearing [0, H); sort; emit; clear [H, H + n).
+// cnt: a group-private shared counter (0 on entry; left at 0).
+template <int G, int BLK, int H, class VT>
+__device__ __forceinline__ void sorted_emit(int32_t* keys, double* vals, int* cnt, int64_t base,
+                                            int32_t* __restrict__ C_col, VT* __restrict__ C_val) {
+    const int t = threadIdx.x % G;
+    for (int s = t; s < H; s += G) {
+        const int32_t c = keys[s];
+        if (c != EMPTY_KEY) {
+            const int at = H + atomicAdd(cnt, 1);
+            keys[at] = c;
+            vals[at] = vals[s];
+            keys[s] = EMPTY_KEY;
+            vals[s] = 0.0;
+        }
+    }
+    group_bar<G, BLK>();
+    const int u = *cnt;
+    int n = 1;
+    while (n < u) n <<= 1;
+    for (int s = u + t; s < n; s += G) keys[H + s] = INT_MAX;  // pads sort last
+    group_bar<G, BLK>();
+    bitonic_pairs<G, BLK>(keys + H, vals + H, n);
+    for (int i = t; i < u; i += G) {
+        st_out(C_col + base + i, keys[H + i]);
+        st_out(C_val + base + i, (VT)vals[H + i]);
+    }
+    group_bar<G, BLK>();
+    for (int s = t; s < n; s += G) { keys[H + s] = EMPTY_KEY; vals[H + s] = 0.0; }
+    if (t == 0) *cnt = 0;
+    group_bar<G, BLK>();
+}
+
 template <int U>
 struct LightTable {
     static constexpr int H = 2 * U;  // home range (load <= 1/2)
@@ -180,16 +312,28 @@ __global__ void __launch_bounds__(32 * R) k_num_light(Mat A, Mat B, const int32_
                                                       VT* __restrict__ C_val) {
     constexpr int H = LightTable<U>::H, P = LightTable<U>::P;
     extern __shared__ double smem_d[];
+    __shared__ int s_cnt[R];
     const int g = threadIdx.x / 32, lane = threadIdx.x & 31;
     double* vals = smem_d + g * P;
     int32_t* keys = reinterpret_cast<int32_t*>(smem_d + R * P) + g * P;
     for (int s = lane; s < P; s += 32) { keys[s] = EMPTY_KEY; vals[s] = 0.0; }
+    if (lane == 0) s_cnt[g] = 0;
     __syncwarp();
     for (int64_t j = (int64_t)blockIdx.x * R + g; j < cnt; j += (int64_t)gridDim.x * R) {
         const int64_t li = list[j];
         const int64_t row = rb + li;
         const int64_t s0 = __ldg(A.rp + row), s1 = __ldg(A.rp + row + 1);
         const int2 sp = span[li];
+        if constexpr (U > SKEW_MIN_U) {
+            if (sp.x < 0) {  // column-skewed row: sorted path
+                for (int64_t pb = s0; pb < s1; pb += 32)
+                    chunk_products<true, VT, 2>(A, B, pb, min(pb + 32, s1), [](int, int64_t&, int&) {},
+                                                [&](int32_t c, double v) { uni_insert<H>(keys, vals, c, v); });
+                __syncwarp();
+                sorted_emit<32, 32 * R, H, VT>(keys, vals, &s_cnt[g], C_rp[li], C_col, C_val);
+                continue;
+            }
+        }
         const int64_t width = (int64_t)sp.y - sp.x + 1;
         const bool ident = width <= P;
         const uint64_t mult = ident ? 0 : (((uint64_t)H << 32) / (uint64_t)width);
@@ -221,18 +365,40 @@ __global__ void __launch_bounds__(NT) k_num_light_blk(Mat A, Mat B, const int32_
     __shared__ double s_a[NT];
     __shared__ long long wsll[33];
     __shared__ int ws[NT / 32];
-    __shared__ int s_hmax;
+    __shared__ int s_hmax, s_cnt;
     const int tid = threadIdx.x, lane = tid & 31;
     double* vals = smem_d;
     int32_t* keys = reinterpret_cast<int32_t*>(smem_d + P);
     for (int s = tid; s < P; s += NT) { keys[s] = EMPTY_KEY; vals[s] = 0.0; }
-    if (tid == 0) s_hmax = -1;
+    if (tid == 0) { s_hmax = -1; s_cnt = 0; }
     __syncthreads();
     for (int64_t j = blockIdx.x; j < cnt; j += gridDim.x) {
         const int64_t li = list[j];
         const int64_t row = rb + li;
         const int64_t s0 = __ldg(A.rp + row), s1 = __ldg(A.rp + row + 1);
         const int2 sp = span[li];
+        if (sp.x < 0) {  // column-skewed row (block-uniform): sorted path
+            for (int64_t c0 = s0; c0 < s1; c0 += NT) {
+                const int64_t i = c0 + tid;
+                int len = 0;
+                int64_t beg = 0;
+                double a = 0.0;
+                if (i < s1) {
+                    const int k = __ldg(A.col + i);
+                    beg = __ldg(B.rp + k);
+                    len = (int)(__ldg(B.rp + k + 1) - beg);
+                    a = ldv<VT>(A.val, i);
+                }
+                int nk;
+                const int tot = chunk_compact<NT, int64_t>(len, beg, a, s_beg, s_off, s_a, &nk, wsll);
+                warp_slice<NT, true, VT, int64_t>(s_beg, s_off, s_a, nk, tot, B, [&](int32_t c, double v) {
+                    if (c >= 0) uni_insert<H>(keys, vals, c, v);
+                });
+                __syncthreads();
+            }
+            sorted_emit<NT, NT, H, VT>(keys, vals, &s_cnt, C_rp[li], C_col, C_val);
+            continue;
+        }
         const int64_t width = (int64_t)sp.y - sp.x + 1;
         const bool ident = width <= P;
         const uint64_t mult = ident ? 0 : (((uint64_t)H << 32) / (uint64_t)width);

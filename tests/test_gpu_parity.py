@@ -393,3 +393,31 @@ def test_dense_window_integer_values_exact(monkeypatch, dtype):
     R = oracle.spgemm(A, A, with_absmag=True)
     compare_rows(rp, col, val, R, dtype, exact_values=True)
     assert info["n_dense"] == info["n_heavy"] > 0
+
+
+@pytest.mark.parametrize("scale,thr", [(14, 4096), (16, 1024)])
+def test_light_skewed_rows_sorted_path(scale, thr):
+    """Un-permuted R-MAT (hubs at low ids): light rows whose columns crowd the order-preserving
+    hash's homes take the uniform-hash + bitonic-sort path; C is unchanged (structure bit-exact)."""
+    A = gen.rmat(scale, permute=False)
+    (rp, col, val), info, _ = _full_product(A, A, thr)
+    R = oracle.spgemm(A, A, with_absmag=True)
+    assert np.array_equal(rp, R.row_ptr)
+    compare_rows(rp, col, val, R, "f64")
+    assert info["n_light_sorted"] > 0
+
+
+def test_light_sorted_path_integer_values_exact():
+    A = gen.rmat(14, permute=False, mode="int")
+    (rp, col, val), info, _ = _full_product(A, A, 4096)
+    R = oracle.spgemm(A, A, with_absmag=True)
+    compare_rows(rp, col, val, R, "f64", exact_values=True)
+    assert info["n_light_sorted"] > 0
+
+
+@pytest.mark.parametrize("name", ["C2", "rmat16"])
+def test_uniform_rows_keep_the_order_preserving_path(name):
+    """Permuted / uniform inputs: (almost) no light row is flagged as column-skewed."""
+    A = gen.config(name)
+    _, info, _ = _full_product(A, A, 4096)
+    assert info["n_light_sorted"] <= max(1, info["n_light"] // 100)
