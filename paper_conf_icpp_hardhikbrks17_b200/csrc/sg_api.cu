@@ -542,8 +542,8 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
         pl->ranges = (RangeRec*)palloc(pl, sizeof(RangeRec) * (size_t)(pl->nslots > 0 ? pl->nslots : 1));
         pl->tp = (uint32_t*)palloc(pl, 4 * (size_t)(pl->nlong > 0 ? pl->nlong : 1) * (size_t)(pl->T + 1));
         if (!pl->ranges || !pl->tp) return fail(SG_ERR_OOM);
-        if (pl->amax > heavy_kc()) {
-            pl->gscr = (int4*)palloc(pl, sizeof(int4) * (size_t)heavy_grid() * (size_t)pl->amax);
+        if (pl->amax > heavy_kc() || pl->amax > dense_kc()) {
+            pl->gscr = (int4*)palloc(pl, sizeof(int4) * (size_t)(heavy_grid() > dense_grid() ? heavy_grid() : dense_grid()) * (size_t)pl->amax);
             if (!pl->gscr) return fail(SG_ERR_OOM);
         }
         if (pl->nlong > 0) CKF(launch_build_tp(b, pl->long_id, pl->T, pl->tp, s));

@@ -20,14 +20,21 @@
 
 namespace sg {
 
-constexpr int DW_T = 1024;              // threads per CTA, one CTA per SM
+#ifndef SG_DW_T
+#define SG_DW_T 1024
+#endif
+#ifndef SG_DW_OCC
+#define SG_DW_OCC 1
+#endif
 #ifndef SG_DW_TILES
 #define SG_DW_TILES 3
 #endif
+constexpr int DW_T = SG_DW_T;           // threads per CTA
+constexpr int DW_OCC = SG_DW_OCC;       // CTAs per SM (while one CTA waits at a window barrier, another accumulates)
 constexpr int DW_TILES = SG_DW_TILES;   // TW tiles per window
 constexpr int WD = DW_TILES * TW;       // 24576 columns per window (192 KB fp64 accumulator)
 constexpr int DW_WORDS = WD / 32;       // 768 occupancy words
-constexpr int CPT = WD / 1024;          // columns per thread in the emission
+constexpr int CPT = WD / DW_T;          // columns per thread in the emission
 constexpr bool kShortCache = DW_TILES == 2;  // smem left for the short-row column cache
 constexpr int DKC = DW_T;               // k entries per chunk (one per thread)
 static_assert(CPT * DW_T == WD && CPT <= 32, "emission: CPT columns per thread");
@@ -44,7 +51,7 @@ struct DenseSmem {
 };
 
 template <class VT>
-__global__ void __launch_bounds__(DW_T, 1) k_num_dense(
+__global__ void __launch_bounds__(DW_T, DW_OCC) k_num_dense(
     Mat A, Mat B, const int32_t* __restrict__ heavy, int64_t ndw, int64_t rb, const int32_t* __restrict__ long_id,
     const uint32_t* __restrict__ tp, int T, const int64_t* __restrict__ C_rp, int32_t* __restrict__ C_col,
     VT* __restrict__ C_val, unsigned long long* counter, int4* __restrict__ gscr, int64_t amax,
@@ -60,6 +67,7 @@ __global__ void __launch_bounds__(DW_T, 1) k_num_dense(
     const int64_t p = B.ncols;
     const int nwin = (int)((p + WD - 1) / WD);
     int4* gs = gscr + (int64_t)blockIdx.x * amax;  // multi-chunk rows: per-k cursor
+    const uint32_t a_vals = smem_addr(S.vals), a_bm = smem_addr(S.bm);
     for (int q = tid; q < WD; q += DW_T) S.vals[q] = 0.0;
     for (int q = tid; q < DW_WORDS + 1; q += DW_T) S.bm[q] = 0u;
     while (true) {
@@ -144,12 +152,15 @@ __global__ void __launch_bounds__(DW_T, 1) k_num_dense(
             if (t == 0) pos = rowbase;                 // wrapped to the row's first window
             const int64_t lo = (int64_t)t * WD, hi = min(p, lo + WD);
             const int th = min((t + 1) * DW_TILES, T);  // tile index of hi
+            // window-relative shared addresses folded into one base each (lo is a multiple of 32):
+            // &vals[c - lo] = vb + 8c, &bm[(c - lo) >> 5] = bb + 4(c >> 5)  (mod 2^32)
+            const uint32_t vb = opaque_u32(a_vals - 8u * (uint32_t)lo);
+            const uint32_t bb = opaque_u32(a_bm - 4u * ((uint32_t)lo >> 5));
             auto acc = [&](int32_t c, double v) {
                 if (c < 0) return;
-                const uint32_t d = (uint32_t)(c - lo);
                 // first arrival (accumulator at exactly 0.0) marks the column; a later product that finds
                 // an exact 0.0 partial sum re-marks it (idempotent)
-                if (atomicAdd(&S.vals[d], v) == 0.0) atomicOr(&S.bm[d >> 5], 1u << (d & 31));
+                if (atom_add_f64_s(vb + 8u * (uint32_t)c, v) == 0.0) red_or_s(bb + 4u * ((uint32_t)c >> 5), 1u << (c & 31));
             };
             int any = 0;
             if (single) {
@@ -244,7 +255,7 @@ cudaError_t launch_num_dense(const Mat& A, const Mat& B, const int32_t* heavy, i
     const int smem = (int)sizeof(DenseSmem);
     cudaError_t e = cudaMemsetAsync(counter, 0, 2 * sizeof(unsigned long long), s);  // row counter, window clock
     if (e != cudaSuccess) return e;
-    const int grid = (int)(ndw < 148 ? ndw : 148);
+    const int grid = (int)(ndw < 148 * DW_OCC ? ndw : 148 * DW_OCC);
     if (A.dt == 0) {
         if ((e = cudaFuncSetAttribute(k_num_dense<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
         SG_LAUNCH("k_num_dense", s, (k_num_dense<double><<<grid, DW_T, smem, s>>>(A, B, heavy, ndw, rb, long_id, tp, T, C_rp,
@@ -258,6 +269,8 @@ cudaError_t launch_num_dense(const Mat& A, const Mat& B, const int32_t* heavy, i
 }
 
 int dense_window_cols() { return WD; }
+int dense_grid() { return 148 * DW_OCC; }
+int dense_kc() { return DKC; }
 
 }  // namespace sg
 

@@ -51,6 +51,45 @@ template <class T> __device__ __forceinline__ void st_out(T* p, T v) {
 #endif
 }
 
+// ---- 32-bit shared-window addressing for the hot accumulators --------------------------------------
+// Taking &S.x[i] of dynamic shared memory yields a GENERIC pointer; under the 64-register cap of
+// 1024-thread CTAs the compiler then re-derives the shared window base (S2R SR_CgaCtaId + LEA) at every
+// product. A 32-bit .shared address computed once keeps the accumulate at LDS/ATOMS [reg].
+__device__ __forceinline__ uint32_t opaque_u32(uint32_t x) {
+    uint32_t a;
+    asm volatile("mov.b32 %0, %1;" : "=r"(a) : "r"(x));
+    return a;
+}
+__device__ __forceinline__ uint32_t smem_addr(const void* p) {
+    // opaque to the optimizer: held in a register instead of being re-derived from SR_CgaCtaId per use
+    uint32_t a;
+    asm volatile("mov.b32 %0, %1;" : "=r"(a) : "r"((uint32_t)__cvta_generic_to_shared(p)));
+    return a;
+}
+__device__ __forceinline__ double atom_add_f64_s(uint32_t a, double v) {
+    double old;
+    asm volatile("atom.shared.add.f64 %0, [%1], %2;" : "=d"(old) : "r"(a), "d"(v) : "memory");
+    return old;
+}
+__device__ __forceinline__ void red_or_s(uint32_t a, uint32_t v) {
+    asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ uint32_t ld_u32_s(uint32_t a) {
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+    return v;
+}
+__device__ __forceinline__ double ld_f64_s(uint32_t a) {
+    double v;
+    asm volatile("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"(a) : "memory");
+    return v;
+}
+__device__ __forceinline__ uint32_t ld_u16_s(uint32_t a) {
+    uint16_t v;
+    asm volatile("ld.shared.u16 %0, [%1];" : "=h"(v) : "r"(a) : "memory");
+    return v;
+}
+
 template <class VT> __device__ __forceinline__ double ldv(const void* v, int64_t q) {
     return (double)__ldg(reinterpret_cast<const VT*>(v) + q);
 }
@@ -282,36 +321,50 @@ __device__ __forceinline__ int chunk_compact(int len, BEG beg, double a, BEG* s_
 // fast path when the batch lies inside one long B segment).
 template <int NT, bool VAL, class VT, class BEG>
 struct SliceCursor {
-    const BEG* s_beg;
-    const int* s_off;
-    const double* s_a;
+    static_assert(sizeof(BEG) == 4 || sizeof(BEG) == 8, "segment begin: int32 or int64");
+    // 32-bit shared addresses of the packed chunk arrays (see smem_addr)
+    // one opaque base register; the other arrays sit at constant byte distances from it
+    uint32_t a_beg, d_off, d_a;
     int nk, tot, j_lo, j_hi, i0;
+    __device__ __forceinline__ BEG beg_at(int i) const {
+        if constexpr (sizeof(BEG) == 4) return (BEG)(int32_t)ld_u32_s(a_beg + 4u * (uint32_t)i);
+        else {
+            int64_t v;
+            asm volatile("ld.shared.s64 %0, [%1];" : "=l"(v) : "r"(a_beg + 8u * (uint32_t)i) : "memory");
+            return (BEG)v;
+        }
+    }
+    __device__ __forceinline__ int off_at(int i) const { return (int)ld_u32_s(a_beg + d_off + 4u * (uint32_t)i); }
+    __device__ __forceinline__ double a_at(int i) const { return ld_f64_s(a_beg + d_a + 8u * (uint32_t)i); }
     __device__ __forceinline__ SliceCursor(const BEG* sb, const int* so, const double* sa, int nk_, int tot_)
-        : s_beg(sb), s_off(so), s_a(sa), nk(nk_), tot(tot_) {
+        : nk(nk_), tot(tot_) {
         constexpr int NW = NT / 32;
+        a_beg = smem_addr(sb);
+        d_off = (uint32_t)((const char*)so - (const char*)sb);
+        d_a = sa ? (uint32_t)((const char*)sa - (const char*)sb) : 0u;
         const int wid = threadIdx.x >> 5;
         const int per = (((tot + NW - 1) / NW) + 31) & ~31;
         j_lo = wid * per;
         j_hi = min(tot, j_lo + per);
-        i0 = j_lo < j_hi ? find_k(s_off, nk, j_lo) : 0;
+        i0 = j_lo < j_hi ? find_k(so, nk, j_lo) : 0;
     }
     // batch [j0, j0 + 32): lane's (column, a_ik * b_kj), c = -1 beyond the slice
     __device__ __forceinline__ void fetch(const Mat& B, int j0, int& c, double& v) {
         const int lane = threadIdx.x & 31;
-        const int e0 = i0 + 1 < nk ? s_off[i0 + 1] : tot;
+        const int e0 = i0 + 1 < nk ? off_at(i0 + 1) : tot;
         if (j0 + 31 < e0) {  // fast path: the whole batch lies inside entry i0 (hub rows of B)
             const int j = j0 + lane;
             c = -1;
             v = 0.0;
             if (j < j_hi) {
-                const int64_t q = (int64_t)s_beg[i0] + (j - s_off[i0]);
+                const int64_t q = (int64_t)beg_at(i0) + (j - off_at(i0));
                 c = __ldg(B.col + q);
-                if (VAL) v = s_a[i0] * ldv<VT>(B.val, q);
+                if (VAL) v = a_at(i0) * ldv<VT>(B.val, q);
             }
             return;
         }
         const int ii = i0 + lane;
-        const int o = ii < nk ? s_off[ii] : INT_MAX;
+        const int o = ii < nk ? off_at(ii) : INT_MAX;
         const int j = j0 + lane;
         int s = 0;
         #pragma unroll
@@ -324,9 +377,9 @@ struct SliceCursor {
         c = -1;
         v = 0.0;
         if (j < j_hi) {
-            const int64_t q = (int64_t)s_beg[kk] + (j - os);
+            const int64_t q = (int64_t)beg_at(kk) + (j - os);
             c = __ldg(B.col + q);
-            if (VAL) v = s_a[kk] * ldv<VT>(B.val, q);
+            if (VAL) v = a_at(kk) * ldv<VT>(B.val, q);
         }
         i0 = __shfl_sync(FULL, kk, 31);
     }

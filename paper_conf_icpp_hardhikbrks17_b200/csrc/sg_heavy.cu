@@ -22,13 +22,22 @@ namespace sg {
 #define SG_INREG 1
 #endif
 constexpr int SYM_T = HEAVY_THREADS;  // symbolic: one CTA of 1024 threads per SM (128 KB bitmap window)
-constexpr int NUM_T = 1024;           // numeric: threads per CTA
-constexpr int NUM_OCC = 1;            // numeric CTAs per SM (smem-bound)
+#ifndef SG_NUM_T
+#define SG_NUM_T 1024
+#endif
+#ifndef SG_NUM_OCC
+#define SG_NUM_OCC 1
+#endif
+#ifndef SG_RCAP
+#define SG_RCAP 16384
+#endif
+constexpr int NUM_T = SG_NUM_T;       // numeric: threads per CTA
+constexpr int NUM_OCC = SG_NUM_OCC;   // numeric CTAs per SM (smem-bound)
 constexpr int KC = NUM_T;             // numeric k entries per chunk: one per thread
 constexpr int KCS = SYM_T;            // symbolic k entries per chunk
 constexpr int RW_TILES = NUM_T / 32;  // max tiles per numeric range (16 -> 128K columns, 16 KB bitmap)
 constexpr int RW_WORDS = RW_TILES * TW / 32;   // = 256 words per warp in the rank prefix
-constexpr int RCAP = 16384;           // max entries per numeric range (fp64 accumulator 128 KB)
+constexpr int RCAP = SG_RCAP;         // max entries per numeric range (fp64 accumulator 128 KB)
 constexpr int RHALF = RCAP / 2;       // range key granularity (a range = run of tiles with equal key)
 
 // ------------------------------------------------------------------------------------------------
@@ -194,8 +203,9 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_sym_heavy(Mat A, Mat B, co
                 }
                 int nk;
                 const int tot = chunk_compact<SYM_T, int64_t>(len, beg, 0.0, s_beg, s_off, nullptr, &nk, wsll);
+                const uint32_t bb = opaque_u32(smem_addr(bm) - 4u * ((uint32_t)wlo >> 5));  // wlo: multiple of 32
                 warp_slice<SYM_T, false, double, int64_t>(s_beg, s_off, nullptr, nk, tot, B, [&](int32_t c, double) {
-                    if (c >= 0) { const uint32_t d = (uint32_t)(c - wlo); atomicOr(&bm[d >> 5], 1u << (d & 31)); }
+                    if (c >= 0) red_or_s(bb + 4u * ((uint32_t)c >> 5), 1u << (c & 31));
                 });
                 __syncthreads();
             }
@@ -345,6 +355,9 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
     int4* gs = gscr + (int64_t)blockIdx.x * amax;  // multi-chunk rows: per-k (cur, -, beg, len)
     for (int q = tid; q < RW_WORDS; q += NUM_T) S.bm[q] = 0u;
     for (int q = tid; q < RCAP + 2; q += NUM_T) S.vals[q] = 0.0;
+    const uint32_t a_bm = smem_addr(S.bm);
+    const uint32_t a_pref = a_bm + (uint32_t)((const char*)S.pref - (const char*)S.bm);
+    const uint32_t a_vals = a_bm + (uint32_t)((const char*)S.vals - (const char*)S.bm);
 #ifndef SG_BULK
 #define SG_BULK 1
 #endif
@@ -418,8 +431,9 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 mark(8);
                 const int ctot = chunk_compact<NUM_T, int32_t>(len, beg, a, S.s_beg, S.s_off, S.s_a, &nk, S.wsll);
                 mark(2);
+                const uint32_t bb = opaque_u32(a_bm - 4u * ((uint32_t)lo >> 5));  // &bm[(c - lo) >> 5] = bb + 4(c >> 5)
                 auto setbit = [&](int32_t c, double) {
-                    if (c >= 0) { const uint32_t d = (uint32_t)(c - lo); atomicOr(&S.bm[d >> 5], 1u << (d & 31)); }
+                    if (c >= 0) red_or_s(bb + 4u * ((uint32_t)c >> 5), 1u << (c & 31));
                 };
                 // small ranges: the products stay in registers from pass 1 to pass 2 (B read once)
                 inreg = SG_INREG && single && warp_slice_regs<NUM_T, VT, int32_t>(S.s_beg, S.s_off, S.s_a, nk, ctot, B, rc, rv);
@@ -471,15 +485,19 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
             // ---- pass 2: every product accumulated at rank(c); the column is written on first arrival ----
             const int64_t base = crow + R.off;
             const int sh = kBulk ? (int)(base & 1) : 0;  // vals[e + sh] and C_val[base + e] share 16 B alignment
+            // lo is a multiple of 32: word (c - lo) >> 5 = (c >> 5) - (lo >> 5), bit c & 31
+            const uint32_t bw = opaque_u32(a_bm - 4u * ((uint32_t)lo >> 5));
+            const uint32_t pw = a_pref - 2u * ((uint32_t)lo >> 5);
+            const uint32_t vb = a_vals + 8u * (uint32_t)sh;
             auto acc = [&](int32_t c, double v) {
                 if (c < 0) return;
-                const uint32_t d = (uint32_t)(c - lo);
-                const uint32_t wv = S.bm[d >> 5];
-                const int rank = S.pref[d >> 5] + __popc(wv & ((1u << (d & 31)) - 1u));
+                const uint32_t cw = (uint32_t)c >> 5;
+                const uint32_t wv = ld_u32_s(bw + 4u * cw);
+                const int rank = (int)ld_u16_s(bw + (pw - bw) + 2u * cw) + __popc(wv & ((1u << (c & 31)) - 1u));
                 // the product that finds the accumulator at exactly 0.0 writes the column: the first
                 // product of every column does (accumulators start at 0.0); a later one only when the
                 // partial sum is exactly 0.0, rewriting the same value
-                if (atomicAdd(&S.vals[rank + sh], v) == 0.0) st_out(C_col + base + rank, c);
+                if (atom_add_f64_s(bw + (vb - bw) + 8u * (uint32_t)rank, v) == 0.0) st_out(C_col + base + rank, c);
             };
             if (inreg) {
                 #pragma unroll

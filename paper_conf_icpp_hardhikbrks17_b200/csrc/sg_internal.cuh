@@ -101,6 +101,8 @@ int dense_window_cols();
 int dense_window_log2(int64_t p);  // SG_DW_LOG2 overrides (>= 62 disables the dense-window path)
 int heavy_kc();
 int heavy_grid();
+int dense_grid();
+int dense_kc();
 // threshold: cost histogram over rows then argmin over t in [0, cap_L]
 struct ThrResult { long long thr, Jmin, base, W_L, W_all, nonempty; };
 cudaError_t launch_cost_hist(const CostModelD& cm, const int64_t* w, const int64_t* a, const int64_t* u, int64_t nr,
