@@ -121,6 +121,20 @@ def peaks():
         return 6650.0, "fallback"
 
 
+def smem_peaks():
+    """Measured shared-memory atomic throughputs (Gop/s, whole GPU) from tools/microbench on a B200."""
+    f = os.path.join(ROOT, "profiles", "r01_microbench_accumulator_primitives.txt")
+    out = {}
+    try:
+        for line in open(f):
+            parts = line.split()
+            if len(parts) >= 5 and parts[4] == "Gop/s":
+                out[parts[0]] = float(parts[3])
+    except OSError:
+        return None
+    return out
+
+
 def csr_bytes(nrows, nnz, vbytes):
     return 8 * (nrows + 1) + (4 + vbytes) * nnz
 
@@ -266,6 +280,8 @@ def main():
     ndense = int(dmask.sum().item())
     nnzC_dense = int(u[dmask].sum().item())
     nnzA_dense = int(a_rows[dmask].sum().item())
+    W_heavy = int(wrow[cls == 2].sum().item())
+    W_dense = int(wrow[dmask].sum().item())
     del cls, u, a_rows, wrow, dmask
     nnzC_total = nnz_local
     if world > 1:
@@ -334,6 +350,21 @@ def main():
         roof = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": hbm, "unit": "GB/s",
                 "frac": achieved / hbm, "traffic": traffic, "peak_kind": peak_kind,
                 "alg_bytes_per_launch": alg[dom], "launch_ms": per_launch_ms, "launches": cnt}
+    # ---- the on-chip bound of the heavy kernels: every product ends in one shared-memory atomic (fp64 CAS add
+    # in the numeric kernels, a 32-bit OR in the symbolic / rank pass 1); peak = our microbenchmark of that
+    # atomic at random addresses on this B200 (profiles/r01_microbench_accumulator_primitives.txt) ----
+    roof_smem = None
+    mb = smem_peaks()
+    if mb and bk:
+        ops = {"k_num_dense": (W_dense, "smem_cas_f64_16K"), "k_num_heavy": (W_heavy - W_dense, "smem_cas_f64_16K"),
+               "k_sym_heavy": (W_heavy, "smem_or32_16K")}
+        roof_smem = {}
+        for k, (nprod, prim) in ops.items():
+            if k in bk and prim in mb:
+                cnt, tot = bk[k]
+                rate = nprod / (tot / cnt / 1e3) / 1e9
+                roof_smem[k] = {"bound": "smem_atomic", "achieved": rate, "peak": mb[prim], "unit": "Gop/s",
+                                "frac": rate / mb[prim], "op": prim, "ops_per_launch": nprod}
     step_alg_bytes = 2 * csr_bytes(H.nrows, H.nnz, vbytes) + csr_bytes(H.nrows, nnzC_total, vbytes)
     compulsory = {"bytes_per_step": step_alg_bytes,
                   "GBps": step_alg_bytes / (ms_per_step / 1e3) / 1e9,
@@ -372,7 +403,7 @@ def main():
                        "thr": thr, "seed": args.seed, "parallelism": f"rows{world}",
                        "l2": "inputs larger than L2 (A=B %.0f MB > 126 MB; C %.1f GB written per step)"
                              % (Bbytes / 1e6, csr_bytes(H.nrows, nnzC_total, vbytes) / 1e9)},
-            "roofline": roof, "compulsory": compulsory, "cpu_baseline": cpu, "e2e": e2e,
+            "roofline": roof, "roofline_smem": roof_smem, "compulsory": compulsory, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": launches, "clocks": ck, "threshold_gap": gap,
             "kernel_share": {k: round(v, 4) for k, v in sorted(share.items(), key=lambda kv: -kv[1])},
             "plan": {k: info[k] for k in ("n_empty", "n_light", "n_heavy", "n_ranges", "n_dense", "dense_log2")},

@@ -1,9 +1,11 @@
-// sg_heavy.cu — the HEAVY path (w_i > thr, "more than t"): one CTA (1024 threads)
-// per heavy row, rows taken heaviest-first from a dynamic counter.
+// sg_heavy.cu — the HEAVY path (w_i > thr, "more than t"): one CTA per heavy row
+// (symbolic: 1024 threads, one CTA per SM; numeric: 512 threads, two CTAs per SM so that one CTA's
+// barriers and serial phases overlap the other's products), rows taken heaviest-first from a
+// dynamic counter.
 //
 // Symbolic: the row's products set bits of a shared-memory bitmap over a 2^20-column window;
 // per-8192-column-tile popcounts give u_i and a plan of column RANGES, each holding at most
-// RCAP = 16384 output entries and spanning at most RW_TILES tiles (the numeric accumulator).
+// RCAP = 8192 output entries and spanning at most RW_TILES tiles (the numeric accumulator).
 //
 // Numeric, per range [lo, hi): pass 1 rebuilds the range's bitmap, a block scan turns word
 // popcounts into a rank prefix, pass 2 accumulates every product into a COMPACT fp64 array at
@@ -23,13 +25,13 @@ namespace sg {
 #endif
 constexpr int SYM_T = HEAVY_THREADS;  // symbolic: one CTA of 1024 threads per SM (128 KB bitmap window)
 #ifndef SG_NUM_T
-#define SG_NUM_T 1024
+#define SG_NUM_T 512
 #endif
 #ifndef SG_NUM_OCC
-#define SG_NUM_OCC 1
+#define SG_NUM_OCC 2
 #endif
 #ifndef SG_RCAP
-#define SG_RCAP 16384
+#define SG_RCAP 8192
 #endif
 constexpr int NUM_T = SG_NUM_T;       // numeric: threads per CTA
 constexpr int NUM_OCC = SG_NUM_OCC;   // numeric CTAs per SM (smem-bound)
@@ -37,7 +39,7 @@ constexpr int KC = NUM_T;             // numeric k entries per chunk: one per th
 constexpr int KCS = SYM_T;            // symbolic k entries per chunk
 constexpr int RW_TILES = NUM_T / 32;  // max tiles per numeric range (16 -> 128K columns, 16 KB bitmap)
 constexpr int RW_WORDS = RW_TILES * TW / 32;   // = 256 words per warp in the rank prefix
-constexpr int RCAP = SG_RCAP;         // max entries per numeric range (fp64 accumulator 128 KB)
+constexpr int RCAP = SG_RCAP;         // max entries per numeric range (fp64 accumulator 64 KB)
 constexpr int RHALF = RCAP / 2;       // range key granularity (a range = run of tiles with equal key)
 
 // ------------------------------------------------------------------------------------------------
