@@ -80,6 +80,9 @@ def _L():
         lib.oracle_threshold.restype = i64
         lib.oracle_threshold.argtypes = [CMP, i64, P, P, P, ctypes.POINTER(i64), ctypes.POINTER(u64)]
         lib.oracle_partition.argtypes = [i64, P, ctypes.c_int, P]
+        lib.oracle_row_cost.restype = i64
+        lib.oracle_row_cost.argtypes = [CMP, i64, P, i64, i64]
+        lib.oracle_partition_cost.argtypes = [CMP, i64, P, i64, P, P, ctypes.c_int, P, ctypes.POINTER(i64)]
         lib.oracle_heavy_share.restype = ctypes.c_double
         lib.oracle_heavy_share.argtypes = [i64, P, i64]
         _lib = lib
@@ -234,6 +237,29 @@ def partition(w, G: int) -> np.ndarray:
     cuts = np.empty(G + 1, dtype=np.int64)
     _L().oracle_partition(w.shape[0], _p(w), G, _p(cuts))
     return cuts
+
+
+def sample_comp(res: "SampleResult") -> np.ndarray:
+    """(U_L, W_L, U_H, W_H): sums of u and w over the sampled rows of each class at res.thr."""
+    w, u = res.w, res.u
+    L = (w > 0) & (w <= res.thr)
+    H = w > res.thr
+    return np.array([int(u[L].sum()), int(w[L].sum()), int(u[H].sum()), int(w[H].sum())], dtype=np.int64)
+
+
+def row_cost(cm: CostModel, thr: int, comp, w: int, a: int) -> int:
+    comp = np.ascontiguousarray(comp, dtype=np.int64)
+    return int(_L().oracle_row_cost(ctypes.byref(cm), thr, _p(comp), w, a))
+
+
+def partition_cost(cm: CostModel, thr: int, comp, w, a, G: int) -> tuple[np.ndarray, int]:
+    """Cost-weighted cuts (NEXT #2, R18) and the total modeled cost."""
+    w, a = (np.ascontiguousarray(x, dtype=np.int64) for x in (w, a))
+    comp = np.ascontiguousarray(comp, dtype=np.int64)
+    cuts = np.empty(G + 1, dtype=np.int64)
+    tot = ctypes.c_int64()
+    _L().oracle_partition_cost(ctypes.byref(cm), thr, _p(comp), w.shape[0], _p(w), _p(a), G, _p(cuts), ctypes.byref(tot))
+    return cuts, int(tot.value)
 
 
 # ---- O6 -------------------------------------------------------------------------------------

@@ -245,6 +245,35 @@ void oracle_partition(int64_t n, const int64_t* w, int G, int64_t* cuts) {
     cuts[G] = n;
 }
 
+// ---- O3': cost-weighted partition (reading R18) -----------
+// Alg. 2 balances L_AB, i.e. flops (L215-L218); the paper's "threshold vector" (L106) splits by
+// what each device will SPEND. Here each row's modeled cost is the path cost of O4 at the routing
+// threshold thr: c(i) = 0 if w_i = 0, c_L(w_i, a_i, uh_i) if w_i <= thr, else c_H(w_i, a_i, uh_i),
+// with u_i (unknown before the symbolic pass) estimated from the sample by its class's compression:
+// uh_i = min(w_i, ceil(w_i * U_c / W_c)) for (U_c, W_c) = (sum u, sum w) over the SAMPLED rows of
+// class c (uh_i = w_i when W_c = 0). Cuts: the O3 rule on the prefix of c.
+int64_t oracle_row_cost(const oracle_cost_model* cm, int64_t thr, const int64_t* comp /*U_L, W_L, U_H, W_H*/,
+                        int64_t w, int64_t a) {
+    if (w == 0) return 0;
+    const bool light = w <= thr;
+    const int64_t U = light ? comp[0] : comp[2], Wc = light ? comp[1] : comp[3];
+    int64_t uh = w;
+    if (Wc > 0) {
+        i128 q = ((i128)w * U + Wc - 1) / Wc;
+        if (q < uh) uh = (int64_t)q;
+    }
+    return light ? oracle_cost_L(cm, w, a, uh) : oracle_cost_H(cm, w, a, uh);
+}
+
+void oracle_partition_cost(const oracle_cost_model* cm, int64_t thr, const int64_t* comp, int64_t n,
+                           const int64_t* w, const int64_t* a, int G, int64_t* cuts, int64_t* cost_total) {
+    std::vector<int64_t> c(n);
+    i128 tot = 0;
+    for (int64_t i = 0; i < n; ++i) { c[i] = oracle_row_cost(cm, thr, comp, w[i], a[i]); tot += c[i]; }
+    oracle_partition(n, c.data(), G, cuts);
+    if (cost_total) *cost_total = (int64_t)tot;
+}
+
 // ---- O6: r(t) = 100 * sum_{w_i > t} w_i / W  (split percentage) -------
 double oracle_heavy_share(int64_t n, const int64_t* w, int64_t t) {
     i128 W = 0, H = 0;
