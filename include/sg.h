@@ -79,6 +79,8 @@ typedef struct {
     int64_t thr;              /* the returned threshold */
     int64_t W_est_L, W_est_H; /* sum of w over sampled light / heavy rows at thr */
     int64_t J_min;            /* min_t J(t; S) in ps (unscaled: the n/|S| factor cancels in the argmin) */
+    int64_t U_est_L, U_est_H; /* sum of u = nnz(C_i) over sampled light / heavy rows at thr (the sample's
+                                 per-class compression, input of sg_partition_cost) */
 } sg_sample_report;
 
 /* Per-class counts of a plan (host struct). */
@@ -145,6 +147,19 @@ sg_status sg_cost_curve(const sg_csr_view* A, const sg_csr_view* B, const sg_cos
  * monotone. Part g owns rows [cuts_out[g], cuts_out[g+1]). flops_out = W. Synchronises. */
 sg_status sg_partition(const sg_csr_view* A, const sg_csr_view* B, int nparts,
                        int64_t* cuts_out /*host, nparts+1*/, int64_t* flops_out /*host, nullable*/, void* stream);
+
+/* Cost-weighted contiguous row blocks (reading R18): the rule of
+ * sg_partition applied to the prefix of each row's MODELED path cost at the routing threshold thr
+ * instead of its flops — Alg. 2's split (L216-L218) as a per-device vector (L106) that balances
+ * predicted time. Row i costs 0 if w_i = 0, c_L(w_i, a_i, uh_i) if w_i <= thr, else c_H(w_i, a_i,
+ * uh_i) (the cost model above; cm == NULL: the default), where uh_i = min(w_i, ceil(w_i*U_c/W_c))
+ * estimates u_i from the sample's per-class compression comp = {U_L, W_L, U_H, W_H} (host, 4;
+ * sg_sample_report's U_est_L, W_est_L, U_est_H, W_est_H; uh_i = w_i where W_c = 0).
+ * cuts_out (host, nparts+1); cost_out (host, nullable) = total modeled cost in ps. Synchronises.
+ * Errors: INVALID_ARG (nparts < 1, thr < 0, negative comp, bad model), SHAPE, DTYPE. */
+sg_status sg_partition_cost(const sg_csr_view* A, const sg_csr_view* B, int nparts, int64_t thr,
+                            const sg_cost_model* cm, const int64_t* comp /*host, 4*/,
+                            int64_t* cuts_out /*host, nparts+1*/, int64_t* cost_out /*host, nullable*/, void* stream);
 
 /* Symbolic phase for rows [row_begin, row_end) at threshold thr (0 <= thr <= SG_CAP_L_MAX):
  * classifies rows (EMPTY w=0, LIGHT 0<w<=thr, HEAVY w>thr; L272-L274), computes u_i = nnz(C_i)

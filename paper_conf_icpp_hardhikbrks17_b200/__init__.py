@@ -34,7 +34,7 @@ _STATUS = ["SG_OK", "SG_ERR_INVALID_ARG", "SG_ERR_SHAPE", "SG_ERR_DTYPE", "SG_ER
            "SG_ERR_EMPTY_SAMPLE", "SG_ERR_OOM", "SG_ERR_CUDA", "SG_ERR_NCCL", "SG_ERR_OVERFLOW"]
 
 # every symbol include/sg.h declares (checked by tests/test_abi.py)
-EXPORTS = ["sg_status_string", "sg_version", "sg_default_cost_model", "sg_row_work", "sg_sample_threshold",
+EXPORTS = ["sg_status_string", "sg_version", "sg_default_cost_model", "sg_row_work", "sg_partition_cost", "sg_sample_threshold",
            "sg_exhaustive_threshold", "sg_cost_curve", "sg_partition", "sg_symbolic", "sg_numeric", "sg_gather",
            "sg_plan_get_info", "sg_plan_get_classes", "sg_plan_get_work", "sg_plan_destroy", "sg_sample_rows",
            "sg_profile_enable", "sg_launch_count", "sg_profile_count", "sg_profile_read", "sg_profile_reset",
@@ -66,7 +66,11 @@ class CostModel(ctypes.Structure):
 
 class SampleReport(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int64) for n in (
-        "sample_rows", "sample_nonempty", "thr", "W_est_L", "W_est_H", "J_min")]
+        "sample_rows", "sample_nonempty", "thr", "W_est_L", "W_est_H", "J_min", "U_est_L", "U_est_H")]
+
+    def comp(self):
+        """The sample's per-class compression (U_L, W_L, U_H, W_H) for sg_partition_cost."""
+        return [int(self.U_est_L), int(self.W_est_L), int(self.U_est_H), int(self.W_est_H)]
 
     def as_dict(self):
         return {n: int(getattr(self, n)) for n, _ in self._fields_}
@@ -113,6 +117,7 @@ def load(build_if_missing: bool = True):
         "sg_exhaustive_threshold": (st, [V, V, CM, pi64, pi64, P]),
         "sg_cost_curve": (st, [V, V, CM, i64, P, P, P]),
         "sg_partition": (st, [V, V, ctypes.c_int, P, pi64, P]),
+        "sg_partition_cost": (st, [V, V, ctypes.c_int, i64, CM, P, P, pi64, P]),
         "sg_symbolic": (st, [V, V, i64, i64, i64, P, pi64, ctypes.POINTER(ctypes.c_void_p), P]),
         "sg_numeric": (st, [P, V, V, P, P, P]),
         "sg_gather": (st, [P, P, ctypes.c_int, P, P, P, P, P, P, pi64, P]),
@@ -274,6 +279,20 @@ def sg_partition(A: DeviceCSR, B: DeviceCSR, nparts: int):
     _check(lib().sg_partition(ctypes.byref(A.view()), ctypes.byref(B.view()), nparts,
                               cuts.ctypes.data_as(ctypes.c_void_p), ctypes.byref(W), _stream()), "sg_partition")
     return [int(x) for x in cuts], int(W.value)
+
+
+def sg_partition_cost(A: DeviceCSR, B: DeviceCSR, nparts: int, thr: int, comp, cm=None):
+    """Cost-weighted cuts (NEXT #2, R18): returns (cuts list of nparts+1, total modeled cost
+    in ps). comp = (U_L, W_L, U_H, W_H), e.g. SampleReport.comp() of the sg_sample_threshold call."""
+    import numpy as np
+    _require_cuda()
+    cuts = np.zeros(nparts + 1, dtype=np.int64)
+    cc = np.ascontiguousarray(comp, dtype=np.int64)
+    tot = ctypes.c_int64(0)
+    _check(lib().sg_partition_cost(ctypes.byref(A.view()), ctypes.byref(B.view()), nparts, int(thr), _cmref(cm),
+                                   cc.ctypes.data_as(ctypes.c_void_p), cuts.ctypes.data_as(ctypes.c_void_p),
+                                   ctypes.byref(tot), _stream()), "sg_partition_cost")
+    return [int(x) for x in cuts], int(tot.value)
 
 
 class Plan:

@@ -30,6 +30,8 @@ struct sg_plan {
     int64_t nslots = 0, amax = 0;
     int64_t ndw = 0;                // heavy[0, ndw): dense-window rows (w >= 2^dw_log2), sg_dense.cu
     int32_t* dtc = nullptr;         // their per-tile output counts (ndw x T), from the symbolic pass
+    int4* ditems = nullptr;         // dense-window work items (row, window range)
+    int64_t* ditem_off = nullptr;   // exclusive prefix of items per dense row; [ndw] = item count
     int64_t nskew = 0;              // light rows on the sorted path (column-skewed; sg_light.cu)
     int dw_log2 = 0;
     int2* span = nullptr;           // light rows: [cmin, cmax] of the output columns
@@ -224,6 +226,16 @@ sg_status identify(const Mat& A, const Mat& B, const int64_t* rows, int64_t nr, 
     CK(launch_argmin(cm, hd, hc, hw, sums, dres, s));
     CK(cudaMemcpyAsync(res, dres, sizeof(ThrResult), cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
+    // per-class sums of u over the rows at the chosen threshold (the sample's compression, used by
+    // the cost-weighted split, R18)
+    unsigned long long* us = (unsigned long long*)sc.get(2 * sizeof(unsigned long long));
+    if (!us) return SG_ERR_OOM;
+    unsigned long long hu[2] = {0, 0};
+    CK(launch_class_usum(rs.w, rs.u, nr, res->thr, us, s));
+    CK(cudaMemcpyAsync(hu, us, sizeof(hu), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    res->U_L = (long long)hu[0];
+    res->U_H = (long long)hu[1];
     return SG_OK;
 }
 
@@ -349,6 +361,8 @@ sg_status sg_sample_threshold(const sg_csr_view* A, const sg_csr_view* B, double
         rep->W_est_L = r.W_L;
         rep->W_est_H = r.W_all - r.W_L;
         rep->J_min = r.Jmin;
+        rep->U_est_L = r.U_L;
+        rep->U_est_H = r.U_H;
     }
     return SG_OK;
 }
@@ -386,6 +400,8 @@ sg_status sg_threshold_on_rows(const sg_csr_view* A, const sg_csr_view* B, const
         rep->W_est_L = r.W_L;
         rep->W_est_H = r.W_all - r.W_L;
         rep->J_min = r.Jmin;
+        rep->U_est_L = r.U_L;
+        rep->U_est_H = r.U_H;
     }
     return SG_OK;
 }
@@ -456,6 +472,39 @@ sg_status sg_partition(const sg_csr_view* A, const sg_csr_view* B, int nparts, i
     CK(cudaMemcpyAsync(&W, P + n, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
     if (flops_out) *flops_out = W;
+    return SG_OK;
+}
+
+sg_status sg_partition_cost(const sg_csr_view* A, const sg_csr_view* B, int nparts, int64_t thr,
+                            const sg_cost_model* cm, const int64_t* comp, int64_t* cuts_out, int64_t* cost_out,
+                            void* stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    init_pool();
+    if (nparts < 1 || !cuts_out || !comp || thr < 0) return SG_ERR_INVALID_ARG;
+    for (int q = 0; q < 4; ++q)
+        if (comp[q] < 0) return SG_ERR_INVALID_ARG;
+    sg_status st = validate_pair(A, B, s);
+    if (st != SG_OK) return st;
+    const sg_cost_model* c = cm ? cm : &kDefaultModel;
+    if ((st = check_model(c)) != SG_OK) return st;
+    const int64_t n = A->nrows;
+    Scratch sc(s);
+    int64_t* w = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(n > 0 ? n : 1));
+    int64_t* cost = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(n > 0 ? n : 1));
+    int64_t* P = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(n + 1));
+    void* tmp = sc.get(scan_tmp_bytes(n));
+    int64_t* dcuts = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(nparts + 1));
+    if (!w || !cost || !P || !tmp || !dcuts) return SG_ERR_OOM;
+    Mat a = mat_of(A), b = mat_of(B);
+    CK(launch_row_work(a, b, 0, n, w, s));
+    CK(launch_row_cost(cm_of(c), thr, comp, A->row_ptr, w, n, cost, s));
+    CK(scan_exclusive(cost, P, n, tmp, s));
+    CK(launch_cuts(P, n, nparts, dcuts, s));
+    CK(cudaMemcpyAsync(cuts_out, dcuts, sizeof(int64_t) * (size_t)(nparts + 1), cudaMemcpyDeviceToHost, s));
+    int64_t tot = 0;
+    CK(cudaMemcpyAsync(&tot, P + n, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if (cost_out) *cost_out = tot;
     return SG_OK;
 }
 
@@ -535,7 +584,12 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
         for (int hb2 = 0; hb2 <= 62 - pl->dw_log2 && hb2 < 64; ++hb2) pl->ndw += hh[hb2];
         if (pl->ndw > 0) {
             pl->dtc = (int32_t*)palloc(pl, sizeof(int32_t) * (size_t)pl->ndw * (size_t)pl->T);
-            if (!pl->dtc) return fail(SG_ERR_OOM);
+            pl->ditems = (int4*)palloc(pl, sizeof(int4) * (size_t)dense_items_bound(pl->ndw, pl->p));
+            pl->ditem_off = (int64_t*)palloc(pl, sizeof(int64_t) * (size_t)(pl->ndw + 1));
+            int64_t* dcnt = (int64_t*)palloc(pl, sizeof(int64_t) * (size_t)pl->ndw);
+            void* t3 = palloc(pl, scan_tmp_bytes(pl->ndw));
+            if (!pl->dtc || !pl->ditems || !pl->ditem_off || !dcnt || !t3) return fail(SG_ERR_OOM);
+            CKF(launch_dense_items(pl->heavy, pl->ndw, pl->w, pl->p, dcnt, pl->ditem_off, t3, pl->ditems, s));
         }
         pl->nslots = hb[0];
         pl->amax = hb[1];
@@ -591,7 +645,7 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
             CKP(pl, cudaMallocAsync((void**)&dd, 8 * sizeof(unsigned long long), s));
             CKP(pl, cudaMemsetAsync(dd, 0, 8 * sizeof(unsigned long long), s));
             CKP(pl, launch_num_dense(a, b, pl->heavy, pl->ndw, pl->rb, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
-                                     C_val, pl->counter, pl->gscr, pl->amax, pl->dtc, s, dd));
+                                     C_val, pl->counter, pl->gscr, pl->amax, pl->dtc, pl->ditems, pl->ditem_off + pl->ndw, s, dd));
             unsigned long long h[8];
             CKP(pl, cudaMemcpyAsync(h, dd, sizeof(h), cudaMemcpyDeviceToHost, s));
             CKP(pl, cudaStreamSynchronize(s));
@@ -601,7 +655,7 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
                     h[0] / 1e6, h[1] / 1e6, h[2] / 1e6, h[3] / 1e6, h[4] / 1e6, h[6]);
         } else {
             CKP(pl, launch_num_dense(a, b, pl->heavy, pl->ndw, pl->rb, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
-                                     C_val, pl->counter, pl->gscr, pl->amax, pl->dtc, s));
+                                     C_val, pl->counter, pl->gscr, pl->amax, pl->dtc, pl->ditems, pl->ditem_off + pl->ndw, s));
         }
         CKP(pl, launch_num_heavy(a, b, pl->heavy, pl->ndw, pl->nheavy, pl->rb, pl->range_off, pl->nranges, pl->ranges,
                                  pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter, pl->gscr, pl->amax, s,

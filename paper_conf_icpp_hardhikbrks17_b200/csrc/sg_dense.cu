@@ -9,9 +9,10 @@
 // then emitted in column order (sorted by construction): one block scan of per-thread popcounts
 // (24 columns each), each thread writing its own set bits; only the emitted slots are cleared.
 //
-// The sweep is phase-synchronised: a row starts at the window the CTAs are at on average and wraps
-// around (output offsets from the symbolic pass's tile counts), so concurrent rows read the same
-// column slice of B, which then stays in L2 (DRAM reads of the kernel halved at R-MAT 20).
+// Work items are (row, window range): a row with w_i products is cut into ceil(w_i / DW_CHUNK_W)
+// chunks of consecutive windows (each chunk's output offset from the symbolic pass's tile counts),
+// taken heaviest-first from a dynamic counter, so the heaviest row (9.7M products at R-MAT 20) is
+// spread over many SMs instead of being one CTA's serial tail.
 // Per-k cursors advance window by window: B rows longer than LONG_ROW read their end from the
 // tile-pointer table tp (prefetched one window ahead), short rows count their entries below the
 // window end (cached in shared memory when two-tile windows leave room for it).
@@ -55,39 +56,39 @@ __global__ void __launch_bounds__(DW_T, DW_OCC) k_num_dense(
     Mat A, Mat B, const int32_t* __restrict__ heavy, int64_t ndw, int64_t rb, const int32_t* __restrict__ long_id,
     const uint32_t* __restrict__ tp, int T, const int64_t* __restrict__ C_rp, int32_t* __restrict__ C_col,
     VT* __restrict__ C_val, unsigned long long* counter, int4* __restrict__ gscr, int64_t amax,
-    const int32_t* __restrict__ dtc, unsigned long long* gclock, unsigned long long* __restrict__ dbg) {
+    const int32_t* __restrict__ dtc, const int4* __restrict__ items, const int64_t* __restrict__ nitems,
+    unsigned long long* __restrict__ dbg) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     unsigned long long tph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
     long long t_last = clock64();
     auto mark = [&](int k) { if (dbg && threadIdx.x == 0) { long long t = clock64(); tph[k] += t - t_last; t_last = t; } };
     DenseSmem& S = *reinterpret_cast<DenseSmem*>(smem_raw);
     __shared__ long long s_j;
-    __shared__ int s_t0;
     const int tid = threadIdx.x;
     const int64_t p = B.ncols;
-    const int nwin = (int)((p + WD - 1) / WD);
     int4* gs = gscr + (int64_t)blockIdx.x * amax;  // multi-chunk rows: per-k cursor
     const uint32_t a_vals = smem_addr(S.vals), a_bm = smem_addr(S.bm);
     for (int q = tid; q < WD; q += DW_T) S.vals[q] = 0.0;
     for (int q = tid; q < DW_WORDS + 1; q += DW_T) S.bm[q] = 0u;
+    const int64_t n_items = *nitems;
     while (true) {
         if (tid == 0) s_j = (long long)atomicAdd(counter, 1ull);
         __syncthreads();
-        const int64_t h = s_j;
+        const int64_t it = s_j;
         __syncthreads();
-        if (h >= ndw) break;
+        if (it >= n_items) break;
         mark(0);
+        // work item: windows [ta, tb) of dense row h (a row with w_i products is cut into
+        // ceil(w_i / DW_CHUNK_W) chunks of consecutive windows, so no single row is a tail)
+        const int4 item = items[it];
+        const int64_t h = item.x;
+        const int ta = item.y, tb = item.z;
         const int64_t li = heavy[h];
         const int64_t row = rb + li;
         const int64_t s0 = __ldg(A.rp + row), s1 = __ldg(A.rp + row + 1);
         const int na = (int)(s1 - s0);
         const bool single = na <= DKC;
-        // Phase-synchronised sweep: the row starts at the window the CTAs are currently at on average
-        // (windows completed by all CTAs / CTAs, mod nwin) and wraps around, so that concurrently
-        // running rows read the same column slice of B and it stays in L2 (B > L2 at R-MAT 20).
-        if (tid == 0) s_t0 = (int)((*(volatile unsigned long long*)gclock / gridDim.x) % (unsigned long long)nwin);
-        __syncthreads();
-        const int t0 = s_t0;
+        const int t0 = ta;
         const int64_t lo0 = (int64_t)t0 * WD;
         // output offset of window t0 inside the row: the row's tile counts below tile t0*DW_TILES
         int64_t off0 = 0;
@@ -145,11 +146,8 @@ __global__ void __launch_bounds__(DW_T, DW_OCC) k_num_dense(
             }
         }
         mark(1);
-        for (int j = 0; j < nwin; ++j) {
-            const int t = t0 + j < nwin ? t0 + j : t0 + j - nwin;
-            const int tn = t + 1 < nwin ? t + 1 : 0;  // next window in sweep order
-            if (tid == 0) atomicAdd(gclock, 1ull);
-            if (t == 0) pos = rowbase;                 // wrapped to the row's first window
+        for (int t = ta; t < tb; ++t) {
+            const int tn = t + 1;  // next window
             const int64_t lo = (int64_t)t * WD, hi = min(p, lo + WD);
             const int th = min((t + 1) * DW_TILES, T);  // tile index of hi
             // window-relative shared addresses folded into one base each (lo is a multiple of 32):
@@ -170,7 +168,7 @@ __global__ void __launch_bounds__(DW_T, DW_OCC) k_num_dense(
                     int end;
                     if (lid >= 0) {
                         end = q0 + (int)tpv;
-                        if (j + 1 < nwin) tpv = __ldg(tp + (int64_t)lid * (T + 1) + min((tn + 1) * DW_TILES, T));
+                        if (tn < tb) tpv = __ldg(tp + (int64_t)lid * (T + 1) + min((tn + 1) * DW_TILES, T));
                     } else if constexpr (kShortCache) {
                         int n = 0;
                         #pragma unroll
@@ -180,7 +178,7 @@ __global__ void __launch_bounds__(DW_T, DW_OCC) k_num_dense(
                         end = seg_end(B, cur, e1r, q0, false, 0u, hi);
                     }
                     len = end - cur;
-                    cur = tn == 0 ? q0 : end;
+                    cur = end;
                 }
                 int nk;
                 any = chunk_compact<DW_T, int32_t>(len, beg, a, S.s_beg, S.s_off, S.s_a, &nk, S.wsll);
@@ -202,7 +200,7 @@ __global__ void __launch_bounds__(DW_T, DW_OCC) k_num_dense(
                         beg = g.x;
                         len = end - g.x;
                         if (len > 0) ai = ldv<VT>(A.val, s0 + i);
-                        gs[i] = make_int4(tn == 0 ? kq0 : end, 0, 0, 0);
+                        gs[i] = make_int4(end, 0, 0, 0);
                     }
                     int nk;
                     const int ctot = chunk_compact<DW_T, int32_t>(len, beg, ai, S.s_beg, S.s_off, S.s_a, &nk, S.wsll);
@@ -247,23 +245,64 @@ __global__ void __launch_bounds__(DW_T, DW_OCC) k_num_dense(
         for (int k = 0; k < 8; ++k) atomicAdd(&dbg[k], tph[k]);
 }
 
+// ---- work items: chunks of consecutive windows per dense row ------------------------------------
+constexpr int64_t DW_CHUNK_W = 1 << 19;  // products per work item (about 1/20 of the heaviest R-MAT 20 row)
+
+__device__ __forceinline__ int64_t dense_nchunk(int64_t w, int nwin) {
+    int64_t c = (w + DW_CHUNK_W - 1) / DW_CHUNK_W;
+    return c < 1 ? 1 : (c > nwin ? nwin : c);
+}
+
+__global__ void k_dense_nchunk(const int32_t* __restrict__ heavy, int64_t ndw, const int64_t* __restrict__ w, int nwin,
+                               int64_t* __restrict__ cnt) {
+    const int64_t h = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (h < ndw) cnt[h] = dense_nchunk(w[heavy[h]], nwin);
+}
+
+__global__ void k_dense_items(const int32_t* __restrict__ heavy, int64_t ndw, const int64_t* __restrict__ w, int nwin,
+                              const int64_t* __restrict__ off, int4* __restrict__ items) {
+    const int64_t h = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (h >= ndw) return;
+    const int64_t nc = dense_nchunk(w[heavy[h]], nwin);
+    for (int64_t c = 0; c < nc; ++c)
+        items[off[h] + c] = make_int4((int)h, (int)(c * nwin / nc), (int)((c + 1) * nwin / nc), 0);
+}
+
+int64_t dense_items_bound(int64_t ndw, int64_t p) {
+    const int64_t nwin = (p + WD - 1) / WD;
+    return ndw * (nwin < 1 ? 1 : nwin);
+}
+
+cudaError_t launch_dense_items(const int32_t* heavy, int64_t ndw, const int64_t* w, int64_t p, int64_t* cnt,
+                               int64_t* off, void* scan_tmp, int4* items, cudaStream_t s) {
+    if (ndw <= 0) return cudaSuccess;
+    const int nwin = (int)((p + WD - 1) / WD);
+    const unsigned g = (unsigned)((ndw + 255) / 256);
+    SG_LAUNCH("k_dense_nchunk", s, (k_dense_nchunk<<<g, 256, 0, s>>>(heavy, ndw, w, nwin, cnt)));
+    cudaError_t e = scan_exclusive(cnt, off, ndw, scan_tmp, s);  // off[ndw] = number of items
+    if (e != cudaSuccess) return e;
+    SG_LAUNCH("k_dense_items", s, (k_dense_items<<<g, 256, 0, s>>>(heavy, ndw, w, nwin, off, items)));
+    return cudaGetLastError();
+}
+
 cudaError_t launch_num_dense(const Mat& A, const Mat& B, const int32_t* heavy, int64_t ndw, int64_t rb,
                              const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
                              void* C_val, unsigned long long* counter, int4* gscr, int64_t amax,
-                             const int32_t* dtc, cudaStream_t s, unsigned long long* dbg) {
+                             const int32_t* dtc, const int4* items, const int64_t* nitems, cudaStream_t s,
+                             unsigned long long* dbg) {
     if (ndw <= 0) return cudaSuccess;
     const int smem = (int)sizeof(DenseSmem);
-    cudaError_t e = cudaMemsetAsync(counter, 0, 2 * sizeof(unsigned long long), s);  // row counter, window clock
+    cudaError_t e = cudaMemsetAsync(counter, 0, sizeof(unsigned long long), s);  // item counter
     if (e != cudaSuccess) return e;
-    const int grid = (int)(ndw < 148 * DW_OCC ? ndw : 148 * DW_OCC);
+    const int grid = 148 * DW_OCC;  // persistent; CTAs beyond the item count exit at once
     if (A.dt == 0) {
         if ((e = cudaFuncSetAttribute(k_num_dense<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
         SG_LAUNCH("k_num_dense", s, (k_num_dense<double><<<grid, DW_T, smem, s>>>(A, B, heavy, ndw, rb, long_id, tp, T, C_rp,
-                                                                                  C_col, (double*)C_val, counter, gscr, amax, dtc, counter + 1, dbg)));
+                                                                                  C_col, (double*)C_val, counter, gscr, amax, dtc, items, nitems, dbg)));
     } else {
         if ((e = cudaFuncSetAttribute(k_num_dense<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
         SG_LAUNCH("k_num_dense", s, (k_num_dense<float><<<grid, DW_T, smem, s>>>(A, B, heavy, ndw, rb, long_id, tp, T, C_rp,
-                                                                                 C_col, (float*)C_val, counter, gscr, amax, dtc, counter + 1, dbg)));
+                                                                                 C_col, (float*)C_val, counter, gscr, amax, dtc, items, nitems, dbg)));
     }
     return cudaGetLastError();
 }

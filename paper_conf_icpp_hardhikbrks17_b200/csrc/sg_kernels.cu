@@ -279,6 +279,60 @@ __device__ __forceinline__ long long costH(const CostModelD& cm, long long w, lo
     return cm.kH + cm.lH * w + cm.tH * a * R + cm.mH * u;
 }
 
+// ---- NEXT #2: modeled per-row cost for the cost-weighted split (R18) -----------------
+// c_i = 0 (w = 0), c_L(w, a, uh) (w <= thr), c_H(w, a, uh) (w > thr); uh = min(w, ceil(w U_c / W_c)).
+__global__ void k_row_cost(CostModelD cm, long long thr, long long UL, long long WL, long long UH, long long WH,
+                           const int64_t* __restrict__ arp, const int64_t* __restrict__ w, int64_t n,
+                           int64_t* __restrict__ cost) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const long long wi = w[i];
+        if (wi == 0) { cost[i] = 0; continue; }
+        const long long ai = arp[i + 1] - arp[i];
+        const bool light = wi <= thr;
+        const long long U = light ? UL : UH, Wc = light ? WL : WH;
+        long long uh = wi;
+        if (Wc > 0) {
+            const __int128 q = ((__int128)wi * U + Wc - 1) / Wc;
+            if (q < (__int128)uh) uh = (long long)q;
+        }
+        cost[i] = light ? costL(cm, wi, ai, uh) : costH(cm, wi, ai, uh);
+    }
+}
+
+cudaError_t launch_row_cost(const CostModelD& cm, int64_t thr, const int64_t* comp, const int64_t* arp,
+                            const int64_t* w, int64_t n, int64_t* cost, cudaStream_t s) {
+    if (n <= 0) return cudaSuccess;
+    SG_LAUNCH("k_row_cost", s, k_row_cost<<<grid_for(n, 256, 148 * 8), 256, 0, s>>>(cm, thr, comp[0], comp[1], comp[2],
+                                                                                       comp[3], arp, w, n, cost));
+    return cudaGetLastError();
+}
+
+// per-class sums of u over a row list at a known threshold: out[0] = sum u (0 < w <= thr),
+// out[1] = sum u (w > thr)
+__global__ void k_class_usum(const int64_t* __restrict__ w, const int64_t* __restrict__ u, int64_t nr, long long thr,
+                             unsigned long long* out) {
+    unsigned long long sl = 0, sh = 0;
+    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < nr; j += (int64_t)gridDim.x * blockDim.x) {
+        const long long wj = w[j];
+        if (wj == 0) continue;
+        if (wj <= thr) sl += (unsigned long long)u[j]; else sh += (unsigned long long)u[j];
+    }
+    sl = warp_sum(sl);
+    sh = warp_sum(sh);
+    if ((threadIdx.x & 31) == 0) {
+        if (sl) atomicAdd(&out[0], sl);
+        if (sh) atomicAdd(&out[1], sh);
+    }
+}
+
+cudaError_t launch_class_usum(const int64_t* w, const int64_t* u, int64_t nr, int64_t thr, unsigned long long* out,
+                              cudaStream_t s) {
+    cudaError_t e = cudaMemsetAsync(out, 0, 2 * sizeof(unsigned long long), s);
+    if (e != cudaSuccess || nr <= 0) return e;
+    SG_LAUNCH("k_class_usum", s, k_class_usum<<<grid_for(nr, 256, 148 * 4), 256, 0, s>>>(w, u, nr, thr, out));
+    return cudaGetLastError();
+}
+
 __global__ void k_cost_hist(CostModelD cm, const int64_t* __restrict__ w, const int64_t* __restrict__ a,
                             const int64_t* __restrict__ u, int64_t nr, unsigned long long* hd, unsigned long long* hc,
                             unsigned long long* hw, unsigned long long* sums) {

@@ -180,6 +180,39 @@ def test_partition_plateaus_and_ties():
         assert cuts == list(oracle.partition(oracle.row_work(A, A), G))
 
 
+@pytest.mark.parametrize("name", ["C1", "rmat12", "rmat12u", "rmat14u"])
+@pytest.mark.parametrize("G", [1, 2, 3, 8])
+def test_partition_cost_bit_exact(name, G):
+    """NEXT #2 (R18): the sample's per-class compression and the cost-weighted cuts,
+    bit-exact against the oracle (permuted and un-permuted R-MAT: hubs at low row ids)."""
+    A = gen.rmat(int(name[4:-1]), 16, seed=1, permute=False) if name.endswith("u") else gen.config(name)
+    dA = _dev(A)
+    cm = sg.sg_default_cost_model()
+    thr, rep = sg.sg_sample_threshold(dA, dA, 0.05, 3, cm)
+    o = oracle.sampled_threshold(A, A, 0.05, 3, _model_from(cm))
+    assert thr == o.thr
+    comp = oracle.sample_comp(o)
+    assert [rep["U_est_L"], rep["W_est_L"], rep["U_est_H"], rep["W_est_H"]] == comp.tolist()
+    cuts, tot = sg.sg_partition_cost(dA, dA, G, thr, comp.tolist(), cm)
+    ocuts, otot = oracle.partition_cost(_model_from(cm), thr, comp, oracle.row_work(A, A), np.diff(A.row_ptr), G)
+    assert cuts == ocuts.tolist() and tot == otot
+
+
+def test_partition_cost_edge_cases():
+    A = gen.config("rmat10")
+    dA = _dev(A)
+    cm = sg.sg_default_cost_model()
+    w, a = oracle.row_work(A, A), np.diff(A.row_ptr)
+    for thr, comp in [(0, [0, 0, 0, 0]), (4096, [5, 7, 0, 0]), (100, [1, 1, 1, 1]), (1, [0, 3, 9, 10])]:
+        cuts, tot = sg.sg_partition_cost(dA, dA, 5, thr, comp, cm)
+        ocuts, otot = oracle.partition_cost(_model_from(cm), thr, comp, w, a, 5)
+        assert cuts == ocuts.tolist() and tot == otot
+    with pytest.raises(RuntimeError):
+        sg.sg_partition_cost(dA, dA, 0, 10, [1, 1, 1, 1], cm)
+    with pytest.raises(RuntimeError):
+        sg.sg_partition_cost(dA, dA, 2, 10, [-1, 1, 1, 1], cm)
+
+
 # ---- a5-a8 symbolic + numeric ---------------------------------------------------------------------
 
 @pytest.mark.parametrize("name", ["C1", "rmat10", "rmat12"])
