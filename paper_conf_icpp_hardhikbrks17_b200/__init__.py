@@ -282,7 +282,7 @@ def sg_partition(A: DeviceCSR, B: DeviceCSR, nparts: int):
 
 
 def sg_partition_cost(A: DeviceCSR, B: DeviceCSR, nparts: int, thr: int, comp, cm=None):
-    """Cost-weighted cuts (NEXT #2, R18): returns (cuts list of nparts+1, total modeled cost
+    """Cost-weighted cuts (NEXT #2, R19): returns (cuts list of nparts+1, total modeled cost
     in ps). comp = (U_L, W_L, U_H, W_H), e.g. SampleReport.comp() of the sg_sample_threshold call."""
     import numpy as np
     _require_cuda()

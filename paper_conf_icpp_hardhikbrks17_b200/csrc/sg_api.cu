@@ -227,7 +227,7 @@ sg_status identify(const Mat& A, const Mat& B, const int64_t* rows, int64_t nr, 
     CK(cudaMemcpyAsync(res, dres, sizeof(ThrResult), cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
     // per-class sums of u over the rows at the chosen threshold (the sample's compression, used by
-    // the cost-weighted split, R18)
+    // the cost-weighted split, R19)
     unsigned long long* us = (unsigned long long*)sc.get(2 * sizeof(unsigned long long));
     if (!us) return SG_ERR_OOM;
     unsigned long long hu[2] = {0, 0};

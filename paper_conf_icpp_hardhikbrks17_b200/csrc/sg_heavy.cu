@@ -41,6 +41,7 @@ constexpr int RW_TILES = NUM_T / 32;  // max tiles per numeric range (16 -> 128K
 constexpr int RW_WORDS = RW_TILES * TW / 32;   // = 256 words per warp in the rank prefix
 constexpr int RCAP = SG_RCAP;         // max entries per numeric range (fp64 accumulator 64 KB)
 constexpr int RHALF = RCAP / 2;       // range key granularity (a range = run of tiles with equal key)
+static_assert(TW <= RCAP, "a single full tile must fit the numeric accumulator");
 
 // ------------------------------------------------------------------------------------------------
 // B tile pointers: for B rows longer than LONG_ROW, tp[id][t] = #entries with col < t*TW
@@ -141,8 +142,9 @@ __global__ void k_range_bounds(const int32_t* __restrict__ heavy, int64_t nh, co
     int64_t mu = wi < p ? wi : p;
     int64_t T = (p + TW - 1) / TW;
     int64_t nwin = (p + WIN - 1) / WIN;
-    // distinct keys per window <= u_win / RHALF + 1 + (tiles per window / RW_TILES)
-    int64_t b = mu / RHALF + nwin * (1 + (WIN / TW) / RW_TILES) + 1;
+    // distinct keys per window <= u_win / RHALF + 1 + (tiles per window / RW_TILES); each big tile
+    // (> RHALF entries, at most u / RHALF of them) adds at most two more range starts
+    int64_t b = 3 * (mu / RHALF) + nwin * (1 + (WIN / TW) / RW_TILES) + 1;
     bounds[j] = b < T ? b : T;
 }
 
@@ -222,7 +224,9 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_sym_heavy(Mat A, Mat B, co
             }
             __syncthreads();
             // range plan (warp 0): key(t) = (ceil(P_t / RHALF) - 1, t / RW_TILES); a range is a run of
-            // equal keys -> count <= RHALF + cnt(first tile) <= RCAP, width <= RW_TILES tiles.
+            // equal keys, and a BIG tile (more than RHALF entries) is a range of its own -> a range without
+            // a big tile holds <= RHALF + cnt(first tile) <= 2 RHALF = RCAP entries, a big tile alone
+            // <= TW <= RCAP; width <= RW_TILES tiles.
             if (wid == 0 && j < ndw) {  // dense-window row (sg_dense.cu): u and its tile counts, no range plan
                 int c = 0;
                 const int64_t Tall = (p + TW - 1) / TW;
@@ -242,15 +246,17 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_sym_heavy(Mat A, Mat B, co
                 for (int q = 0; q < 4; ++q) {
                     const int t = 4 * lane + q;
                     pre += c4[q];
-                    key[q] = ((pre + RHALF - 1) / RHALF - 1) * 8 + t / RW_TILES;
+                    key[q] = ((pre + RHALF - 1) / RHALF - 1) * (WIN / TW / RW_TILES) + t / RW_TILES;
                     if (t < nt) Ps[t] = pre;
                 }
                 const int prevkey = __shfl_up_sync(FULL, key[3], 1);
+                const bool prevbig = __shfl_up_sync(FULL, c4[3], 1) > RHALF;
                 #pragma unroll
                 for (int q = 0; q < 4; ++q) {
                     const int t = 4 * lane + q;
                     const int kp = q == 0 ? prevkey : key[q - 1];
-                    if (t < nt) st[t] = (t == 0 || key[q] != kp) ? 1 : 0;
+                    const bool bigp = q == 0 ? prevbig : c4[q - 1] > RHALF;
+                    if (t < nt) st[t] = (t == 0 || key[q] != kp || c4[q] > RHALF || bigp) ? 1 : 0;
                 }
                 __syncwarp();
                 for (int t0 = 0; t0 < nt; t0 += 32) {

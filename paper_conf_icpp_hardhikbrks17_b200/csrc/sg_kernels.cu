@@ -279,7 +279,7 @@ __device__ __forceinline__ long long costH(const CostModelD& cm, long long w, lo
     return cm.kH + cm.lH * w + cm.tH * a * R + cm.mH * u;
 }
 
-// ---- NEXT #2: modeled per-row cost for the cost-weighted split (R18) -----------------
+// ---- NEXT #2: modeled per-row cost for the cost-weighted split (R19) -----------------
 // c_i = 0 (w = 0), c_L(w, a, uh) (w <= thr), c_H(w, a, uh) (w > thr); uh = min(w, ceil(w U_c / W_c)).
 __global__ void k_row_cost(CostModelD cm, long long thr, long long UL, long long WL, long long UH, long long WH,
                            const int64_t* __restrict__ arp, const int64_t* __restrict__ w, int64_t n,

@@ -183,7 +183,7 @@ def test_partition_plateaus_and_ties():
 @pytest.mark.parametrize("name", ["C1", "rmat12", "rmat12u", "rmat14u"])
 @pytest.mark.parametrize("G", [1, 2, 3, 8])
 def test_partition_cost_bit_exact(name, G):
-    """NEXT #2 (R18): the sample's per-class compression and the cost-weighted cuts,
+    """NEXT #2 (R19): the sample's per-class compression and the cost-weighted cuts,
     bit-exact against the oracle (permuted and un-permuted R-MAT: hubs at low row ids)."""
     A = gen.rmat(int(name[4:-1]), 16, seed=1, permute=False) if name.endswith("u") else gen.config(name)
     dA = _dev(A)
@@ -214,6 +214,40 @@ def test_partition_cost_edge_cases():
 
 
 # ---- a5-a8 symbolic + numeric ---------------------------------------------------------------------
+
+def _csr_from_sets(nrows, ncols, rows, seed):
+    rng = np.random.default_rng(seed)
+    rp, cols = [0], []
+    for r in rows:
+        c = np.unique(np.asarray(r, dtype=np.int64))
+        cols.append(c)
+        rp.append(rp[-1] + len(c))
+    col = np.concatenate(cols).astype(np.int32) if cols else np.zeros(0, np.int32)
+    val = 0.5 + rng.random(col.shape[0])
+    return gen.CSR(nrows, ncols, np.array(rp, np.int64), col, val, "sets")
+
+
+@pytest.mark.parametrize("f32", [False, True])
+def test_rank_kernel_big_tile_ranges(f32):
+    """A heavy (rank-kernel) row whose columns crowd one 8192-column tile far beyond half the range
+    capacity: such a tile must form a range of its own (sg_heavy.cu range plan)."""
+    rng = np.random.default_rng(5)
+    p, m = 1 << 20, 200
+    brows = []
+    for k in range(m):
+        brows.append(np.concatenate([rng.integers(5 * 8192, 6 * 8192, 100), rng.integers(0, 8192, 10),
+                                     rng.integers(9 * 8192, 10 * 8192, 10), rng.integers(0, p, 5)]))
+    B = _csr_from_sets(m, p, brows, 1)
+    A = _csr_from_sets(5, m, [np.arange(m), np.arange(0, m, 2), [], rng.integers(0, m, 10), np.arange(150)], 2)
+    if f32:
+        A, B = A.astype("f32"), B.astype("f32")
+    (rp, col, val), info, cls = _full_product(A, B, 0)
+    assert info["n_heavy"] == 4 and info["n_dense"] == 0
+    R = oracle.spgemm(A, B, with_absmag=True)
+    assert np.array_equal(rp, R.row_ptr)
+    assert int(np.diff(rp)[0]) > 10000
+    compare_rows(rp, col, val, R, "f32" if f32 else "f64")
+
 
 @pytest.mark.parametrize("name", ["C1", "rmat10", "rmat12"])
 @pytest.mark.parametrize("thr", [0, 1, 64, 300, 4096])

@@ -1,4 +1,4 @@
-"""Pins for the oracle's cost-weighted partition (reading R18):
+"""Pins for the oracle's cost-weighted partition (reading R19):
 Alg. 2's closest-prefix split on the modeled per-row cost of O4 (L87-L89) instead
 of the flops L_AB (L206) — the per-device "threshold vector" of L106."""
 import json
