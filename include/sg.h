@@ -148,7 +148,7 @@ sg_status sg_cost_curve(const sg_csr_view* A, const sg_csr_view* B, const sg_cos
 sg_status sg_partition(const sg_csr_view* A, const sg_csr_view* B, int nparts,
                        int64_t* cuts_out /*host, nparts+1*/, int64_t* flops_out /*host, nullable*/, void* stream);
 
-/* Cost-weighted contiguous row blocks (reading R18): the rule of
+/* Cost-weighted contiguous row blocks (reading R19): the rule of
  * sg_partition applied to the prefix of each row's MODELED path cost at the routing threshold thr
  * instead of its flops — Alg. 2's split (L216-L218) as a per-device vector (L106) that balances
  * predicted time. Row i costs 0 if w_i = 0, c_L(w_i, a_i, uh_i) if w_i <= thr, else c_H(w_i, a_i,

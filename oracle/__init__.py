@@ -253,7 +253,7 @@ def row_cost(cm: CostModel, thr: int, comp, w: int, a: int) -> int:
 
 
 def partition_cost(cm: CostModel, thr: int, comp, w, a, G: int) -> tuple[np.ndarray, int]:
-    """Cost-weighted cuts (NEXT #2, R18) and the total modeled cost."""
+    """Cost-weighted cuts (NEXT #2, R19) and the total modeled cost."""
     w, a = (np.ascontiguousarray(x, dtype=np.int64) for x in (w, a))
     comp = np.ascontiguousarray(comp, dtype=np.int64)
     cuts = np.empty(G + 1, dtype=np.int64)

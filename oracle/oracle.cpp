@@ -245,7 +245,7 @@ void oracle_partition(int64_t n, const int64_t* w, int G, int64_t* cuts) {
     cuts[G] = n;
 }
 
-// ---- O3': cost-weighted partition (reading R18) -----------
+// ---- O3': cost-weighted partition (reading R19) -----------
 // Alg. 2 balances L_AB, i.e. flops (L215-L218); the paper's "threshold vector" (L106) splits by
 // what each device will SPEND. Here each row's modeled cost is the path cost of O4 at the routing
 // threshold thr: c(i) = 0 if w_i = 0, c_L(w_i, a_i, uh_i) if w_i <= thr, else c_H(w_i, a_i, uh_i),

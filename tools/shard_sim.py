@@ -3,7 +3,7 @@
 Each rank's work is independent given a replicated B (C_i depends only on A_i and B), so the time a
 G-GPU run spends in symbolic + numeric is max_g T(shard g), where T(shard g) is the time of rank g's
 rows on a whole B200. This tool times every shard alone on the one GPU, for the flops split of Alg. 2
-(sg_partition) and the cost-weighted split (sg_partition_cost, R18), and
+(sg_partition) and the cost-weighted split (sg_partition_cost, R19), and
 reports per-shard times, the imbalance max/mean, and the projected G-GPU makespan (compute only: the
 sampling step, the B broadcast and the NCCL assembly are not included). Not a multi-GPU measurement.
 
