@@ -50,6 +50,8 @@ def parse():
     ap.add_argument("--config", default="C3")
     ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
     ap.add_argument("--seed", type=int, default=1)
+    ap.add_argument("--split", default="cost", choices=["cost", "flops"],
+                    help="N > 1: cost-weighted split (sg_partition_cost, DESIGN.md §7.7) or Alg. 2's flops split")
     ap.add_argument("--sample-frac", type=float, default=0.01)
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-e2e", action="store_true")
@@ -238,11 +240,17 @@ def main():
     vbytes = 8 if args.dtype == "f64" else 4
     stream = torch.cuda.current_stream()
 
+    W_all = sg.sg_partition(A, A, 1)[1]  # the workload's W (a constant of the matrix)
     cbuf = {}  # C buffers reused across steps (same nnz every step; allocation kept out of the loop)
 
     def step(Ad, with_values=False):
         thr, rep = sg.sg_sample_threshold(Ad, Ad, args.sample_frac, args.seed)
-        cuts, W = sg.sg_partition(Ad, Ad, world)
+        if world > 1 and args.split == "cost":
+            comp = [rep["U_est_L"], rep["W_est_L"], rep["U_est_H"], rep["W_est_H"]]
+            cuts, _cost = sg.sg_partition_cost(Ad, Ad, world, thr, comp)
+            W = W_all
+        else:
+            cuts, W = sg.sg_partition(Ad, Ad, world)
         plan = sg.sg_symbolic(Ad, Ad, thr, cuts[rank], cuts[rank + 1])
         if cbuf.get("nnz") != plan.nnz:
             cbuf.clear()
@@ -400,7 +408,7 @@ def main():
             "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
             "config": {"workload": WORKLOADS.get(args.config, args.config), "config_id": args.config,
                        "n": H.nrows, "nnz_A": H.nnz, "W": W, "nnz_C": nnzC_total, "sample_frac": args.sample_frac,
-                       "thr": thr, "seed": args.seed, "parallelism": f"rows{world}",
+                       "thr": thr, "seed": args.seed, "parallelism": f"rows{world}", "split": args.split if world > 1 else "none",
                        "l2": "inputs larger than L2 (A=B %.0f MB > 126 MB; C %.1f GB written per step)"
                              % (Bbytes / 1e6, csr_bytes(H.nrows, nnzC_total, vbytes) / 1e9)},
             "roofline": roof, "roofline_smem": roof_smem, "compulsory": compulsory, "cpu_baseline": cpu, "e2e": e2e,

@@ -104,6 +104,8 @@ const char* sg_status_string(sg_status st);
 const char* sg_version(void);
 /* The calibrated default cost model. */
 void sg_default_cost_model(sg_cost_model* out /*host*/);
+/* The default model of sg_partition_cost: fitted to measured per-shard times. */
+void sg_default_partition_model(sg_cost_model* out /*host*/);
 
 /* Row work volume w_i = sum_{k in A_i} nnz(B_k) = L_AB[i] (Alg. 2 l.1 L215) for rows
  * [row_begin, row_end) into w_out[0 .. row_end-row_begin) (device, caller-owned). If total_out is
@@ -152,7 +154,7 @@ sg_status sg_partition(const sg_csr_view* A, const sg_csr_view* B, int nparts,
  * sg_partition applied to the prefix of each row's MODELED path cost at the routing threshold thr
  * instead of its flops — Alg. 2's split (L216-L218) as a per-device vector (L106) that balances
  * predicted time. Row i costs 0 if w_i = 0, c_L(w_i, a_i, uh_i) if w_i <= thr, else c_H(w_i, a_i,
- * uh_i) (the cost model above; cm == NULL: the default), where uh_i = min(w_i, ceil(w_i*U_c/W_c))
+ * uh_i) (the cost model above; cm == NULL: sg_default_partition_model), where uh_i = min(w_i, ceil(w_i*U_c/W_c))
  * estimates u_i from the sample's per-class compression comp = {U_L, W_L, U_H, W_H} (host, 4;
  * sg_sample_report's U_est_L, W_est_L, U_est_H, W_est_H; uh_i = w_i where W_c = 0).
  * cuts_out (host, nparts+1); cost_out (host, nullable) = total modeled cost in ps. Synchronises.

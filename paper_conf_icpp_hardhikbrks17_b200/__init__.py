@@ -34,7 +34,7 @@ _STATUS = ["SG_OK", "SG_ERR_INVALID_ARG", "SG_ERR_SHAPE", "SG_ERR_DTYPE", "SG_ER
            "SG_ERR_EMPTY_SAMPLE", "SG_ERR_OOM", "SG_ERR_CUDA", "SG_ERR_NCCL", "SG_ERR_OVERFLOW"]
 
 # every symbol include/sg.h declares (checked by tests/test_abi.py)
-EXPORTS = ["sg_status_string", "sg_version", "sg_default_cost_model", "sg_row_work", "sg_partition_cost", "sg_sample_threshold",
+EXPORTS = ["sg_status_string", "sg_version", "sg_default_cost_model", "sg_row_work", "sg_partition_cost", "sg_default_partition_model", "sg_sample_threshold",
            "sg_exhaustive_threshold", "sg_cost_curve", "sg_partition", "sg_symbolic", "sg_numeric", "sg_gather",
            "sg_plan_get_info", "sg_plan_get_classes", "sg_plan_get_work", "sg_plan_destroy", "sg_sample_rows",
            "sg_profile_enable", "sg_launch_count", "sg_profile_count", "sg_profile_read", "sg_profile_reset",
@@ -110,6 +110,7 @@ def load(build_if_missing: bool = True):
         "sg_status_string": (ctypes.c_char_p, [st]),
         "sg_version": (ctypes.c_char_p, []),
         "sg_default_cost_model": (None, [CM]),
+        "sg_default_partition_model": (None, [CM]),
         "sg_row_work": (st, [V, V, i64, i64, P, pi64, P]),
         "sg_sample_rows": (st, [i64, i64, ctypes.c_double, u64, P, i64, pi64, P]),
         "sg_sample_threshold": (st, [V, V, ctypes.c_double, u64, CM, pi64, ctypes.POINTER(SampleReport), P]),
@@ -200,6 +201,13 @@ class DeviceCSR:
 def sg_default_cost_model() -> CostModel:
     cm = CostModel()
     lib().sg_default_cost_model(ctypes.byref(cm))
+    return cm
+
+
+def sg_default_partition_model() -> CostModel:
+    """The cost model sg_partition_cost uses when none is given (fitted to measured shard times)."""
+    cm = CostModel()
+    lib().sg_default_partition_model(ctypes.byref(cm))
     return cm
 
 

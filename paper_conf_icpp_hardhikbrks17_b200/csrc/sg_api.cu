@@ -159,6 +159,14 @@ const sg_cost_model kDefaultModel = {
     /*kappa_H*/ 17907513, /*lambda_H*/ 1102, /*tau_H*/ 68338, /*mu_H*/ 209,
     /*tiles_fixed*/ 1, /*capu*/ 12288, /*cap_L*/ SG_CAP_L_MAX};
 
+// Partition model (reading R19): fitted by tools/fit_partition_model.py to 88 measured
+// shard times (R-MAT 20 and 18, permuted and un-permuted, G = 2..16; profiles/r01s4_partition_model_fit.json):
+// a light row costs rho_L per output, a heavy row lambda_H per product (ps of SM time).
+const sg_cost_model kPartitionModel = {
+    /*kappa_L*/ 0, /*lambda_L*/ 0, /*sigma_L*/ 0, /*rho_L*/ 22705,
+    /*kappa_H*/ 0, /*lambda_H*/ 2064, /*tau_H*/ 0, /*mu_H*/ 0,
+    /*tiles_fixed*/ 1, /*capu*/ 0, /*cap_L*/ SG_CAP_L_MAX};
+
 // Identify over a row list (rows == nullptr: rows [0, nr)). Computes w, a, u of those rows on the
 // device (exact sample-symbolic at routing threshold cap_L), then the cost histogram.
 struct RowStats {
@@ -269,6 +277,10 @@ const char* sg_version(void) { return "sg 0.1.0 sm_100a"; }
 
 void sg_default_cost_model(sg_cost_model* out) {
     if (out) *out = kDefaultModel;
+}
+
+void sg_default_partition_model(sg_cost_model* out) {
+    if (out) *out = kPartitionModel;
 }
 
 sg_status sg_row_work(const sg_csr_view* A, const sg_csr_view* B, int64_t row_begin, int64_t row_end, int64_t* w_out,
@@ -485,7 +497,7 @@ sg_status sg_partition_cost(const sg_csr_view* A, const sg_csr_view* B, int npar
         if (comp[q] < 0) return SG_ERR_INVALID_ARG;
     sg_status st = validate_pair(A, B, s);
     if (st != SG_OK) return st;
-    const sg_cost_model* c = cm ? cm : &kDefaultModel;
+    const sg_cost_model* c = cm ? cm : &kPartitionModel;
     if ((st = check_model(c)) != SG_OK) return st;
     const int64_t n = A->nrows;
     Scratch sc(s);

@@ -24,7 +24,7 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, q):
+def _worker(rank, world, port, q, split="flops"):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
@@ -34,9 +34,14 @@ def _worker(rank, world, port, q):
         import paper_conf_icpp_hardhikbrks17_b200 as sg
         A = gen.config("rmat11")
         w = oracle.row_work(A, A)
-        cuts = oracle.partition(w, world)
         cm = oracle.CostModel(**sg.sg_default_cost_model().as_dict())
-        thr = oracle.sampled_threshold(A, A, 0.05, 3, cm, w_all=w).thr
+        smp = oracle.sampled_threshold(A, A, 0.05, 3, cm, w_all=w)
+        thr = smp.thr
+        if split == "cost":  # cost-weighted split with the default partition model
+            pm = oracle.CostModel(**sg.sg_default_partition_model().as_dict())
+            cuts, _ = oracle.partition_cost(pm, thr, oracle.sample_comp(smp), w, np.diff(A.row_ptr), world)
+        else:
+            cuts = oracle.partition(w, world)
         mine = [cuts.tolist(), thr]
         every = [None] * world
         dist.all_gather_object(every, mine)
@@ -62,13 +67,14 @@ def _worker(rank, world, port, q):
         dist.destroy_process_group()
 
 
-def test_two_rank_partition_and_assembly():
+@pytest.mark.parametrize("split", ["flops", "cost"])
+def test_two_rank_partition_and_assembly(split):
     import oracle
     import sginputs as gen
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q, split)) for r in range(2)]
     for p in procs:
         p.start()
     res = [q.get(timeout=300) for _ in range(2)]

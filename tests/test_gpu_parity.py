@@ -198,6 +198,21 @@ def test_partition_cost_bit_exact(name, G):
     assert cuts == ocuts.tolist() and tot == otot
 
 
+@pytest.mark.parametrize("name", ["rmat12", "rmat14u"])
+def test_partition_cost_default_partition_model(name):
+    """cm = NULL selects sg_default_partition_model; same cuts as the oracle with it."""
+    A = gen.rmat(int(name[4:-1]), 16, seed=1, permute=False) if name.endswith("u") else gen.config(name)
+    dA = _dev(A)
+    thr, rep = sg.sg_sample_threshold(dA, dA, 0.05, 3)
+    comp = [rep["U_est_L"], rep["W_est_L"], rep["U_est_H"], rep["W_est_H"]]
+    pm = sg.sg_default_partition_model()
+    assert pm.rho_L > 0 and pm.lambda_H > 0
+    for G in (2, 8):
+        cuts, tot = sg.sg_partition_cost(dA, dA, G, thr, comp)
+        ocuts, otot = oracle.partition_cost(_model_from(pm), thr, comp, oracle.row_work(A, A), np.diff(A.row_ptr), G)
+        assert cuts == ocuts.tolist() and tot == otot
+
+
 def test_partition_cost_edge_cases():
     A = gen.config("rmat10")
     dA = _dev(A)

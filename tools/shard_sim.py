@@ -26,6 +26,9 @@ def main():
     ap.add_argument("--G", type=int, nargs="+", default=[8])
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--sample-frac", type=float, default=0.01)
+    ap.add_argument("--kinds", nargs="+", default=["flops", "cost"])
+    ap.add_argument("--seed", type=int, default=1, help="matrix seed")
+    ap.add_argument("--cm-json", default="", help="cost model for the cost split (tools/fit_partition_model.py output)")
     ap.add_argument("--out", default="")
     a = ap.parse_args()
     import torch
@@ -33,16 +36,21 @@ def main():
     import paper_conf_icpp_hardhikbrks17_b200 as sg
     if a.unperm:
         scale = {"C3": 20, "R18": 18, "C4": 22}[a.config]
-        H = gen.rmat(scale, 16, seed=1, permute=False)
+        H = gen.rmat(scale, 16, seed=a.seed, permute=False)
     else:
-        H = gen.config(a.config)
+        H = gen.config(a.config, seed=a.seed)
     A = sg.DeviceCSR.from_host(H)
     cm = sg.sg_default_cost_model()
+    pcm = cm
+    if a.cm_json:
+        pcm = sg.sg_default_cost_model()
+        for k, v in json.load(open(a.cm_json))["model"].items():
+            setattr(pcm, k, int(v))
     thr, rep = sg.sg_sample_threshold(A, A, a.sample_frac, 1, cm)
     comp = [rep["U_est_L"], rep["W_est_L"], rep["U_est_H"], rep["W_est_H"]]
     _, W = sg.sg_partition(A, A, 1)
     w = sg.sg_row_work(A, A).cpu()
-    out = {"config": a.config, "unperm": a.unperm, "n": H.nrows, "W": W, "thr": thr, "comp": comp, "splits": {}}
+    out = {"config": a.config, "unperm": a.unperm, "seed": a.seed, "n": H.nrows, "W": W, "thr": thr, "comp": comp, "splits": {}}
 
     def shard_ms(r0, r1):
         best = None
@@ -63,11 +71,11 @@ def main():
         return best
 
     for G in a.G:
-        for kind in ("flops", "cost"):
+        for kind in a.kinds:
             if kind == "flops":
                 cuts, _ = sg.sg_partition(A, A, G)
             else:
-                cuts, _ = sg.sg_partition_cost(A, A, G, thr, comp, cm)
+                cuts, _ = sg.sg_partition_cost(A, A, G, thr, comp, pcm)
             ts, ws = [], []
             for g in range(G):
                 ts.append(shard_ms(cuts[g], cuts[g + 1]))
