@@ -453,3 +453,47 @@ def spgemm(A: DeviceCSR, B: DeviceCSR, sample_frac: float = 0.01, seed: int = 1,
     info = {"thr": thr, "sample": rep, "nnz": plan.nnz}
     plan.destroy()
     return C, info
+
+
+def spgemm_to_host(A: DeviceCSR, B: DeviceCSR, sink, blocks: int = 8, sample_frac: float = 0.01, seed: int = 1,
+                   cm: CostModel | None = None, thr: int | None = None, inflight: int = 3):
+    """Row-blocked SpGEMM whose result streams to the host while the next block computes.
+
+    Rows are cut into `blocks` work-balanced blocks (sg_partition, Alg. 2's split); block g+1's
+    symbolic + numeric run on the current stream while block g's C crosses PCIe on a copy stream, so
+    the D2H of the result overlaps the compute. For each block, sink(g, row_begin, row_end, row_ptr,
+    col, val) is called with the copy stream as the current stream: it enqueues its device->host copies
+    (non_blocking) there; row_ptr is the block's LOCAL prefix (add the returned offset of the block).
+    At most `inflight` blocks' C stay on the device (the host waits for older copies first).
+    Returns info with the per-block C offsets."""
+    _require_cuda()
+    comp = torch.cuda.current_stream()
+    copy = torch.cuda.Stream(device=A.row_ptr.device)
+    rep = None
+    if thr is None:
+        thr, rep = sg_sample_threshold(A, B, sample_frac, seed, cm)
+    cuts, W = sg_partition(A, B, blocks)
+    done, offs = [], [0]
+    for g in range(blocks):
+        if g >= inflight:
+            done[g - inflight].synchronize()  # bounds the device memory held by in-flight blocks
+        r0, r1 = cuts[g], cuts[g + 1]
+        plan = sg_symbolic(A, B, thr, r0, r1)
+        col, val = sg_numeric(plan, A, B)
+        rp = plan.row_ptr
+        ready = torch.cuda.Event()
+        ready.record(comp)
+        copy.wait_event(ready)
+        with torch.cuda.stream(copy):
+            sink(g, r0, r1, rp, col, val)
+            ev = torch.cuda.Event()
+            ev.record(copy)
+        for t in (rp, col, val):
+            t.record_stream(copy)  # the caching allocator keeps them until the copy stream is past them
+        done.append(ev)
+        offs.append(offs[-1] + plan.nnz)
+        plan.destroy()
+        del rp, col, val
+    comp.wait_stream(copy)
+    return {"thr": thr, "sample": rep, "nnz": offs[-1], "cuts": cuts, "offsets": offs, "W": W}
+

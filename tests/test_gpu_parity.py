@@ -503,3 +503,31 @@ def test_uniform_rows_keep_the_order_preserving_path(name):
     A = gen.config(name)
     _, info, _ = _full_product(A, A, 4096)
     assert info["n_light_sorted"] <= max(1, info["n_light"] // 100)
+
+
+@pytest.mark.parametrize("blocks", [1, 3, 8])
+def test_spgemm_to_host_blocks(blocks):
+    """Row-blocked C streamed to the host while later blocks compute equals the oracle."""
+    A = gen.config("rmat12")
+    dA = _dev(A)
+    R = oracle.spgemm(A, A, with_absmag=True)
+    parts = []
+
+    def sink(g, r0, r1, drp, dcol, dval):  # runs with the copy stream current
+        parts.append((g, r0, r1, drp[:-1].to("cpu", non_blocking=True), dcol.to("cpu", non_blocking=True),
+                      dval.to("cpu", non_blocking=True)))
+
+    info = sg.spgemm_to_host(dA, dA, sink, blocks=blocks, sample_frac=0.05, seed=3)
+    torch.cuda.synchronize()
+    off = info["offsets"]
+    assert info["nnz"] == R.nnz and len(parts) == blocks
+    rp = np.zeros(A.nrows + 1, dtype=np.int64)
+    col = np.zeros(R.nnz, dtype=np.int32)
+    val = np.zeros(R.nnz, dtype=np.float64)
+    for g, r0, r1, prp, pc, pv in parts:
+        rp[r0:r1] = prp.numpy() + off[g]
+        col[off[g]:off[g + 1]] = pc.numpy()
+        val[off[g]:off[g + 1]] = pv.numpy()
+    rp[A.nrows] = off[-1]
+    assert np.array_equal(rp, R.row_ptr)
+    compare_rows(rp, col, val, R, "f64")
