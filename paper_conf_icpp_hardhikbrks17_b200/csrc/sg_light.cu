@@ -4,8 +4,8 @@
 // Numeric: order-preserving hash accumulator over that span; emission places every entry at
 // (#occupied slots before its run) + (rank inside its run) -> sorted row, no sort pass.
 //
-// Bins U <= 512: one WARP per row, several rows per block, products flattened over the warp (one k
-// per lane). Bins U >= 1024: one BLOCK per row, products flattened over the block (packed k
+// Bins U <= 512 (numeric: U <= 256): one WARP per row, several rows per block, products flattened over
+// the warp (one k per lane). Larger bins: one BLOCK per row, products flattened over the block (packed k
 // entries, one contiguous slice per warp; sg_device.cuh) — such rows often have few k with long B
 // rows, which per-warp k chunks would leave to one warp.
 #include "sg_device.cuh"
@@ -29,6 +29,12 @@ namespace sg {
     X(10, 1024, 256)           \
     X(11, 2048, 512)           \
     X(12, 4096, 1024)
+// The NUMERIC pass puts U = 512 rows on 4-warp blocks instead: a warp-per-row table of 3U slots
+// (18 KB) allowed only 12 warps per SM; one 4-warp block per row keeps 48 (C2: light numeric
+// 3.17 -> 2.59 ms). The symbolic pass (2U keys only) keeps the warp layout, which is faster there.
+#define SG_NUM_LIGHT_WARP_BINS(X) \
+    X(0, 1, 8) X(1, 2, 8) X(2, 4, 8) X(3, 8, 8) X(4, 16, 8) X(5, 32, 8) X(6, 64, 8) X(7, 128, 8) X(8, 256, 8)
+#define SG_NUM_LIGHT_BLOCK_BINS(X) X(9, 512, 128) X(10, 1024, 256) X(11, 2048, 512) X(12, 4096, 1024)
 
 // the keys-only hash set insert of the symbolic pass (any hash; order is irrelevant there)
 template <int P, int LOGP>
@@ -451,7 +457,7 @@ static cudaError_t num_light_V(int b, const Mat& A, const Mat& B, const int32_t*
                                         A, B, list, cnt, rb, span, C_rp, C_col, (VT*)C_val)));                 \
         break;                                                                                                \
     }
-        SG_LIGHT_WARP_BINS(X)
+        SG_NUM_LIGHT_WARP_BINS(X)
 #undef X
 #define X(B_, U_, NT_)                                                                                        \
     case B_: {                                                                                                \
@@ -461,11 +467,11 @@ static cudaError_t num_light_V(int b, const Mat& A, const Mat& B, const int32_t*
             cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);     \
             if (e != cudaSuccess) return e;                                                                   \
         }                                                                                                     \
-        SG_LAUNCH("k_num_light", s, (kern<<<grid_for(cnt, 1, 148 * 8), NT_, smem, s>>>(                       \
+        SG_LAUNCH("k_num_light", s, (kern<<<grid_for(cnt, 1, 148 * 16), NT_, smem, s>>>(                      \
                                         A, B, list, cnt, rb, span, C_rp, C_col, (VT*)C_val)));                 \
         break;                                                                                                \
     }
-        SG_LIGHT_BLOCK_BINS(X)
+        SG_NUM_LIGHT_BLOCK_BINS(X)
 #undef X
         default: return cudaErrorInvalidValue;
     }
