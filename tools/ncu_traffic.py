@@ -21,6 +21,8 @@ def parse(path):
     for r in csv.DictReader(lines[start:]):
         k = re.sub(r"^void ", "", r["Kernel Name"]).split("<")[0].split("(")[0].split("::")[-1]
         v = float(r["Metric Value"].replace(",", ""))
+        v *= {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12,
+              "nsecond": 1, "ns": 1, "usecond": 1e3, "us": 1e3, "msecond": 1e6, "ms": 1e6}.get(r.get("Metric Unit", ""), 1)
         per[(int(r["ID"]), k)][r["Metric Name"]] = v
     return per
 
