@@ -555,7 +555,8 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 bm4[2 * tid + 1] = make_uint4(0, 0, 0, 0);
             }
             mark(10);
-            __syncthreads();
+            // no barrier here: the next range's first reads of the cleared bitmap / accumulator and its
+            // rewrite of the packed chunk arrays all come after chunk_compact's barriers
             mark(6);
         }
     }
