@@ -146,6 +146,90 @@ __global__ void __launch_bounds__(DW_T, DW_OCC) k_num_dense(
             }
         }
         mark(1);
+#ifndef SG_DW_PIPE
+#define SG_DW_PIPE 1
+#endif
+        if (SG_DW_PIPE && single) {
+            // Single-chunk rows, software-pipelined: window t+1's segments are found while window t is
+            // emitted, and ONE block scan (block_scan2) places both window t's output entries and window
+            // t+1's packed chunk entries: 3 barriers per window instead of 4.
+            auto seg_next = [&](int tw, int& len, int& beg) {  // segment of this thread's k in window tw
+                len = 0;
+                beg = cur;
+                if (tid < na && tw < tb) {
+                    const int64_t whi = min(p, (int64_t)(tw + 1) * WD);
+                    int end;
+                    if (lid >= 0) {
+                        end = q0 + (int)tpv;
+                        if (tw + 1 < tb) tpv = __ldg(tp + (int64_t)lid * (T + 1) + min((tw + 2) * DW_TILES, T));
+                    } else if constexpr (kShortCache) {
+                        int n = 0;
+                        #pragma unroll
+                        for (int q = 0; q < LONG_ROW; ++q) n += S.sc[q][tid] < whi;
+                        end = q0 + n;
+                    } else {
+                        end = seg_end(B, cur, e1r, q0, false, 0u, whi);
+                    }
+                    len = end - cur;
+                    cur = end;
+                }
+            };
+            int nk, any;
+            {
+                int len, beg;
+                seg_next(ta, len, beg);
+                any = chunk_compact<DW_T, int32_t>(len, beg, a, S.s_beg, S.s_off, S.s_a, &nk, S.wsll);
+            }
+            for (int t = ta; t < tb; ++t) {
+                const int64_t lo = (int64_t)t * WD;
+                const uint32_t vb = opaque_u32(a_vals - 8u * (uint32_t)lo);
+                const uint32_t bb = opaque_u32(a_bm - 4u * ((uint32_t)lo >> 5));
+                if (any > 0)
+                    warp_slice<DW_T, true, VT, int32_t>(S.s_beg, S.s_off, S.s_a, nk, any, B, [&](int32_t c, double v) {
+                        if (c < 0) return;
+                        if (atom_add_f64_s(vb + 8u * (uint32_t)c, v) == 0.0)
+                            red_or_s(bb + 4u * ((uint32_t)c >> 5), 1u << (c & 31));
+                    });
+                __syncthreads();  // window t accumulated; the packed chunk arrays are free
+                uint32_t hw;
+                {
+                    const int b0 = CPT * tid, w0 = b0 >> 5, shv = b0 & 31;
+                    const unsigned long long two = ((unsigned long long)S.bm[w0 + 1] << 32) | S.bm[w0];
+                    hw = (uint32_t)(two >> shv) & (CPT == 32 ? 0xFFFFFFFFu : ((1u << CPT) - 1u));
+                }
+                int len, beg;
+                seg_next(t + 1, len, beg);
+                int ex, wtot;
+                long long exc, totc;
+                block_scan2<DW_T>(__popc(hw), ((long long)len << 16) | (len > 0 ? 1 : 0), &ex, &wtot, &exc, &totc, S.ws,
+                                  S.wsll);
+                for (int q = tid; q < DW_WORDS; q += DW_T) S.bm[q] = 0u;  // every bitmap read preceded the scan
+                {
+                    uint32_t m = hw;
+                    int64_t at = pos + ex;
+                    const int ebase = tid * CPT;
+                    while (m) {
+                        const int e = ebase + __ffs(m) - 1;
+                        m &= m - 1u;
+                        st_out(C_col + at, (int32_t)(lo + e));
+                        st_out(C_val + at, (VT)S.vals[e]);
+                        S.vals[e] = 0.0;
+                        ++at;
+                    }
+                }
+                pos += wtot;
+                if (len > 0) {
+                    const int ci = (int)(exc & 0xFFFF);
+                    S.s_beg[ci] = beg;
+                    S.s_off[ci] = (int)(exc >> 16);
+                    S.s_a[ci] = a;
+                }
+                nk = (int)(totc & 0xFFFF);
+                any = (int)(totc >> 16);
+                __syncthreads();  // chunk arrays of window t+1 published; clears ordered before its products
+            }
+            continue;
+        }
         for (int t = ta; t < tb; ++t) {
             const int tn = t + 1;  // next window
             const int64_t lo = (int64_t)t * WD, hi = min(p, lo + WD);

@@ -282,6 +282,26 @@ __device__ __forceinline__ T block_scan1(T v, T* total, T* ws) {
 template <int NT>
 __device__ __forceinline__ int block_scan(int v, int* total, int* ws) { return block_scan1<NT, int>(v, total, ws); }
 
+// Two exclusive scans (an int and a long long per thread) sharing ONE barrier (same ws rule as
+// block_scan1 for both ws arrays).
+template <int NT>
+__device__ __forceinline__ void block_scan2(int v1, long long v2, int* ex1, int* tot1, long long* ex2, long long* tot2,
+                                            int* ws1, long long* ws2) {
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int i1 = warp_incl_scan(v1);
+    const long long i2 = warp_incl_scan(v2);
+    if (lane == 31) { ws1[wid] = i1; ws2[wid] = i2; }
+    __syncthreads();
+    const int x1 = lane < NT / 32 ? ws1[lane] : 0;
+    const long long x2 = lane < NT / 32 ? ws2[lane] : 0LL;
+    const int y1 = warp_incl_scan(x1);
+    const long long y2 = warp_incl_scan(x2);
+    *tot1 = __shfl_sync(FULL, y1, 31);
+    *tot2 = __shfl_sync(FULL, y2, 31);
+    *ex1 = __shfl_sync(FULL, y1 - x1, wid) + i1 - v1;
+    *ex2 = __shfl_sync(FULL, y2 - x2, wid) + i2 - v2;
+}
+
 // largest i in [0, nk) with off[i] <= j (that entry has len > 0)
 __device__ __forceinline__ int find_k(const int* off, int nk, int j) {
     int lo = 0, hi = nk - 1;
