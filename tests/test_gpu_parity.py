@@ -531,3 +531,23 @@ def test_spgemm_to_host_blocks(blocks):
     rp[A.nrows] = off[-1]
     assert np.array_equal(rp, R.row_ptr)
     compare_rows(rp, col, val, R, "f64")
+
+
+def test_spgemm_to_host_more_blocks_than_rows_and_empty():
+    """Degenerate row blocking: more blocks than rows (empty blocks), and an empty matrix."""
+    A = gen.config("C1")
+    small = gen.CSR(3, A.ncols, A.row_ptr[:4].copy(), A.col[:A.row_ptr[3]].copy(), A.val[:A.row_ptr[3]].copy(), "3rows")
+    dS, dA = _dev(small), _dev(A)
+    got = []
+    info = sg.spgemm_to_host(dS, dA, lambda g, r0, r1, rp, c, v: got.append((r0, r1, int(c.numel()))), blocks=8,
+                             thr=16)
+    torch.cuda.synchronize()
+    R = oracle.spgemm(small, A)
+    assert info["nnz"] == R.nnz and sum(x[2] for x in got) == R.nnz and len(got) == 8
+    E = gen.CSR(0, A.ncols, np.zeros(1, np.int64), np.zeros(0, np.int32), np.zeros(0), "empty")
+    dE = _dev(E)
+    info = sg.spgemm_to_host(dE, dA, lambda *a: None, blocks=4, thr=16)
+    assert info["nnz"] == 0
+    cuts, tot = sg.sg_partition_cost(dE, dA, 3, 16, [0, 0, 0, 0])
+    assert cuts == [0, 0, 0, 0] and tot == 0
+
