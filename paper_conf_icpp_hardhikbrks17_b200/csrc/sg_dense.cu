@@ -223,6 +223,7 @@ __global__ void __launch_bounds__(DW_T, DW_OCC) k_num_dense(
                     S.s_beg[ci] = beg;
                     S.s_off[ci] = (int)(exc >> 16);
                     S.s_a[ci] = a;
+                    mark_slice_starts<DW_T>(ci, (int)(exc >> 16), len, (int)(totc >> 16));
                 }
                 nk = (int)(totc & 0xFFFF);
                 any = (int)(totc >> 16);

@@ -317,6 +317,22 @@ __device__ __forceinline__ long long block_scan_ll(long long v, long long* total
     return block_scan1<NT, long long>(v, total, ws);
 }
 
+// First packed entry of every warp's product slice (see SliceCursor): written by the entry whose
+// product range contains the slice start, so no warp binary-searches the packed offsets.
+__shared__ int sg_wstart[32];
+
+// slice length per warp for tot products over NW warps (a multiple of 32; SliceCursor uses the same)
+__device__ __forceinline__ int slice_per(int tot, int NW) { return (((tot + NW - 1) / NW) + 31) & ~31; }
+
+// entry ci holds products [o, o + len) of a packing with tot products: mark the slices starting inside
+template <int NT>
+__device__ __forceinline__ void mark_slice_starts(int ci, int o, int len, int tot) {
+    constexpr int NW = NT / 32;
+    const int per = slice_per(tot, NW);
+    if (len <= 0 || per <= 0) return;
+    for (int w = (o + per - 1) / per; w < NW && w * per < o + len; ++w) sg_wstart[w] = ci;
+}
+
 // One chunk of k entries (one per thread): pack the entries with len > 0, in order, into
 // s_beg / s_off (exclusive prefix of len) / s_a; returns the chunk's product count, *nk = packed.
 template <int NT, class BEG>
@@ -329,6 +345,7 @@ __device__ __forceinline__ int chunk_compact(int len, BEG beg, double a, BEG* s_
         s_beg[ci] = beg;
         s_off[ci] = (int)(ex >> 16);
         if (s_a) s_a[ci] = a;
+        mark_slice_starts<NT>(ci, (int)(ex >> 16), len, (int)(tot >> 16));
     }
     *nk = (int)(tot & 0xFFFF);
     __syncthreads();
@@ -363,10 +380,10 @@ struct SliceCursor {
         d_off = (uint32_t)((const char*)so - (const char*)sb);
         d_a = sa ? (uint32_t)((const char*)sa - (const char*)sb) : 0u;
         const int wid = threadIdx.x >> 5;
-        const int per = (((tot + NW - 1) / NW) + 31) & ~31;
+        const int per = slice_per(tot, NW);
         j_lo = wid * per;
         j_hi = min(tot, j_lo + per);
-        i0 = j_lo < j_hi ? find_k(so, nk, j_lo) : 0;
+        i0 = j_lo < j_hi ? sg_wstart[wid] : 0;  // written by the packing (chunk_compact)
     }
     // batch [j0, j0 + 32): lane's (column, a_ik * b_kj), c = -1 beyond the slice
     __device__ __forceinline__ void fetch(const Mat& B, int j0, int& c, double& v) {
