@@ -28,6 +28,7 @@ struct sg_plan {
     int32_t* nranges = nullptr;
     RangeRec* ranges = nullptr;
     int64_t nslots = 0, amax = 0;
+    int64_t nbig = 0;               // heavy rows [0, nbig) with w >= 2^20 (1024-thread symbolic kernel)
     int64_t ndw = 0;                // heavy[0, ndw): dense-window rows (w >= 2^dw_log2), sg_dense.cu
     int32_t* dtc = nullptr;         // their per-tile output counts (ndw x T), from the symbolic pass
     int4* ditems = nullptr;         // dense-window work items (row, window range)
@@ -212,7 +213,7 @@ sg_status row_stats(const Mat& A, const Mat& B, const int64_t* rows, int64_t nr,
     unsigned long long* counter = (unsigned long long*)sc.get(sizeof(unsigned long long));
     if (!counter) return SG_ERR_OOM;
     CK(launch_sym_heavy(A, B, lists + off[BIN_HEAVY], cnt[BIN_HEAVY], rows, 0, rs.u, nullptr, nullptr, nullptr,
-                        0, nullptr, counter, s));
+                        0, nullptr, nullptr, nullptr, 0, counter, s, cnt[BIN_HEAVY]));
     return SG_OK;
 }
 
@@ -594,6 +595,9 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
         // heavy order bucket b = 62 - floor(log2 w) (ascending = heaviest first): w >= 2^m <=> b <= 62 - m
         pl->ndw = 0;
         for (int hb2 = 0; hb2 <= 62 - pl->dw_log2 && hb2 < 64; ++hb2) pl->ndw += hh[hb2];
+        // rows with w >= 2^20 take the 1024-thread symbolic kernel (one such row must not be a tail)
+        pl->nbig = 0;
+        for (int hb2 = 0; hb2 <= 62 - 20; ++hb2) pl->nbig += hh[hb2];
         if (pl->ndw > 0) {
             pl->dtc = (int32_t*)palloc(pl, sizeof(int32_t) * (size_t)pl->ndw * (size_t)pl->T);
             pl->ditems = (int4*)palloc(pl, sizeof(int4) * (size_t)dense_items_bound(pl->ndw, pl->p));
@@ -619,7 +623,8 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
         CKF(launch_sym_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], nullptr, row_begin, pl->u, pl->span,
                              (unsigned long long*)(pl->dbin + 2 * NBINS + 1), s));
     CKF(launch_sym_heavy(a, b, pl->heavy, pl->nheavy, nullptr, row_begin, pl->u, pl->range_off, pl->ranges,
-                         pl->nranges, pl->ndw, pl->dtc, pl->counter, s));
+                         pl->nranges, pl->ndw, pl->dtc, pl->long_id, pl->nlong > 0 ? pl->tp : nullptr, pl->T,
+                         pl->counter, s, pl->nbig));
     CKF(scan_exclusive(pl->u, C_row_ptr, nr, stmp, s));
     CKF(cudaMemcpyAsync(&pl->nnz_c, C_row_ptr + nr, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     CKF(cudaMemcpyAsync(&pl->nskew, pl->dbin + 2 * NBINS + 1, sizeof(int64_t), cudaMemcpyDeviceToHost, s));

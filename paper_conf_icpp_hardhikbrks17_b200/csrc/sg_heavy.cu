@@ -1,9 +1,10 @@
 // sg_heavy.cu — the HEAVY path (w_i > thr, "more than t"): one CTA per heavy row
-// (symbolic: 1024 threads, one CTA per SM; numeric: 512 threads, two CTAs per SM so that one CTA's
-// barriers and serial phases overlap the other's products), rows taken heaviest-first from a
-// dynamic counter.
+// (symbolic: 256 threads, six CTAs per SM, 2^18-column bitmap windows; numeric: 512 threads, two CTAs
+// per SM — several CTAs per SM so that one CTA's barriers and serial phases overlap the others'
+// products), rows taken heaviest-first from a dynamic counter.
 //
-// Symbolic: the row's products set bits of a shared-memory bitmap over a 2^20-column window;
+// Symbolic: the row's products set bits of a shared-memory bitmap over a WIN-column window (a window's
+// segment of each B row from the tile pointers);
 // per-8192-column-tile popcounts give u_i and a plan of column RANGES, each holding at most
 // RCAP = 8192 output entries and spanning at most RW_TILES tiles (the numeric accumulator).
 //
@@ -23,7 +24,7 @@ namespace sg {
 #ifndef SG_INREG
 #define SG_INREG 1
 #endif
-constexpr int SYM_T = HEAVY_THREADS;  // symbolic: one CTA of 1024 threads per SM (128 KB bitmap window)
+constexpr int SYM_T = HEAVY_THREADS;  // symbolic threads per CTA (SYM_OCC CTAs per SM, WIN/8 bytes of bitmap each)
 #ifndef SG_NUM_T
 #define SG_NUM_T 512
 #endif
@@ -158,27 +159,30 @@ cudaError_t launch_range_bounds(const int32_t* heavy, int64_t nh, const int64_t*
 // ------------------------------------------------------------------------------------------------
 // a6 heavy symbolic
 // ------------------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(HEAVY_THREADS, 1) k_sym_heavy(Mat A, Mat B, const int32_t* __restrict__ list,
+template <int ST, int SOCC, int SWIN>
+__global__ void __launch_bounds__(ST, SOCC) k_sym_heavy(Mat A, Mat B, const int32_t* __restrict__ list, int64_t j0,
                                                                  int64_t cnt, const int64_t* __restrict__ rowmap,
                                                                  int64_t rb, int64_t* __restrict__ u,
                                                                  const int64_t* __restrict__ range_off,
                                                                  RangeRec* __restrict__ ranges,
                                                                  int32_t* __restrict__ nranges, int64_t ndw,
-                                                                 int32_t* __restrict__ dtc, unsigned long long* counter) {
-    extern __shared__ uint32_t bm[];  // WIN/32 words
-    __shared__ int64_t s_beg[KCS];
-    __shared__ int s_off[KCS];
-    __shared__ int tcnt[WIN / TW];
-    __shared__ int Ps[WIN / TW];
-    __shared__ unsigned char st[WIN / TW];
+                                                                 int32_t* __restrict__ dtc, const int32_t* __restrict__ long_id,
+                                                                 const uint32_t* __restrict__ tp, int T,
+                                                                 unsigned long long* counter) {
+    extern __shared__ uint32_t bm[];  // SWIN/32 words
+    __shared__ int64_t s_beg[ST];
+    __shared__ int s_off[ST];
+    __shared__ int tcnt[SWIN / TW];
+    __shared__ int Ps[SWIN / TW];
+    __shared__ unsigned char st[SWIN / TW];
     __shared__ long long wsll[33];
     __shared__ long long s_j;
     __shared__ int s_nr, s_u;
-    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5, nwarps = HEAVY_THREADS / 32;
+    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5, nwarps = ST / 32;
     const int64_t p = B.ncols;
-    const int64_t nwin = (p + WIN - 1) / WIN;
+    const int64_t nwin = (p + SWIN - 1) / SWIN;
     while (true) {
-        if (tid == 0) s_j = (long long)atomicAdd(counter, 1ull);
+        if (tid == 0) s_j = j0 + (long long)atomicAdd(counter, 1ull);
         __syncthreads();
         const int64_t j = s_j;
         __syncthreads();
@@ -188,10 +192,10 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_sym_heavy(Mat A, Mat B, co
         const int64_t s0 = __ldg(A.rp + row), s1 = __ldg(A.rp + row + 1);
         int utot = 0, nr = 0;
         for (int64_t win = 0; win < nwin; ++win) {
-            const int64_t wlo = win * WIN, whi = min(p, wlo + WIN);
+            const int64_t wlo = win * SWIN, whi = min(p, wlo + SWIN);
             const int nwords = (int)((whi - wlo + 31) / 32);
-            for (int q = tid; q < nwords; q += HEAVY_THREADS) bm[q] = 0u;
-            for (int64_t c0 = s0; c0 < s1; c0 += KCS) {
+            for (int q = tid; q < nwords; q += ST) bm[q] = 0u;
+            for (int64_t c0 = s0; c0 < s1; c0 += ST) {
                 const int64_t i = c0 + tid;
                 int len = 0;
                 int64_t beg = 0;
@@ -199,16 +203,34 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_sym_heavy(Mat A, Mat B, co
                     const int k = __ldg(A.col + i);
                     int64_t q0 = __ldg(B.rp + k), q1 = __ldg(B.rp + k + 1);
                     if (nwin > 1) {
-                        q0 = lower_bound_col(B.col, q0, q1, wlo);
-                        q1 = lower_bound_col(B.col, q0, q1, whi);
+                        if (tp && q1 - q0 > LONG_ROW) {  // the window's segment from the B tile pointers
+                            const uint32_t* tr = tp + (int64_t)__ldg(long_id + k) * (T + 1);
+                            const int64_t b0 = q0;
+                            q0 = b0 + __ldg(tr + wlo / TW);
+                            q1 = b0 + __ldg(tr + (whi == p ? T : (int)(whi / TW)));
+                        } else if (tp) {  // short row: count its entries below the window bounds
+                            int n0 = 0, n1 = 0;
+                            #pragma unroll
+                            for (int q = 0; q < LONG_ROW; ++q)
+                                if (q0 + q < q1) {
+                                    const int c = __ldg(B.col + q0 + q);
+                                    n0 += c < wlo;
+                                    n1 += c < whi;
+                                }
+                            q1 = q0 + n1;
+                            q0 = q0 + n0;
+                        } else {
+                            q0 = lower_bound_col(B.col, q0, q1, wlo);
+                            q1 = lower_bound_col(B.col, q0, q1, whi);
+                        }
                     }
                     beg = q0;
                     len = (int)(q1 - q0);
                 }
                 int nk;
-                const int tot = chunk_compact<SYM_T, int64_t>(len, beg, 0.0, s_beg, s_off, nullptr, &nk, wsll);
+                const int tot = chunk_compact<ST, int64_t>(len, beg, 0.0, s_beg, s_off, nullptr, &nk, wsll);
                 const uint32_t bb = opaque_u32(smem_addr(bm) - 4u * ((uint32_t)wlo >> 5));  // wlo: multiple of 32
-                warp_slice<SYM_T, false, double, int64_t>(s_beg, s_off, nullptr, nk, tot, B, [&](int32_t c, double) {
+                warp_slice<ST, false, double, int64_t>(s_beg, s_off, nullptr, nk, tot, B, [&](int32_t c, double) {
                     if (c >= 0) red_or_s(bb + 4u * ((uint32_t)c >> 5), 1u << (c & 31));
                 });
                 __syncthreads();
@@ -246,7 +268,7 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_sym_heavy(Mat A, Mat B, co
                 for (int q = 0; q < 4; ++q) {
                     const int t = 4 * lane + q;
                     pre += c4[q];
-                    key[q] = ((pre + RHALF - 1) / RHALF - 1) * (WIN / TW / RW_TILES) + t / RW_TILES;
+                    key[q] = ((pre + RHALF - 1) / RHALF - 1) * (SWIN / TW / RW_TILES) + t / RW_TILES;
                     if (t < nt) Ps[t] = pre;
                 }
                 const int prevkey = __shfl_up_sync(FULL, key[3], 1);
@@ -295,18 +317,38 @@ __global__ void __launch_bounds__(HEAVY_THREADS, 1) k_sym_heavy(Mat A, Mat B, co
     }
 }
 
-cudaError_t launch_sym_heavy(const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, const int64_t* rowmap,
-                             int64_t rb, int64_t* u, const int64_t* range_off, RangeRec* ranges, int32_t* nranges,
-                             int64_t ndw, int32_t* dtc, unsigned long long* counter, cudaStream_t s) {
-    if (cnt <= 0) return cudaSuccess;
-    const int smem = (WIN / 32) * 4;
-    cudaError_t e = cudaFuncSetAttribute(k_sym_heavy, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+template <int ST, int SOCC, int SWIN>
+static cudaError_t sym_heavy_part(const Mat& A, const Mat& B, const int32_t* list, int64_t j0, int64_t cnt,
+                                  const int64_t* rowmap, int64_t rb, int64_t* u, const int64_t* range_off,
+                                  RangeRec* ranges, int32_t* nranges, int64_t ndw, int32_t* dtc, const int32_t* long_id,
+                                  const uint32_t* tp, int T, unsigned long long* counter, cudaStream_t s) {
+    if (cnt - j0 <= 0) return cudaSuccess;
+    const int smem = (SWIN / 32) * 4;
+    cudaError_t e = cudaFuncSetAttribute(k_sym_heavy<ST, SOCC, SWIN>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
     if ((e = cudaMemsetAsync(counter, 0, sizeof(unsigned long long), s)) != cudaSuccess) return e;
-    const int grid = (int)(cnt < 148 ? cnt : 148);
-    SG_LAUNCH("k_sym_heavy", s, (k_sym_heavy<<<grid, HEAVY_THREADS, smem, s>>>(A, B, list, cnt, rowmap, rb, u, range_off,
-                                                                                ranges, nranges, ndw, dtc, counter)));
+    const int64_t n = cnt - j0;
+    const int grid = (int)(n < 148 * SOCC ? n : 148 * SOCC);
+    SG_LAUNCH("k_sym_heavy", s, (k_sym_heavy<ST, SOCC, SWIN><<<grid, ST, smem, s>>>(A, B, list, j0, cnt, rowmap, rb, u,
+                                                                                     range_off, ranges, nranges, ndw, dtc,
+                                                                                     long_id, tp, T, counter)));
     return cudaGetLastError();
+}
+
+// Heavy rows [0, nbig) of the heaviest-first list (the ones whose single-CTA time could be a tail)
+// run on 1024-thread CTAs over 2^20-column windows; the rest on SYM_OCC smaller CTAs per SM over
+// WIN-column windows (segments from the tile pointers), whose barriers overlap each other.
+cudaError_t launch_sym_heavy(const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, const int64_t* rowmap,
+                             int64_t rb, int64_t* u, const int64_t* range_off, RangeRec* ranges, int32_t* nranges,
+                             int64_t ndw, int32_t* dtc, const int32_t* long_id, const uint32_t* tp, int T,
+                             unsigned long long* counter, cudaStream_t s, int64_t nbig) {
+    if (cnt <= 0) return cudaSuccess;
+    if (nbig > cnt) nbig = cnt;
+    cudaError_t e = sym_heavy_part<1024, 1, (1 << 20)>(A, B, list, 0, nbig, rowmap, rb, u, range_off, ranges, nranges, ndw,
+                                                        dtc, long_id, tp, T, counter, s);
+    if (e != cudaSuccess) return e;
+    return sym_heavy_part<HEAVY_THREADS, SYM_OCC, WIN>(A, B, list, nbig, cnt, rowmap, rb, u, range_off, ranges, nranges,
+                                                       ndw, dtc, long_id, tp, T, counter, s);
 }
 
 // ------------------------------------------------------------------------------------------------
@@ -314,7 +356,7 @@ cudaError_t launch_sym_heavy(const Mat& A, const Mat& B, const int32_t* list, in
 // ------------------------------------------------------------------------------------------------
 struct HeavySmem {
     uint32_t bm[RW_WORDS];       // 32 KB  range bitmap
-    double vals[RCAP + 2];       // 128 KB compact accumulator: rank r at vals[r + sh], sh = C offset parity
+    double vals[RCAP + 2];       // 64 KB compact accumulator: rank r at vals[r + sh], sh = C offset parity
     uint16_t pref[RW_WORDS];     // 16 KB  rank prefix per bitmap word
     int32_t s_beg[KC];           // packed chunk entries: segment begin (B position)
     int32_t s_off[KC];           //                       exclusive prefix of segment lengths

@@ -26,8 +26,18 @@ constexpr int NBINS = 15;
 // ---- heavy path geometry ---------------------------------------------------
 constexpr int TW = 8192;          // column tile width of the heavy path (tile = unit of range planning)
 constexpr int LONG_ROW = 8;       // B rows longer than this get per-tile pointers
-constexpr int WIN = 1 << 20;      // heavy symbolic bitmap window (columns); 128 KB of smem
-constexpr int HEAVY_THREADS = 1024;
+#ifndef SG_SYM_WIN_LOG2
+#define SG_SYM_WIN_LOG2 18
+#endif
+#ifndef SG_SYM_T
+#define SG_SYM_T 256
+#endif
+#ifndef SG_SYM_OCC
+#define SG_SYM_OCC 6
+#endif
+constexpr int WIN = 1 << SG_SYM_WIN_LOG2;  // heavy symbolic bitmap window (columns); WIN/8 bytes of smem
+constexpr int HEAVY_THREADS = SG_SYM_T;    // heavy symbolic threads per CTA
+constexpr int SYM_OCC = SG_SYM_OCC;        // heavy symbolic CTAs per SM
 
 constexpr int32_t EMPTY_KEY = -1;
 constexpr uint64_t TAG_SAMPLE = 0x53414d504c450001ULL;  // DESIGN.md R4 (stream tag of the row sampler)
@@ -83,8 +93,9 @@ cudaError_t launch_range_bounds(const int32_t* heavy_list, int64_t nheavy, const
                                 int64_t dw_min_w, int64_t* bounds, cudaStream_t s);
 cudaError_t launch_sym_heavy(const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, const int64_t* rowmap,
                              int64_t rb, int64_t* u, const int64_t* range_off, RangeRec* ranges, int32_t* nranges,
-                             int64_t ndw, int32_t* dtc /*ndw x T tile counts, nullable*/, unsigned long long* counter,
-                             cudaStream_t s);
+                             int64_t ndw, int32_t* dtc /*ndw x T tile counts, nullable*/, const int32_t* long_id /*nullable*/,
+                             const uint32_t* tp /*nullable: binary search*/, int T, unsigned long long* counter,
+                             cudaStream_t s, int64_t nbig /*rows [0, nbig) on the 1024-thread kernel*/);
 cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, int64_t h0, int64_t nheavy, int64_t rb,
                              const int64_t* range_off, const int32_t* nranges, const RangeRec* ranges,
                              const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,

@@ -41,7 +41,7 @@ def main():
         H = gen.config(a.config, seed=a.seed)
     A = sg.DeviceCSR.from_host(H)
     cm = sg.sg_default_cost_model()
-    pcm = cm
+    pcm = None  # sg_partition_cost's default: the partition model fitted to measured shard times
     if a.cm_json:
         pcm = sg.sg_default_cost_model()
         for k, v in json.load(open(a.cm_json))["model"].items():
