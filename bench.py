@@ -371,9 +371,11 @@ def main():
         for k, (nprod, prim) in ops.items():
             if k in bk and prim in mb:
                 cnt, tot = bk[k]
-                rate = nprod / (tot / cnt / 1e3) / 1e9
+                # per STEP (a kernel may launch several times a step: the symbolic runs as a 1024-thread
+                # part for the rows with w >= 2^20 and a small-CTA part, plus the sampler's pass)
+                rate = nprod / (tot / args.steps / 1e3) / 1e9
                 roof_smem[k] = {"bound": "smem_atomic", "achieved": rate, "peak": mb[prim], "unit": "Gop/s",
-                                "frac": rate / mb[prim], "op": prim, "ops_per_launch": nprod}
+                                "frac": rate / mb[prim], "op": prim, "ops_per_step": nprod, "launches_per_step": cnt / args.steps}
     step_alg_bytes = 2 * csr_bytes(H.nrows, H.nnz, vbytes) + csr_bytes(H.nrows, nnzC_total, vbytes)
     compulsory = {"bytes_per_step": step_alg_bytes,
                   "GBps": step_alg_bytes / (ms_per_step / 1e3) / 1e9,
