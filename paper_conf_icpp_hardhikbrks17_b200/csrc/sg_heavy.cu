@@ -24,7 +24,6 @@ namespace sg {
 #ifndef SG_INREG
 #define SG_INREG 1
 #endif
-constexpr int SYM_T = HEAVY_THREADS;  // symbolic threads per CTA (SYM_OCC CTAs per SM, WIN/8 bytes of bitmap each)
 #ifndef SG_NUM_T
 #define SG_NUM_T 512
 #endif
@@ -37,7 +36,6 @@ constexpr int SYM_T = HEAVY_THREADS;  // symbolic threads per CTA (SYM_OCC CTAs 
 constexpr int NUM_T = SG_NUM_T;       // numeric: threads per CTA
 constexpr int NUM_OCC = SG_NUM_OCC;   // numeric CTAs per SM (smem-bound)
 constexpr int KC = NUM_T;             // numeric k entries per chunk: one per thread
-constexpr int KCS = SYM_T;            // symbolic k entries per chunk
 constexpr int RW_TILES = NUM_T / 32;  // max tiles per numeric range (16 -> 128K columns, 16 KB bitmap)
 constexpr int RW_WORDS = RW_TILES * TW / 32;   // = 256 words per warp in the rank prefix
 constexpr int RCAP = SG_RCAP;         // max entries per numeric range (fp64 accumulator 64 KB)
