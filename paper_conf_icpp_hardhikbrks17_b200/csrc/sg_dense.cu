@@ -400,13 +400,14 @@ int dense_kc() { return DKC; }
 
 namespace sg {
 // Rows with w >= 2^m take the dense-window kernel. Its fixed cost grows with the number of windows
-// (p / WD) while its saving over the rank kernel grows with w, so m tracks log2 p: 2^18 at p = 2^20 (measured best of 2^16..2^20 on R-MAT 20).
+// (p / WD) while its saving over the rank kernel grows with w, so m tracks log2 p: 2^19 at p = 2^20
+// (C3: 283.5 vs 284.6 ms/step at 2^18), 2^17 at p = 2^18 (R-MAT 18: 35.2 vs 35.6 ms).
 int dense_window_log2(int64_t p) {
     const char* e = getenv("SG_DW_LOG2");
     if (e && *e) return atoi(e);
     int lp = 0;
     while (lp < 62 && ((int64_t)1 << lp) < p) ++lp;
-    const int m = lp - 2;
+    const int m = lp - 1;
     return m < 4 ? 4 : m;
 }
 }  // namespace sg
