@@ -215,3 +215,70 @@ def test_partition_concatenation_equals_whole():
         vals.append(R.val)
     assert np.array_equal(np.concatenate(cols), whole.col)
     assert np.array_equal(np.concatenate(vals), whole.val)
+
+
+# ---- the branches production uses: capu > 0 (non-exact u/capu), rho_L > 0 ----------------------
+
+GOLD2 = os.path.join(os.path.dirname(__file__), "golden", "o4_capu_rho_example.json")
+
+
+def test_worked_example_capu_and_rho_branches():
+    """Hand-derived fixture (tests/golden/o4_capu_rho_example.json): R(u) = max(1, ceil(u/capu))
+    at non-exact u/capu, and c_L's rho_L*u term.
+    A floor instead of the ceil, or rho_L*(u+1), changes c_H / c_L of some row here."""
+    g = json.load(open(GOLD2))
+    cm = _cm(**g["cost_model"])
+    rows = np.array(g["rows"], dtype=np.int64)
+    w, a, u = rows[:, 0], rows[:, 1], rows[:, 2]
+    for r in range(1, len(w)):
+        assert oracle.cost_L(cm, w[r], a[r], u[r]) == g["c_L"][r]
+        assert oracle.cost_H(cm, w[r], a[r], u[r]) == g["c_H"][r]
+    for t, Jt in g["J"].items():
+        assert oracle.J(cm, w, a, u, int(t)) == Jt
+    thr, Jmin = oracle.threshold(cm, w, a, u)
+    assert thr == g["thr_star"] and Jmin == g["J"][str(thr)]
+    S = np.array(g["sample_rows"])
+    for t, Jt in g["J_sample"].items():
+        assert oracle.J(cm, w[S], a[S], u[S], int(t)) == Jt
+    assert oracle.threshold(cm, w[S], a[S], u[S])[0] == g["thr_s"]
+
+
+def test_worked_example_cost_split_nonexact_uh():
+    """uh_i = min(w_i, ceil(w_i U_c / W_c)) at non-exact quotients (reading R19), capu > 0 and
+    rho_L > 0 inside the per-row costs; closest-prefix cuts on their prefix."""
+    g = json.load(open(GOLD2))
+    cm = _cm(**g["cost_model"])
+    sp = g["split"]
+    wa = np.array(sp["rows_wa"], dtype=np.int64)
+    w, a = wa[:, 0], wa[:, 1]
+    costs = [oracle.row_cost(cm, sp["thr"], sp["comp"], int(x), int(y)) for x, y in zip(w, a)]
+    assert costs == sp["cost"]
+    for (wi, ai), uh, c in zip(sp["rows_wa"], sp["uh"], sp["cost"]):
+        if wi == 0:
+            continue
+        ref = oracle.cost_L(cm, wi, ai, uh) if wi <= sp["thr"] else oracle.cost_H(cm, wi, ai, uh)
+        assert ref == c
+    for G, cuts in sp["cuts"].items():
+        got, tot = oracle.partition_cost(cm, sp["thr"], sp["comp"], w, a, int(G))
+        assert got.tolist() == cuts and tot == sp["total"]
+
+
+def test_cost_H_tile_count_closed_form():
+    """R(u) = max(1, ceil(u/capu)) for capu > 0 at every u in [0, 5*capu]: with every other
+    constant 0 and tau_H = a = 1, c_H(u) IS R(u) (closed form, checked against integer ceil)."""
+    for capu in (1, 3, 16, 100):
+        cm = _cm(tau_H=1, tiles_fixed=7, capu=capu, cap_L=100)
+        for uu in range(0, 5 * capu + 2):
+            assert oracle.cost_H(cm, 0, 1, uu) == max(1, -(-uu // capu))
+    cm = _cm(tau_H=1, tiles_fixed=7, capu=0, cap_L=100)
+    assert oracle.cost_H(cm, 0, 1, 12345) == 7
+
+
+def test_cost_L_rho_term_closed_form():
+    """With only rho_L = 1: c_L = u exactly; with only sigma_L = 1: u * ceil(log2 max(u, 2))."""
+    cm = _cm(rho_L=1, cap_L=100)
+    for uu in (0, 1, 2, 3, 17, 1000):
+        assert oracle.cost_L(cm, 5, 1, uu) == uu
+    cm = _cm(sigma_L=1, cap_L=100)
+    for uu, lg in ((0, 1), (1, 1), (2, 1), (3, 2), (4, 2), (5, 3), (1024, 10), (1025, 11)):
+        assert oracle.cost_L(cm, 5, 1, uu) == uu * lg
