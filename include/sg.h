@@ -39,12 +39,13 @@ typedef enum {
     SG_ERR_INVALID_ARG = 1,   /* null pointer, sample_frac outside (0,1], thr outside [0,cap_L], bad row range */
     SG_ERR_SHAPE = 2,         /* A.ncols != B.nrows, or a buffer shape mismatch */
     SG_ERR_DTYPE = 3,         /* A and B value dtypes differ, or unknown dtype */
-    SG_ERR_NOT_CANONICAL = 4, /* only with SG_VALIDATE=1 in the environment: unsorted/duplicate/out-of-range columns */
+    SG_ERR_NOT_CANONICAL = 4, /* only with SG_OPT_VALIDATE = 1: unsorted/duplicate/out-of-range columns, bad row_ptr */
     SG_ERR_EMPTY_SAMPLE = 5,  /* the sample holds no non-empty row */
     SG_ERR_OOM = 6,           /* device workspace allocation failed */
     SG_ERR_CUDA = 7,          /* a CUDA runtime error (or a poisoned plan) */
     SG_ERR_NCCL = 8,          /* an NCCL error in sg_gather */
-    SG_ERR_OVERFLOW = 9       /* a dimension exceeds INT32_MAX columns, or a cost sum could overflow int64 */
+    SG_ERR_OVERFLOW = 9       /* a dimension exceeds INT32_MAX, B.nnz >= INT32_MAX, or sum_i (c_L(i) + c_H(i)) over the
+                                 rows a cost-model call sees, evaluated in fp64, reaches 2^62 (so no int64 sum can wrap) */
 } sg_status;
 
 typedef enum { SG_F64 = 0, SG_F32 = 1 } sg_dtype;
@@ -63,7 +64,8 @@ typedef struct {
  *   c_H(i) = kappa_H + lambda_H*w_i + tau_H*a_i*R(u_i) + mu_H*u_i
  *   R(u)   = tiles_fixed if capu == 0, else max(1, ceil(u/capu))
  * with a_i = nnz(A_i), w_i = L_AB[i], u_i = nnz(C_i). cap_L is the largest admissible
- * threshold (the light path's table capacity); it must be <= SG_CAP_L_MAX. */
+ * threshold (the light path's table capacity); it must be <= SG_CAP_L_MAX. Every coefficient must be
+ * >= 0 (INVALID_ARG otherwise): costs are then non-negative and every cost prefix is monotone. */
 typedef struct {
     int64_t kappa_L, lambda_L, sigma_L, rho_L;
     int64_t kappa_H, lambda_H, tau_H, mu_H;
@@ -92,11 +94,21 @@ typedef struct {
     int64_t n_ranges;         /* heavy column ranges (numeric work items of the heavy path) */
     int64_t light_bins[13];   /* light rows per bin b: 2^(b-1) < w <= 2^b (b = 0: w == 1) */
     int64_t n_dense;          /* heavy rows on the dense-window kernel (w >= 2^dense_log2) */
-    int64_t dense_log2;       /* that row-work bound (SG_DW_LOG2 overrides; >= 62: path disabled) */
+    int64_t dense_log2;       /* that row-work bound (SG_OPT_DENSE_LOG2 overrides; 62: path disabled) */
     int64_t n_light_sorted;   /* light rows whose columns cluster (hash homes crowded): uniform hash + sort */
 } sg_plan_info;
 
 typedef struct sg_plan sg_plan;   /* opaque; owns only its workspace */
+
+/* Process-wide options, read by every later call (not per plan; set them before sg_symbolic).
+ *   SG_OPT_VALIDATE    0/1: check canonical CSR inputs on every call (SG_ERR_NOT_CANONICAL).
+ *   SG_OPT_DENSE_LOG2  -1 (default) = automatic; m in [0, 62]: heavy rows with w >= 2^m take the
+ *                      dense-window numeric kernel; 62 disables that path.
+ * The environment seeds them once, at the library's first call (SG_VALIDATE=1, SG_DW_LOG2=m).
+ * Errors: INVALID_ARG (unknown key or value out of range). sg_get_option: INT64_MIN if unknown. */
+typedef enum { SG_OPT_VALIDATE = 0, SG_OPT_DENSE_LOG2 = 1, SG_OPT_COUNT = 2 } sg_option;
+sg_status sg_set_option(int key, int64_t value);
+int64_t sg_get_option(int key);
 
 /* Human-readable status name (static storage). */
 const char* sg_status_string(sg_status st);
@@ -173,20 +185,29 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
 
 /* Numeric phase: writes C_col (int32[nnz_c]) and C_val (dtype[nnz_c]) for the plan's rows, each
  * row at [C_row_ptr[i], C_row_ptr[i+1]) with ascending columns; c_ij = sum_k a_ik*b_kj accumulated
- * in fp64 (stored in the input dtype). A and B must be the views given to sg_symbolic. */
+ * in fp64 (stored in the input dtype). A and B must be the views given to sg_symbolic. C_col must
+ * be 4-byte aligned and C_val aligned to its element size (INVALID_ARG otherwise); no larger
+ * alignment is assumed. `stream` may differ from the plan's stream: the plan's later frees are
+ * ordered after this call's work. A plan is not thread-safe: do not run two sg_numeric calls on one
+ * plan concurrently (they share its work counters). */
 sg_status sg_numeric(sg_plan* plan, const sg_csr_view* A, const sg_csr_view* B,
                      int32_t* C_col, void* C_val, void* stream);
 
 /* Assembly of the row-distributed C (Alg. 2 l.7, L224) over NCCL: rank r of the communicator owns
  * the plan rows [row_begin_r, row_end_r) (contiguous, in rank order, covering [0, n)). Gathers the
- * per-rank nnz (allgather), writes the GLOBAL row_ptr (n+1, device) on every rank (allgatherv of
+ * per-rank layout (allgather), writes the GLOBAL row_ptr (n+1, device) on every rank (allgatherv of
  * the local prefixes + offset fix-up) and, if gather_values != 0, the full C_col / C_val (nnz_total,
  * device) on every rank. nccl_comm is an ncclComm_t (e.g. ProcessGroupNCCL._comm_ptr()).
  * local_row_ptr / local_col / local_val are this rank's sg_symbolic / sg_numeric outputs.
- * nnz_total_out (host). Synchronises. Errors: NCCL, SHAPE (ranges not contiguous). */
+ * row_ptr_cap = entries of C_row_ptr_global, nnz_cap = entries of C_col_global / C_val_global
+ * (ignored when gather_values == 0): every rank's capacities are exchanged with the layout and the
+ * call returns SHAPE on EVERY rank, before any output is written, if some rank's buffers are smaller
+ * than n+1 / nnz_total. nnz_total_out (host). Synchronises. Errors: NCCL, SHAPE (ranges not
+ * contiguous, or a capacity too small), INVALID_ARG. */
 sg_status sg_gather(sg_plan* plan, void* nccl_comm, int gather_values,
                     const int64_t* local_row_ptr, const int32_t* local_col, const void* local_val,
-                    int64_t* C_row_ptr_global, int32_t* C_col_global /*nullable*/, void* C_val_global /*nullable*/,
+                    int64_t* C_row_ptr_global, int64_t row_ptr_cap,
+                    int32_t* C_col_global /*nullable*/, void* C_val_global /*nullable*/, int64_t nnz_cap,
                     int64_t* nnz_total_out /*host*/, void* stream);
 
 /* The host-only arithmetic of sg_gather (no device work, usable without a GPU): lay holds the

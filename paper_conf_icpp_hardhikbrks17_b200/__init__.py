@@ -38,7 +38,9 @@ EXPORTS = ["sg_status_string", "sg_version", "sg_default_cost_model", "sg_row_wo
            "sg_exhaustive_threshold", "sg_cost_curve", "sg_partition", "sg_symbolic", "sg_numeric", "sg_gather",
            "sg_plan_get_info", "sg_plan_get_classes", "sg_plan_get_work", "sg_plan_destroy", "sg_sample_rows",
            "sg_profile_enable", "sg_launch_count", "sg_profile_count", "sg_profile_read", "sg_profile_reset",
-           "sg_gather_layout", "sg_threshold_on_rows"]
+           "sg_gather_layout", "sg_threshold_on_rows", "sg_set_option", "sg_get_option"]
+
+SG_OPT_VALIDATE, SG_OPT_DENSE_LOG2 = 0, 1
 
 
 class SgError(RuntimeError):
@@ -121,7 +123,9 @@ def load(build_if_missing: bool = True):
         "sg_partition_cost": (st, [V, V, ctypes.c_int, i64, CM, P, P, pi64, P]),
         "sg_symbolic": (st, [V, V, i64, i64, i64, P, pi64, ctypes.POINTER(ctypes.c_void_p), P]),
         "sg_numeric": (st, [P, V, V, P, P, P]),
-        "sg_gather": (st, [P, P, ctypes.c_int, P, P, P, P, P, P, pi64, P]),
+        "sg_gather": (st, [P, P, ctypes.c_int, P, P, P, P, i64, P, P, i64, pi64, P]),
+        "sg_set_option": (st, [ctypes.c_int, i64]),
+        "sg_get_option": (i64, [ctypes.c_int]),
         "sg_plan_get_info": (st, [P, ctypes.POINTER(PlanInfo)]),
         "sg_plan_get_classes": (st, [P, P, P]),
         "sg_plan_get_work": (st, [P, P, P]),
@@ -365,23 +369,28 @@ def sg_numeric(plan: Plan, A: DeviceCSR, B: DeviceCSR, out=None):
     return col, val
 
 
-def sg_gather(plan: Plan, comm_ptr: int, local_col=None, local_val=None, gather_values: bool = False,
-              n_global: int | None = None, nnz_global: int | None = None):
+def sg_gather(plan: Plan, comm_ptr: int, n_global: int, local_col=None, local_val=None, gather_values: bool = False,
+              nnz_global: int | None = None):
     """Assembles the row-distributed C over NCCL (comm_ptr: ncclComm_t as int, e.g.
-    ProcessGroupNCCL._comm_ptr()). Returns (row_ptr_global, col_global|None, val_global|None, nnz_total)."""
+    ProcessGroupNCCL._comm_ptr()). n_global = rows of the global C (A.nrows); with gather_values,
+    nnz_global = total nnz of C (e.g. the sum of every rank's plan.nnz). The library checks both
+    against the gathered layout on every rank (SgError(SHAPE) everywhere if too small).
+    Returns (row_ptr_global, col_global|None, val_global|None, nnz_total)."""
     _require_cuda()
     dev = plan.row_ptr.device
-    n = n_global if n_global is not None else plan.row_end  # caller passes n when not the last rank
-    rp = torch.empty(n + 1, dtype=torch.int64, device=dev)
+    rp = torch.empty(n_global + 1, dtype=torch.int64, device=dev)
     col = val = None
+    cap = 0
     if gather_values:
-        assert nnz_global is not None, "gather_values needs nnz_global (allocate once, e.g. from a prior gather)"
+        if nnz_global is None:
+            raise ValueError("gather_values needs nnz_global (the total nnz of C over all ranks)")
         col = torch.empty(nnz_global, dtype=torch.int32, device=dev)
         val = torch.empty(nnz_global, dtype=plan.dtype, device=dev)
+        cap = nnz_global
     tot = ctypes.c_int64(0)
     _check(lib().sg_gather(plan.handle, ctypes.c_void_p(comm_ptr), int(gather_values), _ptr(plan.row_ptr),
-                           _ptr(local_col), _ptr(local_val), _ptr(rp), _ptr(col), _ptr(val), ctypes.byref(tot),
-                           _stream()), "sg_gather")
+                           _ptr(local_col), _ptr(local_val), _ptr(rp), n_global + 1, _ptr(col), _ptr(val), cap,
+                           ctypes.byref(tot), _stream()), "sg_gather")
     return rp, col, val, int(tot.value)
 
 
@@ -423,6 +432,15 @@ class profile:
 
 def launch_count() -> int:
     return int(lib().sg_launch_count())
+
+
+def set_option(key: int, value: int) -> None:
+    """sg_set_option: process-wide library options (SG_OPT_VALIDATE 0/1, SG_OPT_DENSE_LOG2 -1 or 0..62)."""
+    _check(lib().sg_set_option(int(key), int(value)), "sg_set_option")
+
+
+def get_option(key: int) -> int:
+    return int(lib().sg_get_option(int(key)))
 
 
 def sg_gather_layout(layouts):

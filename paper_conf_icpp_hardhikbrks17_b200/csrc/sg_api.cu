@@ -6,6 +6,7 @@
 #include <cmath>
 #include <vector>
 #include <mutex>
+#include <atomic>
 
 using namespace sg;
 
@@ -96,9 +97,25 @@ Mat mat_of(const sg_csr_view* v) {
     return m;
 }
 
+// Process-wide options (sg_set_option). The environment seeds them ONCE, at the first call
+// (SG_VALIDATE=1, SG_DW_LOG2=m); no call reads the environment afterwards.
+std::once_flag g_opt_once;
+std::atomic<int64_t> g_opt[SG_OPT_COUNT];
+
+void init_options() {
+    std::call_once(g_opt_once, [] {
+        g_opt[SG_OPT_VALIDATE] = 0;
+        g_opt[SG_OPT_DENSE_LOG2] = -1;
+        const char* e = getenv("SG_VALIDATE");
+        if (e && e[0] == '1') g_opt[SG_OPT_VALIDATE] = 1;
+        e = getenv("SG_DW_LOG2");
+        if (e && *e) g_opt[SG_OPT_DENSE_LOG2] = atoll(e);
+    });
+}
+
 bool env_validate() {
-    const char* e = getenv("SG_VALIDATE");
-    return e && e[0] == '1';
+    init_options();
+    return g_opt[SG_OPT_VALIDATE].load() != 0;
 }
 
 __global__ void k_validate(Mat M, int* bad) {
@@ -217,6 +234,17 @@ sg_status row_stats(const Mat& A, const Mat& B, const int64_t* rows, int64_t nr,
     return SG_OK;
 }
 
+// SG_ERR_OVERFLOW when sum_i (c_L(i) + c_H(i)) could leave int64 (kCostLimit = 2^62 in fp64)
+sg_status check_cost_bound(const CostModelD& cm, const RowStats& rs, int64_t nr, Scratch& sc, cudaStream_t s) {
+    double* dm = (double*)sc.get(sizeof(double));
+    if (!dm) return SG_ERR_OOM;
+    CK(launch_cost_mag(cm, rs.w, rs.a, rs.u, nr, dm, s));
+    double hm = 0.0;
+    CK(cudaMemcpyAsync(&hm, dm, sizeof(double), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    return hm >= kCostLimit ? SG_ERR_OVERFLOW : SG_OK;
+}
+
 sg_status identify(const Mat& A, const Mat& B, const int64_t* rows, int64_t nr, const sg_cost_model* c,
                    ThrResult* res, cudaStream_t s) {
     Scratch sc(s);
@@ -224,6 +252,7 @@ sg_status identify(const Mat& A, const Mat& B, const int64_t* rows, int64_t nr, 
     sg_status st = row_stats(A, B, rows, nr, c->cap_L, sc, rs, s);
     if (st != SG_OK) return st;
     CostModelD cm = cm_of(c);
+    if ((st = check_cost_bound(cm, rs, nr, sc, s)) != SG_OK) return st;
     size_t hb = sizeof(long long) * (size_t)(c->cap_L + 1);
     long long* hd = (long long*)sc.get(hb);
     long long* hc = (long long*)sc.get(hb);
@@ -248,9 +277,14 @@ sg_status identify(const Mat& A, const Mat& B, const int64_t* rows, int64_t nr, 
     return SG_OK;
 }
 
+// Non-negative coefficients keep every cost prefix monotone (k_cuts' binary search relies on it) and
+// make the fp64 magnitude sum of check_cost_bound an upper bound of every integer sum.
 sg_status check_model(const sg_cost_model* c) {
     if (c->cap_L < 0 || c->cap_L > SG_CAP_L_MAX) return SG_ERR_INVALID_ARG;
-    if (c->capu < 0 || c->tiles_fixed < 0) return SG_ERR_INVALID_ARG;
+    const int64_t co[] = {c->kappa_L, c->lambda_L, c->sigma_L, c->rho_L, c->kappa_H, c->lambda_H, c->tau_H, c->mu_H,
+                          c->tiles_fixed, c->capu};
+    for (int64_t x : co)
+        if (x < 0) return SG_ERR_INVALID_ARG;
     return SG_OK;
 }
 
@@ -275,6 +309,21 @@ const char* sg_status_string(sg_status st) {
 }
 
 const char* sg_version(void) { return "sg 0.1.0 sm_100a"; }
+
+sg_status sg_set_option(int key, int64_t value) {
+    init_options();
+    if (key < 0 || key >= SG_OPT_COUNT) return SG_ERR_INVALID_ARG;
+    if (key == SG_OPT_VALIDATE && value != 0 && value != 1) return SG_ERR_INVALID_ARG;
+    if (key == SG_OPT_DENSE_LOG2 && (value < -1 || value > 62)) return SG_ERR_INVALID_ARG;
+    g_opt[key] = value;
+    return SG_OK;
+}
+
+int64_t sg_get_option(int key) {
+    init_options();
+    if (key < 0 || key >= SG_OPT_COUNT) return INT64_MIN;
+    return g_opt[key].load();
+}
 
 void sg_default_cost_model(sg_cost_model* out) {
     if (out) *out = kDefaultModel;
@@ -450,6 +499,7 @@ sg_status sg_cost_curve(const sg_csr_view* A, const sg_csr_view* B, const sg_cos
     Mat a = mat_of(A), b = mat_of(B);
     st = row_stats(a, b, nullptr, A->nrows, c->cap_L, sc, rs, s);
     if (st != SG_OK) return st;
+    if ((st = check_cost_bound(cm_of(c), rs, A->nrows, sc, s)) != SG_OK) return st;
     int64_t* dt = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(nt > 0 ? nt : 1));
     long long* dJ = (long long*)sc.get(sizeof(long long) * (size_t)(nt > 0 ? nt : 1));
     if (!dt || !dJ) return SG_ERR_OOM;
@@ -507,10 +557,17 @@ sg_status sg_partition_cost(const sg_csr_view* A, const sg_csr_view* B, int npar
     int64_t* P = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(n + 1));
     void* tmp = sc.get(scan_tmp_bytes(n));
     int64_t* dcuts = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(nparts + 1));
-    if (!w || !cost || !P || !tmp || !dcuts) return SG_ERR_OOM;
+    double* dm = (double*)sc.get(sizeof(double));
+    if (!w || !cost || !P || !tmp || !dcuts || !dm) return SG_ERR_OOM;
     Mat a = mat_of(A), b = mat_of(B);
     CK(launch_row_work(a, b, 0, n, w, s));
-    CK(launch_row_cost(cm_of(c), thr, comp, A->row_ptr, w, n, cost, s));
+    CK(launch_row_cost(cm_of(c), thr, comp, A->row_ptr, w, n, cost, dm, s));
+    {
+        double hm = 0.0;
+        CK(cudaMemcpyAsync(&hm, dm, sizeof(double), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (hm >= kCostLimit) return SG_ERR_OVERFLOW;
+    }
     CK(scan_exclusive(cost, P, n, tmp, s));
     CK(launch_cuts(P, n, nparts, dcuts, s));
     CK(cudaMemcpyAsync(cuts_out, dcuts, sizeof(int64_t) * (size_t)(nparts + 1), cudaMemcpyDeviceToHost, s));
@@ -580,7 +637,8 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
         if (!pl->heavy || !hist || !pl->range_bounds || !pl->range_off || !pl->nranges || !t2) return fail(SG_ERR_OOM);
         CKF(launch_heavy_order(pl->lists + pl->bin_off[BIN_HEAVY], pl->nheavy, pl->w, hist, pl->heavy, s));
         // dense-window rows: w >= 2^dw_log2, a prefix of the heaviest-first order
-        pl->dw_log2 = dense_window_log2(pl->p);
+        init_options();
+        pl->dw_log2 = dense_window_log2(pl->p, g_opt[SG_OPT_DENSE_LOG2].load());
         const int64_t dw_min_w = pl->dw_log2 >= 62 ? INT64_MAX : ((int64_t)1 << pl->dw_log2);
         CKF(launch_range_bounds(pl->heavy, pl->nheavy, pl->w, pl->p, dw_min_w, pl->range_bounds, s));
         CKF(scan_exclusive(pl->range_bounds, pl->range_off, pl->nheavy, t2, s));
@@ -644,49 +702,24 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
     if (A->nrows < pl->re || B->ncols != pl->p || B->nrows != pl->m) return SG_ERR_SHAPE;
     if ((int)A->dtype != pl->dt || (int)B->dtype != pl->dt) return SG_ERR_DTYPE;
     if (pl->nnz_c > 0 && (!C_col || !C_val)) return SG_ERR_INVALID_ARG;
+    if (((uintptr_t)C_col & 3u) || ((uintptr_t)C_val & (pl->dt == 0 ? 7u : 3u))) return SG_ERR_INVALID_ARG;
     if (pl->nnz_c == 0) return SG_OK;
     Mat a = mat_of(A), b = mat_of(B);
     for (int k = 0; k < NBIN_LIGHT; ++k)
         CKP(pl, launch_num_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], pl->rb, pl->span, pl->C_rp,
                                  C_col, C_val, s));
     if (pl->nheavy > 0) {
-        // SG_DEBUG_HEAVY=1: per-phase cycle counters of the heavy numeric kernel, printed to stderr
-        const char* dbe = getenv("SG_DEBUG_HEAVY");
-        unsigned long long* dbg = nullptr;
-        if (dbe && dbe[0] == '1') {
-            CKP(pl, cudaMallocAsync((void**)&dbg, 17 * sizeof(unsigned long long), s));
-            CKP(pl, cudaMemsetAsync(dbg, 0, 17 * sizeof(unsigned long long), s));
-        }
-        if (dbg) {
-            unsigned long long* dd = nullptr;
-            CKP(pl, cudaMallocAsync((void**)&dd, 8 * sizeof(unsigned long long), s));
-            CKP(pl, cudaMemsetAsync(dd, 0, 8 * sizeof(unsigned long long), s));
-            CKP(pl, launch_num_dense(a, b, pl->heavy, pl->ndw, pl->rb, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
-                                     C_val, pl->counter, pl->gscr, pl->amax, pl->dtc, pl->ditems, pl->ditem_off + pl->ndw, s, dd));
-            unsigned long long h[8];
-            CKP(pl, cudaMemcpyAsync(h, dd, sizeof(h), cudaMemcpyDeviceToHost, s));
-            CKP(pl, cudaStreamSynchronize(s));
-            cudaFreeAsync(dd, s);
-            fprintf(stderr, "[sg dense] rows %lld Mcycles (sum over CTAs): fetch %.1f setup %.1f seg+compact %.1f "
-                            "products %.1f emit %.1f | windows %llu\n", (long long)pl->ndw,
-                    h[0] / 1e6, h[1] / 1e6, h[2] / 1e6, h[3] / 1e6, h[4] / 1e6, h[6]);
-        } else {
-            CKP(pl, launch_num_dense(a, b, pl->heavy, pl->ndw, pl->rb, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
-                                     C_val, pl->counter, pl->gscr, pl->amax, pl->dtc, pl->ditems, pl->ditem_off + pl->ndw, s));
-        }
+        CKP(pl, launch_num_dense(a, b, pl->heavy, pl->ndw, pl->rb, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
+                                 C_val, pl->counter, pl->gscr, pl->amax, pl->dtc, pl->ditems, pl->ditem_off + pl->ndw, s));
         CKP(pl, launch_num_heavy(a, b, pl->heavy, pl->ndw, pl->nheavy, pl->rb, pl->range_off, pl->nranges, pl->ranges,
-                                 pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter, pl->gscr, pl->amax, s,
-                                 dbg));
-        if (dbg) {
-            unsigned long long h[16];
-            CKP(pl, cudaMemcpyAsync(h, dbg, sizeof(h), cudaMemcpyDeviceToHost, s));
-            CKP(pl, cudaStreamSynchronize(s));
-            cudaFreeAsync(dbg, s);
-            fprintf(stderr, "[sg heavy] Mcycles (sum over CTAs): fetch %.1f init %.1f seg+compact %.1f pass1 %.1f "
-                            "prefix %.1f pass2 %.1f emit %.1f | ranges %llu | extra %.1f %.1f %.1f %.1f\n",
-                    h[0] / 1e6, h[1] / 1e6, h[2] / 1e6, h[3] / 1e6, h[4] / 1e6, h[5] / 1e6, h[6] / 1e6, h[7],
-                    h[8] / 1e6, h[9] / 1e6, h[10] / 1e6, h[11] / 1e6);
-        }
+                                 pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter, pl->gscr, pl->amax, s));
+    }
+    if (s != pl->s) {  // the plan's workspace frees (on pl->s) wait for this call's kernels
+        cudaEvent_t ev;
+        CKP(pl, cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+        CKP(pl, cudaEventRecord(ev, s));
+        CKP(pl, cudaStreamWaitEvent(pl->s, ev, 0));
+        cudaEventDestroy(ev);
     }
     return SG_OK;
 }

@@ -17,7 +17,6 @@
 // tile-pointer table tp (prefetched one window ahead), short rows count their entries below the
 // window end (cached in shared memory when two-tile windows leave room for it).
 #include "sg_device.cuh"
-#include <cstdlib>
 
 namespace sg {
 
@@ -56,12 +55,8 @@ __global__ void __launch_bounds__(DW_T, DW_OCC) k_num_dense(
     Mat A, Mat B, const int32_t* __restrict__ heavy, int64_t ndw, int64_t rb, const int32_t* __restrict__ long_id,
     const uint32_t* __restrict__ tp, int T, const int64_t* __restrict__ C_rp, int32_t* __restrict__ C_col,
     VT* __restrict__ C_val, unsigned long long* counter, int4* __restrict__ gscr, int64_t amax,
-    const int32_t* __restrict__ dtc, const int4* __restrict__ items, const int64_t* __restrict__ nitems,
-    unsigned long long* __restrict__ dbg) {
+    const int32_t* __restrict__ dtc, const int4* __restrict__ items, const int64_t* __restrict__ nitems) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    unsigned long long tph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-    long long t_last = clock64();
-    auto mark = [&](int k) { if (dbg && threadIdx.x == 0) { long long t = clock64(); tph[k] += t - t_last; t_last = t; } };
     DenseSmem& S = *reinterpret_cast<DenseSmem*>(smem_raw);
     __shared__ long long s_j;
     const int tid = threadIdx.x;
@@ -77,7 +72,6 @@ __global__ void __launch_bounds__(DW_T, DW_OCC) k_num_dense(
         const int64_t it = s_j;
         __syncthreads();
         if (it >= n_items) break;
-        mark(0);
         // work item: windows [ta, tb) of dense row h (a row with w_i products is cut into
         // ceil(w_i / DW_CHUNK_W) chunks of consecutive windows, so no single row is a tail)
         const int4 item = items[it];
@@ -145,7 +139,6 @@ __global__ void __launch_bounds__(DW_T, DW_OCC) k_num_dense(
                 gs[i] = make_int4(c0, 0, 0, 0);
             }
         }
-        mark(1);
 #ifndef SG_DW_PIPE
 #define SG_DW_PIPE 1
 #endif
@@ -267,7 +260,6 @@ __global__ void __launch_bounds__(DW_T, DW_OCC) k_num_dense(
                 }
                 int nk;
                 any = chunk_compact<DW_T, int32_t>(len, beg, a, S.s_beg, S.s_off, S.s_a, &nk, S.wsll);
-                mark(2);
                 if (any == 0) continue;  // block-uniform: nothing in this window
                 warp_slice<DW_T, true, VT, int32_t>(S.s_beg, S.s_off, S.s_a, nk, any, B, acc);
             } else {
@@ -294,9 +286,7 @@ __global__ void __launch_bounds__(DW_T, DW_OCC) k_num_dense(
                 }
                 if (any == 0) continue;
             }
-            if (dbg && tid == 0) tph[6] += 1;
             __syncthreads();  // every product of the window accumulated
-            mark(3);
             // ---- emission: thread tid owns columns [CPT*tid, CPT*tid + CPT) of the window; one block
             // scan of their popcounts places every run; each thread writes its set bits in order ----
             uint32_t hw;
@@ -322,12 +312,9 @@ __global__ void __launch_bounds__(DW_T, DW_OCC) k_num_dense(
                 }
             }
             pos += wtot;
-            mark(4);
             // the next window's chunk_compact barriers order these clears before its products
         }
     }
-    if (dbg && threadIdx.x == 0)
-        for (int k = 0; k < 8; ++k) atomicAdd(&dbg[k], tph[k]);
 }
 
 // ---- work items: chunks of consecutive windows per dense row ------------------------------------
@@ -373,8 +360,7 @@ cudaError_t launch_dense_items(const int32_t* heavy, int64_t ndw, const int64_t*
 cudaError_t launch_num_dense(const Mat& A, const Mat& B, const int32_t* heavy, int64_t ndw, int64_t rb,
                              const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
                              void* C_val, unsigned long long* counter, int4* gscr, int64_t amax,
-                             const int32_t* dtc, const int4* items, const int64_t* nitems, cudaStream_t s,
-                             unsigned long long* dbg) {
+                             const int32_t* dtc, const int4* items, const int64_t* nitems, cudaStream_t s) {
     if (ndw <= 0) return cudaSuccess;
     const int smem = (int)sizeof(DenseSmem);
     cudaError_t e = cudaMemsetAsync(counter, 0, sizeof(unsigned long long), s);  // item counter
@@ -383,11 +369,11 @@ cudaError_t launch_num_dense(const Mat& A, const Mat& B, const int32_t* heavy, i
     if (A.dt == 0) {
         if ((e = cudaFuncSetAttribute(k_num_dense<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
         SG_LAUNCH("k_num_dense", s, (k_num_dense<double><<<grid, DW_T, smem, s>>>(A, B, heavy, ndw, rb, long_id, tp, T, C_rp,
-                                                                                  C_col, (double*)C_val, counter, gscr, amax, dtc, items, nitems, dbg)));
+                                                                                  C_col, (double*)C_val, counter, gscr, amax, dtc, items, nitems)));
     } else {
         if ((e = cudaFuncSetAttribute(k_num_dense<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
         SG_LAUNCH("k_num_dense", s, (k_num_dense<float><<<grid, DW_T, smem, s>>>(A, B, heavy, ndw, rb, long_id, tp, T, C_rp,
-                                                                                 C_col, (float*)C_val, counter, gscr, amax, dtc, items, nitems, dbg)));
+                                                                                 C_col, (float*)C_val, counter, gscr, amax, dtc, items, nitems)));
     }
     return cudaGetLastError();
 }
@@ -402,9 +388,8 @@ namespace sg {
 // Rows with w >= 2^m take the dense-window kernel. Its fixed cost grows with the number of windows
 // (p / WD) while its saving over the rank kernel grows with w, so m tracks log2 p: 2^19 at p = 2^20
 // (C3: 283.5 vs 284.6 ms/step at 2^18), 2^17 at p = 2^18 (R-MAT 18: 35.2 vs 35.6 ms).
-int dense_window_log2(int64_t p) {
-    const char* e = getenv("SG_DW_LOG2");
-    if (e && *e) return atoi(e);
+int dense_window_log2(int64_t p, int64_t opt) {
+    if (opt >= 0) return (int)(opt > 62 ? 62 : opt);  // sg_set_option(SG_OPT_DENSE_LOG2); 62 disables the path
     int lp = 0;
     while (lp < 62 && ((int64_t)1 << lp) < p) ++lp;
     const int m = lp - 1;

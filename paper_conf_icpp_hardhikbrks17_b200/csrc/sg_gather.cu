@@ -51,8 +51,10 @@ extern "C" sg_status sg_gather_layout(const int64_t* lay, int nranks, int64_t* b
 
 extern "C" sg_status sg_gather(sg_plan* plan, void* nccl_comm, int gather_values, const int64_t* local_row_ptr,
                                const int32_t* local_col, const void* local_val, int64_t* C_row_ptr_global,
-                               int32_t* C_col_global, void* C_val_global, int64_t* nnz_total_out, void* stream) {
+                               int64_t row_ptr_cap, int32_t* C_col_global, void* C_val_global, int64_t nnz_cap,
+                               int64_t* nnz_total_out, void* stream) {
     if (!plan || !nccl_comm || !local_row_ptr || !C_row_ptr_global || !nnz_total_out) return SG_ERR_INVALID_ARG;
+    if (row_ptr_cap < 0 || nnz_cap < 0) return SG_ERR_INVALID_ARG;
     if (sg_internal_plan_poisoned(plan)) return SG_ERR_CUDA;
     cudaStream_t s = (cudaStream_t)stream;
     ncclComm_t comm = (ncclComm_t)nccl_comm;
@@ -65,19 +67,28 @@ extern "C" sg_status sg_gather(sg_plan* plan, void* nccl_comm, int gather_values
         return SG_ERR_INVALID_ARG;
     // 1. layout allgather
     int64_t* dlay = nullptr;
-    if (cudaMallocAsync(&dlay, sizeof(int64_t) * 3 * (size_t)(nranks + 1) * 2, s) != cudaSuccess) return SG_ERR_OOM;
-    int64_t mine[3] = {rb, re, nnz};
-    std::vector<int64_t> lay(3 * (size_t)nranks);
+    // every rank publishes (row_begin, row_end, nnz, row_ptr_cap, nnz_cap): the capacity check below is
+    // then evaluated on identical data by every rank, so all of them skip (or run) the broadcasts together
+    constexpr int NL = 5;
+    if (cudaMallocAsync(&dlay, sizeof(int64_t) * NL * (size_t)(nranks + 1) * 2, s) != cudaSuccess) return SG_ERR_OOM;
+    int64_t mine[NL] = {rb, re, nnz, row_ptr_cap, gather_values ? nnz_cap : INT64_MAX};
+    std::vector<int64_t> lay5(NL * (size_t)nranks), lay(3 * (size_t)nranks);
     sg_status st = SG_OK;
     do {
         if (cudaMemcpyAsync(dlay, mine, sizeof(mine), cudaMemcpyHostToDevice, s) != cudaSuccess) { st = SG_ERR_CUDA; break; }
-        if (ncclAllGather(dlay, dlay + 3, 3, ncclInt64, comm, s) != ncclSuccess) { st = SG_ERR_NCCL; break; }
-        if (cudaMemcpyAsync(lay.data(), dlay + 3, sizeof(int64_t) * 3 * nranks, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+        if (ncclAllGather(dlay, dlay + NL, NL, ncclInt64, comm, s) != ncclSuccess) { st = SG_ERR_NCCL; break; }
+        if (cudaMemcpyAsync(lay5.data(), dlay + NL, sizeof(int64_t) * NL * nranks, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
             cudaStreamSynchronize(s) != cudaSuccess) { st = SG_ERR_CUDA; break; }
+        for (int r = 0; r < nranks; ++r)
+            for (int q = 0; q < 3; ++q) lay[3 * r + q] = lay5[NL * r + q];
         // contiguity: rank order, covering [0, n); entry offsets of every rank's C rows
         std::vector<int64_t> off(nranks + 1, 0), begin(nranks);
         int64_t n = 0, total = 0;
         if ((st = sg_gather_layout(lay.data(), nranks, begin.data(), off.data(), &n, &total)) != SG_OK) break;
+        // capacities of EVERY rank's outputs (identical decision on all ranks; nothing written yet)
+        for (int r = 0; r < nranks; ++r)
+            if (lay5[NL * r + 3] < n + 1 || lay5[NL * r + 4] < total) st = SG_ERR_SHAPE;
+        if (st != SG_OK) break;
         // 2. allgatherv of the local prefixes (rows_r entries each, excluding the trailing total)
         if (ncclGroupStart() != ncclSuccess) { st = SG_ERR_NCCL; break; }
         for (int r = 0; r < nranks; ++r) {

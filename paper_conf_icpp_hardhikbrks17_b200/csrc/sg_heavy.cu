@@ -390,12 +390,8 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
     Mat A, Mat B, const int32_t* __restrict__ heavy, int64_t h0, int64_t nheavy, int64_t rb, const int64_t* __restrict__ range_off,
     const int32_t* __restrict__ nranges, const RangeRec* __restrict__ ranges, const int32_t* __restrict__ long_id,
     const uint32_t* __restrict__ tp, int T, const int64_t* __restrict__ C_rp, int32_t* __restrict__ C_col,
-    VT* __restrict__ C_val, unsigned long long* counter, int4* __restrict__ gscr, int64_t amax,
-    unsigned long long* __restrict__ dbg) {
+    VT* __restrict__ C_val, unsigned long long* counter, int4* __restrict__ gscr, int64_t amax) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    unsigned long long tph[12] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
-    long long t_last = clock64();
-    auto mark = [&](int k) { if (dbg && threadIdx.x == 0) { long long t = clock64(); tph[k] += t - t_last; t_last = t; } };
     HeavySmem& S = *reinterpret_cast<HeavySmem*>(smem_raw);
     __shared__ long long s_j;
     const int tid = threadIdx.x;
@@ -417,7 +413,6 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
         const int64_t h = s_j;
         __syncthreads();
         if (h >= nheavy) break;
-        mark(0);
         const int64_t li = heavy[h];
         const int64_t row = rb + li;
         const int64_t s0 = __ldg(A.rp + row), s1 = __ldg(A.rp + row + 1);
@@ -441,8 +436,6 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
             }
         }
         __syncthreads();
-        mark(1);
-        if (dbg && tid == 0) tph[7] += nr;
         RangeRec Rn;  // next range's record, loaded one range ahead
         if (nr > 0) Rn = rr[0];
         for (int ri = 0; ri < nr; ++ri) {
@@ -476,9 +469,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                     }
                 }
                 int nk;
-                mark(8);
                 const int ctot = chunk_compact<NUM_T, int32_t>(len, beg, a, S.s_beg, S.s_off, S.s_a, &nk, S.wsll);
-                mark(2);
                 const uint32_t bb = opaque_u32(a_bm - 4u * ((uint32_t)lo >> 5));  // &bm[(c - lo) >> 5] = bb + 4(c >> 5)
                 auto setbit = [&](int32_t c, double) {
                     if (c >= 0) red_or_s(bb + 4u * ((uint32_t)c >> 5), 1u << (c & 31));
@@ -502,7 +493,6 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 if (!single) __syncthreads();
             }
             __syncthreads();
-            mark(3);
             // ---- rank prefix over the range's words: thread t owns words [8t, 8t+8) (two 128-bit
             // loads, a sequential local prefix, one block scan, one 128-bit store of 8 uint16) ----
             {
@@ -513,7 +503,6 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 const int c4 = __popc(q1.x), c5 = __popc(q1.y), c6 = __popc(q1.z), c7 = __popc(q1.w);
                 int t2;
                 if (kBulk && tid == 0) bulk_wait_read();  // previous range's values have left shared memory
-                mark(9);
                 const int p0 = block_scan<NUM_T>(c0 + c1 + c2 + c3 + c4 + c5 + c6 + c7, &t2, S.ws);
                 if (kBulk) {
                     for (int e = tid; e < clear_n; e += NUM_T) S.vals[e] = 0.0;
@@ -529,10 +518,11 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 reinterpret_cast<uint4*>(S.pref)[tid] = o;  // words >= nwords are zero: harmless prefixes
             }
             __syncthreads();
-            mark(4);
             // ---- pass 2: every product accumulated at rank(c); the column is written on first arrival ----
             const int64_t base = crow + R.off;
-            const int sh = kBulk ? (int)(base & 1) : 0;  // vals[e + sh] and C_val[base + e] share 16 B alignment
+            // vals[e + sh] and C_val[base + e] share 16 B alignment: sh from the ADDRESS (C_val is 8 B aligned,
+            // sg_numeric checks; the caller's buffer itself need not be 16 B aligned)
+            const int sh = kBulk ? (int)(((uintptr_t)(C_val + base) >> 3) & 1u) : 0;
             // lo is a multiple of 32: word (c - lo) >> 5 = (c >> 5) - (lo >> 5), bit c & 31
             const uint32_t bw = opaque_u32(a_bm - 4u * ((uint32_t)lo >> 5));
             const uint32_t pw = a_pref - 2u * ((uint32_t)lo >> 5);
@@ -570,7 +560,6 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
             }
             if (kBulk) fence_proxy_async_smem();  // accumulator writes visible to the bulk copy
             __syncthreads();
-            mark(5);
             // ---- values by rank; bitmap cleared for the next range ----
             const int cnt = R.cnt;
             if constexpr (kBulk) {
@@ -594,22 +583,17 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 bm4[2 * tid] = make_uint4(0, 0, 0, 0);
                 bm4[2 * tid + 1] = make_uint4(0, 0, 0, 0);
             }
-            mark(10);
             // no barrier here: the next range's first reads of the cleared bitmap / accumulator and its
             // rewrite of the packed chunk arrays all come after chunk_compact's barriers
-            mark(6);
         }
     }
     if (kBulk && tid == 0) bulk_wait_all();
-    if (dbg && threadIdx.x == 0)
-        for (int k = 0; k < 12; ++k) atomicAdd(&dbg[k], tph[k]);
 }
 
 cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, int64_t h0, int64_t nheavy, int64_t rb,
                              const int64_t* range_off, const int32_t* nranges, const RangeRec* ranges,
                              const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
-                             void* C_val, unsigned long long* counter, int4* gscr, int64_t amax, cudaStream_t s,
-                             unsigned long long* dbg) {
+                             void* C_val, unsigned long long* counter, int4* gscr, int64_t amax, cudaStream_t s) {
     if (nheavy - h0 <= 0) return cudaSuccess;
     const int smem = (int)sizeof(HeavySmem);
     cudaError_t e = cudaMemsetAsync(counter, 0, sizeof(unsigned long long), s);
@@ -620,12 +604,12 @@ cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, i
         if ((e = cudaFuncSetAttribute(k_num_heavy<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
         SG_LAUNCH("k_num_heavy", s, (k_num_heavy<double><<<grid, NUM_T, smem, s>>>(
                                         A, B, heavy, h0, nheavy, rb, range_off, nranges, ranges, long_id, tp, T, C_rp, C_col,
-                                        (double*)C_val, counter, gscr, amax, dbg)));
+                                        (double*)C_val, counter, gscr, amax)));
     } else {
         if ((e = cudaFuncSetAttribute(k_num_heavy<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
         SG_LAUNCH("k_num_heavy", s, (k_num_heavy<float><<<grid, NUM_T, smem, s>>>(
                                         A, B, heavy, h0, nheavy, rb, range_off, nranges, ranges, long_id, tp, T, C_rp, C_col,
-                                        (float*)C_val, counter, gscr, amax, dbg)));
+                                        (float*)C_val, counter, gscr, amax)));
     }
     return cudaGetLastError();
 }

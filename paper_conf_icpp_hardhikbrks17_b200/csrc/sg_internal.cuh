@@ -99,22 +99,20 @@ cudaError_t launch_sym_heavy(const Mat& A, const Mat& B, const int32_t* list, in
 cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, int64_t h0, int64_t nheavy, int64_t rb,
                              const int64_t* range_off, const int32_t* nranges, const RangeRec* ranges,
                              const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
-                             void* C_val, unsigned long long* counter, int4* gscr, int64_t amax, cudaStream_t s,
-                             unsigned long long* dbg = nullptr);
+                             void* C_val, unsigned long long* counter, int4* gscr, int64_t amax, cudaStream_t s);
 cudaError_t launch_max_a(const Mat& A, const int32_t* list, int64_t cnt, int64_t rb, unsigned long long* out,
                          cudaStream_t s);
 // dense-window heavy rows (sg_dense.cu): heavy[0, ndw), all with w >= 2^dense_window_log2(p)
 cudaError_t launch_num_dense(const Mat& A, const Mat& B, const int32_t* heavy, int64_t ndw, int64_t rb,
                              const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
                              void* C_val, unsigned long long* counter, int4* gscr, int64_t amax,
-                             const int32_t* dtc, const int4* items, const int64_t* nitems, cudaStream_t s,
-                             unsigned long long* dbg = nullptr);
+                             const int32_t* dtc, const int4* items, const int64_t* nitems, cudaStream_t s);
 // dense-window work items (row, window range): at most dense_items_bound(ndw, p); off[ndw] = count
 int64_t dense_items_bound(int64_t ndw, int64_t p);
 cudaError_t launch_dense_items(const int32_t* heavy, int64_t ndw, const int64_t* w, int64_t p, int64_t* cnt,
                                int64_t* off, void* scan_tmp, int4* items, cudaStream_t s);
 int dense_window_cols();
-int dense_window_log2(int64_t p);  // SG_DW_LOG2 overrides (>= 62 disables the dense-window path)
+int dense_window_log2(int64_t p, int64_t opt);  // opt >= 0 overrides (sg_set_option; 62 disables the path)
 int heavy_kc();
 int heavy_grid();
 int dense_grid();
@@ -130,7 +128,12 @@ cudaError_t launch_cost_curve(const CostModelD& cm, const int64_t* w, const int6
                               const int64_t* t, int nt, long long* J, cudaStream_t s);
 cudaError_t launch_cuts(const int64_t* P, int64_t n, int G, int64_t* cuts, cudaStream_t s);
 cudaError_t launch_row_cost(const CostModelD& cm, int64_t thr, const int64_t* comp /*host, 4*/, const int64_t* arp,
-                            const int64_t* w, int64_t n, int64_t* cost, cudaStream_t s);
+                            const int64_t* w, int64_t n, int64_t* cost, double* mag /*sum of c_L + c_H in fp64*/,
+                            cudaStream_t s);
+// sum over rows with w > 0 of c_L + c_H in fp64 (the overflow bound; sg_kernels.cu)
+cudaError_t launch_cost_mag(const CostModelD& cm, const int64_t* w, const int64_t* a, const int64_t* u, int64_t nr,
+                            double* out, cudaStream_t s);
+constexpr double kCostLimit = 4611686018427387904.0;  // 2^62: a cost bound at or above it -> SG_ERR_OVERFLOW
 cudaError_t launch_class_usum(const int64_t* w, const int64_t* u, int64_t nr, int64_t thr, unsigned long long* out,
                               cudaStream_t s);
 cudaError_t launch_gather_rows(const int64_t* src, const int64_t* rows, int64_t nr, int64_t* dst, cudaStream_t s);

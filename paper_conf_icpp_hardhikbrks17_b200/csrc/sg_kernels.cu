@@ -279,11 +279,42 @@ __device__ __forceinline__ long long costH(const CostModelD& cm, long long w, lo
     return cm.kH + cm.lH * w + cm.tH * a * R + cm.mH * u;
 }
 
+// Overflow guard (include/sg.h SG_ERR_OVERFLOW): the same per-row costs evaluated in fp64. Every
+// coefficient is non-negative (check_model), so sum over rows of c_L + c_H bounds |J|, every prefix
+// of the histogram and every cut target; the host rejects the model when that bound reaches 2^62.
+__device__ __forceinline__ double cost_mag(const CostModelD& cm, double w, double a, double u) {
+    const double lg = (double)ceil_log2_max2((long long)u);
+    const double R = cm.capu == 0 ? (double)cm.tiles_fixed : fmax(1.0, ceil(u / (double)cm.capu));
+    const double cl = (double)cm.kL + (double)cm.lL * w + (double)cm.sL * u * lg + (double)cm.rL * u;
+    const double ch = (double)cm.kH + (double)cm.lH * w + (double)cm.tH * a * R + (double)cm.mH * u;
+    return cl + ch;
+}
+
+__global__ void k_cost_mag(CostModelD cm, const int64_t* __restrict__ w, const int64_t* __restrict__ a,
+                           const int64_t* __restrict__ u, int64_t nr, double* out) {
+    double m = 0.0;
+    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < nr; j += (int64_t)gridDim.x * blockDim.x) {
+        const long long wj = w[j];
+        if (wj > 0) m += cost_mag(cm, (double)wj, (double)a[j], (double)u[j]);
+    }
+    m = warp_sum(m);
+    if ((threadIdx.x & 31) == 0 && m != 0.0) atomicAdd(out, m);
+}
+
+cudaError_t launch_cost_mag(const CostModelD& cm, const int64_t* w, const int64_t* a, const int64_t* u, int64_t nr,
+                            double* out, cudaStream_t s) {
+    cudaError_t e = cudaMemsetAsync(out, 0, sizeof(double), s);
+    if (e != cudaSuccess || nr <= 0) return e;
+    SG_LAUNCH("k_cost_mag", s, k_cost_mag<<<grid_for(nr, 1024, 148 * 8), 256, 0, s>>>(cm, w, a, u, nr, out));
+    return cudaGetLastError();
+}
+
 // ---- NEXT #2: modeled per-row cost for the cost-weighted split (R19) -----------------
 // c_i = 0 (w = 0), c_L(w, a, uh) (w <= thr), c_H(w, a, uh) (w > thr); uh = min(w, ceil(w U_c / W_c)).
 __global__ void k_row_cost(CostModelD cm, long long thr, long long UL, long long WL, long long UH, long long WH,
                            const int64_t* __restrict__ arp, const int64_t* __restrict__ w, int64_t n,
-                           int64_t* __restrict__ cost) {
+                           int64_t* __restrict__ cost, double* __restrict__ mag) {
+    double m = 0.0;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         const long long wi = w[i];
         if (wi == 0) { cost[i] = 0; continue; }
@@ -296,14 +327,18 @@ __global__ void k_row_cost(CostModelD cm, long long thr, long long UL, long long
             if (q < (__int128)uh) uh = (long long)q;
         }
         cost[i] = light ? costL(cm, wi, ai, uh) : costH(cm, wi, ai, uh);
+        m += cost_mag(cm, (double)wi, (double)ai, (double)uh);
     }
+    m = warp_sum(m);
+    if ((threadIdx.x & 31) == 0 && m != 0.0) atomicAdd(mag, m);
 }
 
 cudaError_t launch_row_cost(const CostModelD& cm, int64_t thr, const int64_t* comp, const int64_t* arp,
-                            const int64_t* w, int64_t n, int64_t* cost, cudaStream_t s) {
-    if (n <= 0) return cudaSuccess;
+                            const int64_t* w, int64_t n, int64_t* cost, double* mag, cudaStream_t s) {
+    cudaError_t e = cudaMemsetAsync(mag, 0, sizeof(double), s);
+    if (e != cudaSuccess || n <= 0) return e;
     SG_LAUNCH("k_row_cost", s, k_row_cost<<<grid_for(n, 256, 148 * 8), 256, 0, s>>>(cm, thr, comp[0], comp[1], comp[2],
-                                                                                       comp[3], arp, w, n, cost));
+                                                                                       comp[3], arp, w, n, cost, mag));
     return cudaGetLastError();
 }
 

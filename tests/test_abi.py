@@ -45,3 +45,35 @@ def test_product_path_never_imports_the_oracle():
             if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
                 txt = open(os.path.join(dp, f)).read()
                 assert "oracle" not in re.sub(r"(#|//).*", "", txt).lower().replace("oracle/", ""), f
+
+
+def test_options_roundtrip_and_validation():
+    """sg_set_option / sg_get_option (host-only): ranges enforced, unknown keys rejected."""
+    import paper_conf_icpp_hardhikbrks17_b200 as sg
+    old = sg.get_option(sg.SG_OPT_DENSE_LOG2)
+    try:
+        sg.set_option(sg.SG_OPT_DENSE_LOG2, 17)
+        assert sg.get_option(sg.SG_OPT_DENSE_LOG2) == 17
+        for bad in (-2, 63):
+            with pytest.raises(sg.SgError, match="INVALID_ARG"):
+                sg.set_option(sg.SG_OPT_DENSE_LOG2, bad)
+        with pytest.raises(sg.SgError, match="INVALID_ARG"):
+            sg.set_option(sg.SG_OPT_VALIDATE, 2)
+        with pytest.raises(sg.SgError, match="INVALID_ARG"):
+            sg.set_option(99, 0)
+        assert sg.load().sg_get_option(99) == -(2**63)
+    finally:
+        sg.set_option(sg.SG_OPT_DENSE_LOG2, old)
+
+
+def test_negative_cost_coefficients_rejected_before_device_work():
+    """A cost model with a negative coefficient is INVALID_ARG (include/sg.h): the check precedes
+    any device access, so it runs here on fake (never dereferenced) pointers."""
+    import paper_conf_icpp_hardhikbrks17_b200 as sg
+    L = sg.load()
+    v = sg.CsrView(4, 4, 0, 8, 0, 0, 0)
+    cm = sg.sg_default_cost_model()
+    cm.tau_H = -1
+    thr = ctypes.c_int64(0)
+    st = L.sg_sample_threshold(ctypes.byref(v), ctypes.byref(v), 0.5, 1, ctypes.byref(cm), ctypes.byref(thr), None, None)
+    assert st == 1  # SG_ERR_INVALID_ARG

@@ -21,6 +21,14 @@ def _dev(H):
     return sg.DeviceCSR.from_host(H)
 
 
+@pytest.fixture
+def dense_log2():
+    """Forces the dense-window bound (sg_set_option(SG_OPT_DENSE_LOG2, m)); restored afterwards."""
+    old = sg.get_option(sg.SG_OPT_DENSE_LOG2)
+    yield lambda m: sg.set_option(sg.SG_OPT_DENSE_LOG2, m)
+    sg.set_option(sg.SG_OPT_DENSE_LOG2, old)
+
+
 def _model_from(cm_sg):
     o = oracle.CostModel()
     for k, v in cm_sg.as_dict().items():
@@ -419,8 +427,7 @@ def test_gather_single_rank_nccl():
         dA = _dev(A)
         plan = sg.sg_symbolic(dA, dA, 256)
         col, val = sg.sg_numeric(plan, dA, dA)
-        rp, gcol, gval, tot = sg.sg_gather(plan, comm, col, val, gather_values=True, n_global=A.nrows,
-                                           nnz_global=plan.nnz)
+        rp, gcol, gval, tot = sg.sg_gather(plan, comm, A.nrows, col, val, gather_values=True, nnz_global=plan.nnz)
         torch.cuda.synchronize()
         assert tot == plan.nnz
         assert torch.equal(rp, plan.row_ptr)
@@ -451,11 +458,11 @@ def test_rmat22_multi_window_row_subset():
     plan.destroy()
 
 
-@pytest.mark.parametrize("dw", ["0", "99"])
+@pytest.mark.parametrize("dw", ["0", "62"])
 @pytest.mark.parametrize("name,thr", [("rmat12", 0), ("rmat16", 2048), ("C1", 16)])
-def test_dense_window_path_forced(monkeypatch, name, thr, dw):
-    """Every heavy row on the dense-window kernel (SG_DW_LOG2=0) or none (99): same C either way."""
-    monkeypatch.setenv("SG_DW_LOG2", dw)
+def test_dense_window_path_forced(dense_log2, name, thr, dw):
+    """Every heavy row on the dense-window kernel (SG_OPT_DENSE_LOG2 = 0) or none (62): same C either way."""
+    dense_log2(int(dw))
     A = gen.config(name)
     (rp, col, val), info, _ = _full_product(A, A, thr)
     R = oracle.spgemm(A, A, with_absmag=True)
@@ -465,10 +472,10 @@ def test_dense_window_path_forced(monkeypatch, name, thr, dw):
 
 
 @pytest.mark.parametrize("dtype", ["f64", "f32"])
-def test_dense_window_integer_values_exact(monkeypatch, dtype):
+def test_dense_window_integer_values_exact(dense_log2, dtype):
     """Dense-window accumulation in integer-value mode: values bit-exact (R11); includes
     rows with more than 1024 k entries (multi-chunk) at R-MAT 16."""
-    monkeypatch.setenv("SG_DW_LOG2", "0")
+    dense_log2(0)
     A = gen.config("rmat16", mode="int", dtype=dtype)
     (rp, col, val), info, _ = _full_product(A, A, 1024)
     assert int(np.diff(A.row_ptr).max()) > 1024
