@@ -10,6 +10,7 @@ Functions and the passage each follows (details in oracle.cpp's header):
 
 * ``row_work``            O2  w_i = sum_{k in A_i} nnz(B_k)
 * ``spgemm`` / ``counts`` O1  Gustavson, sorted-map accumulator
+* ``moments``             O1  per-row structure digest (u, sum c^1..3) PAPER L74, L222-L223
 * ``sample_rows``         sampler, Bernoulli(f) by SplitMix64       PAPER L92 (uniform sampling)
 * ``J`` / ``threshold``   O4  Identify: best candidate on the sample PAPER L87-L89, L232-L236
 * ``sampled_threshold``   Sample -> Identify -> Extrapolate(identity)
@@ -68,6 +69,7 @@ def _L():
         lib.oracle_tag_sample.restype = u64
         lib.oracle_row_work.argtypes = [i64, P, P, P, P]
         lib.oracle_spgemm_count.argtypes = [P, P, P, P, i64, P, P]
+        lib.oracle_spgemm_moments.argtypes = [P, P, P, P, i64, P, P]
         lib.oracle_spgemm_fill.argtypes = [P, P, P, ctypes.c_int, P, P, P, ctypes.c_int, i64, P, P, P, P, P]
         lib.oracle_sample_rows.restype = i64
         lib.oracle_sample_rows.argtypes = [i64, i64, u64, ctypes.c_double, P]
@@ -138,6 +140,15 @@ class RowsResult:
     @property
     def nnz(self):
         return int(self.row_ptr[-1])
+
+
+def moments(A, B, rows=None) -> np.ndarray:
+    """Per listed row (u_i, sum c, sum c^2, sum c^3) over the columns of C_i, sums mod 2^64 (uint64[n, 4])."""
+    rows = np.arange(A.nrows, dtype=np.int64) if rows is None else np.ascontiguousarray(rows, dtype=np.int64)
+    out = np.zeros((rows.shape[0], 4), dtype=np.uint64)
+    if rows.shape[0]:
+        _L().oracle_spgemm_moments(_p(A.row_ptr), _p(A.col), _p(B.row_ptr), _p(B.col), rows.shape[0], _p(rows), _p(out))
+    return out
 
 
 def spgemm(A, B, rows=None, with_absmag: bool = False) -> RowsResult:

@@ -17,6 +17,8 @@
  *        l.5-6 (L222-L223). Structural semantics: an entry exists iff some product exists,
  *        even if its value sums to zero (reading R9). Accumulation in fp64 from the
  *        (possibly fp32) inputs.
+ *        oracle_spgemm_moments: the same accumulator, reporting per row u_i and the sums of c, c^2,
+ *        c^3 over its columns (mod 2^64) — a structure digest for C that does not fit in host memory.
  *   O2 oracle_row_work
  *        L_AB = A x V_B with V_B[k] = nnz(B_k): w_i = sum_{k in A_i} nnz(B_k), the work volume
  *        of row i (Alg. 2 l.1 L215).
@@ -109,6 +111,33 @@ void oracle_spgemm_count(const int64_t* Arp, const int32_t* Acol,
             for (int64_t q = Brp[k]; q < Brp[k + 1]; ++q) acc[Bcol[q]] += 0.0;
         }
         u[s] = (int64_t)acc.size();
+    }
+}
+
+// Structure moments of the listed rows (for parity at sizes whose C does not fit host memory):
+// m[4s..4s+3] = (u_i, sum c, sum c^2, sum c^3) over the columns c of C_i = the keys of the same
+// sorted-map accumulator, sums modulo 2^64 (unsigned wrap-around).
+void oracle_spgemm_moments(const int64_t* Arp, const int32_t* Acol, const int64_t* Brp, const int32_t* Bcol,
+                           int64_t nsel, const int64_t* rows, uint64_t* m) {
+    #pragma omp parallel for schedule(dynamic, 1)
+    for (int64_t s = 0; s < nsel; ++s) {
+        int64_t i = rows[s];
+        std::map<int32_t, double> acc;
+        for (int64_t p = Arp[i]; p < Arp[i + 1]; ++p) {
+            int32_t k = Acol[p];
+            for (int64_t q = Brp[k]; q < Brp[k + 1]; ++q) acc[Bcol[q]] += 0.0;
+        }
+        uint64_t s1 = 0, s2 = 0, s3 = 0;
+        for (const auto& kv : acc) {
+            uint64_t c = (uint64_t)(uint32_t)kv.first;
+            s1 += c;
+            s2 += c * c;
+            s3 += c * c * c;
+        }
+        m[4 * s] = (uint64_t)acc.size();
+        m[4 * s + 1] = s1;
+        m[4 * s + 2] = s2;
+        m[4 * s + 3] = s3;
     }
 }
 

@@ -40,7 +40,7 @@ EXPORTS = ["sg_status_string", "sg_version", "sg_default_cost_model", "sg_row_wo
            "sg_profile_enable", "sg_launch_count", "sg_profile_count", "sg_profile_read", "sg_profile_reset",
            "sg_gather_layout", "sg_threshold_on_rows", "sg_set_option", "sg_get_option"]
 
-SG_OPT_VALIDATE, SG_OPT_DENSE_LOG2 = 0, 1
+SG_OPT_VALIDATE, SG_OPT_DENSE_LOG2, SG_OPT_VARIANT = 0, 1, 2
 
 
 class SgError(RuntimeError):

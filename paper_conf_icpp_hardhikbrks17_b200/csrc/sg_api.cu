@@ -38,6 +38,9 @@ struct sg_plan {
     int dw_log2 = 0;
     int2* span = nullptr;           // light rows: [cmin, cmax] of the output columns
     int4* gscr = nullptr;           // heavy rows with more than KC entries: per-k cursor scratch
+    void* pscr = nullptr;           // dense2: per-CTA part scratch for rows with many k entries
+    int64_t pscr_cap = 0;
+    int variant = 0;
     int32_t* long_id = nullptr;
     uint32_t* tp = nullptr;
     int64_t nlong = 0;
@@ -106,6 +109,7 @@ void init_options() {
     std::call_once(g_opt_once, [] {
         g_opt[SG_OPT_VALIDATE] = 0;
         g_opt[SG_OPT_DENSE_LOG2] = -1;
+        g_opt[SG_OPT_VARIANT] = 0;
         const char* e = getenv("SG_VALIDATE");
         if (e && e[0] == '1') g_opt[SG_OPT_VALIDATE] = 1;
         e = getenv("SG_DW_LOG2");
@@ -315,6 +319,7 @@ sg_status sg_set_option(int key, int64_t value) {
     if (key < 0 || key >= SG_OPT_COUNT) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_VALIDATE && value != 0 && value != 1) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_DENSE_LOG2 && (value < -1 || value > 62)) return SG_ERR_INVALID_ARG;
+    if (key == SG_OPT_VARIANT && (value < 0 || value > 1)) return SG_ERR_INVALID_ARG;
     g_opt[key] = value;
     return SG_OK;
 }
@@ -670,6 +675,12 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
         pl->ranges = (RangeRec*)palloc(pl, sizeof(RangeRec) * (size_t)(pl->nslots > 0 ? pl->nslots : 1));
         pl->tp = (uint32_t*)palloc(pl, 4 * (size_t)(pl->nlong > 0 ? pl->nlong : 1) * (size_t)(pl->T + 1));
         if (!pl->ranges || !pl->tp) return fail(SG_ERR_OOM);
+        pl->variant = (int)g_opt[SG_OPT_VARIANT].load();
+        if (pl->ndw > 0 && pl->amax + 32 > dense2_pcap()) {
+            pl->pscr_cap = pl->amax + 32;
+            pl->pscr = palloc(pl, dense2_part_bytes() * (size_t)pl->pscr_cap * 148);
+            if (!pl->pscr) return fail(SG_ERR_OOM);
+        }
         if (pl->amax > heavy_kc() || pl->amax > dense_kc()) {
             pl->gscr = (int4*)palloc(pl, sizeof(int4) * (size_t)(heavy_grid() > dense_grid() ? heavy_grid() : dense_grid()) * (size_t)pl->amax);
             if (!pl->gscr) return fail(SG_ERR_OOM);
@@ -709,8 +720,13 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
         CKP(pl, launch_num_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], pl->rb, pl->span, pl->C_rp,
                                  C_col, C_val, s));
     if (pl->nheavy > 0) {
-        CKP(pl, launch_num_dense(a, b, pl->heavy, pl->ndw, pl->rb, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
-                                 C_val, pl->counter, pl->gscr, pl->amax, pl->dtc, pl->ditems, pl->ditem_off + pl->ndw, s));
+        if (pl->variant & 1)
+            CKP(pl, launch_num_dense(a, b, pl->heavy, pl->ndw, pl->rb, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
+                                     C_val, pl->counter, pl->gscr, pl->amax, pl->dtc, pl->ditems, pl->ditem_off + pl->ndw, s));
+        else
+            CKP(pl, launch_num_dense2(a, b, pl->heavy, pl->ndw, pl->rb, pl->w, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
+                                      C_val, pl->counter, pl->pscr, pl->pscr_cap, pl->dtc, pl->ditems,
+                                      pl->ditem_off + pl->ndw, s));
         CKP(pl, launch_num_heavy(a, b, pl->heavy, pl->ndw, pl->nheavy, pl->rb, pl->range_off, pl->nranges, pl->ranges,
                                  pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter, pl->gscr, pl->amax, s));
     }

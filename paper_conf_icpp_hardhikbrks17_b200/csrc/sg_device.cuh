@@ -71,6 +71,17 @@ __device__ __forceinline__ double atom_add_f64_s(uint32_t a, double v) {
     asm volatile("atom.shared.add.f64 %0, [%1], %2;" : "=d"(old) : "r"(a), "d"(v) : "memory");
     return old;
 }
+// The same two accumulator atomics WITHOUT a compiler memory clobber: global loads may be scheduled
+// across them (software pipelining of the B gathers). Only for accumulators whose plain shared reads
+// and writes are all separated from the atomics by __syncthreads().
+__device__ __forceinline__ double atom_add_f64_s_nc(uint32_t a, double v) {
+    double old;
+    asm volatile("atom.shared.add.f64 %0, [%1], %2;" : "=d"(old) : "r"(a), "d"(v));
+    return old;
+}
+__device__ __forceinline__ void red_or_s_nc(uint32_t a, uint32_t v) {
+    asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(v));
+}
 __device__ __forceinline__ void red_or_s(uint32_t a, uint32_t v) {
     asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
 }

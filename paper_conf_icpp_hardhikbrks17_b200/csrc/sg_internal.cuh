@@ -107,6 +107,14 @@ cudaError_t launch_num_dense(const Mat& A, const Mat& B, const int32_t* heavy, i
                              const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
                              void* C_val, unsigned long long* counter, int4* gscr, int64_t amax,
                              const int32_t* dtc, const int4* items, const int64_t* nitems, cudaStream_t s);
+// dense-window rows, lean product walk (sg_dense2.cu); pscr: per-CTA part scratch (pscr_cap parts) for
+// rows with more than dense2_pcap() - 32 k entries
+cudaError_t launch_num_dense2(const Mat& A, const Mat& B, const int32_t* heavy, int64_t ndw, int64_t rb,
+                              const int64_t* w, const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp,
+                              int32_t* C_col, void* C_val, unsigned long long* counter, void* pscr, int64_t pscr_cap,
+                              const int32_t* dtc, const int4* items, const int64_t* nitems, cudaStream_t s);
+size_t dense2_part_bytes();
+int dense2_pcap();
 // dense-window work items (row, window range): at most dense_items_bound(ndw, p); off[ndw] = count
 int64_t dense_items_bound(int64_t ndw, int64_t p);
 cudaError_t launch_dense_items(const int32_t* heavy, int64_t ndw, const int64_t* w, int64_t p, int64_t* cnt,

@@ -22,8 +22,9 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 _SO = os.path.join(_HERE, "libsginputs.so")
 _lib = None
 
-VAL_REAL, VAL_INT, VAL_ONES = 0, 1, 2
-_MODES = {"real": VAL_REAL, "int": VAL_INT, "ones": VAL_ONES}
+VAL_REAL, VAL_INT, VAL_ONES, VAL_SIGNED, VAL_ZEROS = 0, 1, 2, 3, 4
+# real U[0.5,1.5); int {1,2,3,4}; ones; signed {-2,-1,1,2} (exact cancellation); zeros {-1,0,1,2} (stored zeros)
+_MODES = {"real": VAL_REAL, "int": VAL_INT, "ones": VAL_ONES, "signed": VAL_SIGNED, "zeros": VAL_ZEROS}
 
 
 def build(force: bool = False) -> str:

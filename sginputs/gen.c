@@ -128,7 +128,9 @@ int64_t sginputs_csr_from_edges(int64_t n, int64_t m, const int32_t* ei, const i
     return off;
 }
 
-/* Values per unique (i, j) (Q11). mode 0: real U[0.5,1.5); 1: integer {1,2,3,4}; 2: all ones.
+/* Values per unique (i, j) (Q11). mode 0: real U[0.5,1.5); 1: integer {1,2,3,4}; 2: all ones;
+ * 3: signed integer {-2,-1,1,2} (exact cancellation to 0 happens: structural zeros, R9);
+ * 4: {-1, 0, 1, 2} (explicitly STORED zeros in the inputs).
  * out is double (is_f32 == 0) or float (is_f32 == 1). */
 void sginputs_values(int64_t n, int64_t p, const int64_t* row_ptr, const int32_t* col,
                      uint64_t seed, int mode, int is_f32, void* out) {
@@ -140,6 +142,8 @@ void sginputs_values(int64_t n, int64_t p, const int64_t* row_ptr, const int32_t
             else {
                 uint64_t x = h3(seed, TAG_VAL, (uint64_t)i * (uint64_t)p + (uint64_t)col[q]);
                 if (mode == 1) v = (double)(1 + (x & 3));
+                else if (mode == 3) v = (double)((int)(x & 3) - 2 + ((x & 3) >= 2));
+                else if (mode == 4) v = (double)((int)(x & 3) - 1);
                 else v = 0.5 + (double)(x >> 11) * 0x1.0p-53;
             }
             if (is_f32) ((float*)out)[q] = (float)v; else ((double*)out)[q] = v;

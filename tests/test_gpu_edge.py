@@ -1,0 +1,111 @@
+"""GPU parity on the method's edge cases: exact cancellation and explicitly stored zeros (structural
+semantics, reading R9) with every kernel path forced, in fp64, fp32 and integer values.
+
+Values here are small signed integers ({-2,-1,1,2} or {-1,0,1,2}, sginputs modes "signed" / "zeros"),
+so every sum is an exact integer below 2^24: values must be BIT-EXACT in fp64 and fp32 alike, and an
+entry whose sum is 0 must still be present (C's structure = the boolean product of the stored
+patterns, PAPER L74 / Alg. 2 l.5-6, L222-L223). The heavy kernels decide occupancy by "the
+accumulator was exactly 0.0 when this product arrived" (sg_dense2.cu, sg_heavy.cu), which is exactly
+what these inputs stress.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import sginputs as gen
+from _util import compare_rows
+
+pytestmark = pytest.mark.gpu
+
+sg = pytest.importorskip("paper_conf_icpp_hardhikbrks17_b200")
+
+# path -> (thr, dense_log2): light = every row with w <= cap_L on the light kernels; rank = every
+# non-empty row heavy on the rank kernel; dense = every non-empty row heavy on the dense-window kernel
+PATHS = {"light": (4096, 62), "rank": (0, 62), "dense": (0, 0), "mixed": (256, 10)}
+
+
+@pytest.fixture
+def options():
+    old = (sg.get_option(sg.SG_OPT_DENSE_LOG2), sg.get_option(sg.SG_OPT_VARIANT))
+    yield
+    sg.set_option(sg.SG_OPT_DENSE_LOG2, old[0])
+    sg.set_option(sg.SG_OPT_VARIANT, old[1])
+
+
+def _run(A, thr):
+    dA = sg.DeviceCSR.from_host(A)
+    plan = sg.sg_symbolic(dA, dA, thr)
+    col, val = sg.sg_numeric(plan, dA, dA)
+    torch.cuda.synchronize()
+    info = plan.info()
+    out = plan.row_ptr.cpu().numpy(), col.cpu().numpy(), val.cpu().numpy()
+    plan.destroy()
+    return out, info
+
+
+@pytest.mark.parametrize("path", list(PATHS))
+@pytest.mark.parametrize("mode", ["signed", "zeros"])
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+def test_cancellation_and_stored_zeros_every_path(options, path, mode, dtype):
+    thr, dl = PATHS[path]
+    sg.set_option(sg.SG_OPT_DENSE_LOG2, dl)
+    A = gen.config("rmat13", mode=mode, dtype=dtype)
+    (rp, col, val), info = _run(A, thr)
+    R = oracle.spgemm(A, A)
+    assert np.array_equal(rp, R.row_ptr)
+    compare_rows(rp, col, val, R, dtype, exact_values=True)
+    assert int((R.val == 0).sum()) > 0, "fixture must contain structural zeros"
+    if path == "dense":
+        assert info["n_dense"] == info["n_heavy"] > 0
+    if path == "rank":
+        assert info["n_dense"] == 0 and info["n_heavy"] > 0
+
+
+@pytest.mark.parametrize("variant", [0, 1])
+def test_cancellation_dense_kernel_variants(options, variant):
+    """Both dense-window kernels (SG_OPT_VARIANT 0: sg_dense2.cu, 1: sg_dense.cu) on multi-chunk rows
+    (more than 1024 k entries at R-MAT 16) with signed values: bit-exact."""
+    sg.set_option(sg.SG_OPT_VARIANT, variant)
+    sg.set_option(sg.SG_OPT_DENSE_LOG2, 0)
+    A = gen.config("rmat16", mode="signed")
+    assert int(np.diff(A.row_ptr).max()) > 1024
+    (rp, col, val), info = _run(A, 1024)
+    R = oracle.spgemm(A, A)
+    assert np.array_equal(rp, R.row_ptr)
+    compare_rows(rp, col, val, R, "f64", exact_values=True)
+    assert info["n_dense"] > 0
+
+
+@pytest.mark.parametrize("mode", ["signed", "zeros"])
+def test_sorted_light_path_with_cancellation(mode):
+    """Un-permuted R-MAT (column-skewed light rows take the uniform-hash + bitonic-sort path)."""
+    A = gen.rmat(14, permute=False, mode=mode)
+    (rp, col, val), info = _run(A, 4096)
+    R = oracle.spgemm(A, A)
+    compare_rows(rp, col, val, R, "f64", exact_values=True)
+    assert info["n_light_sorted"] > 0
+
+
+def test_all_zero_values_keep_full_structure(options):
+    """Every stored value 0: C's values are all 0 and its structure is the full boolean product."""
+    A = gen.config("rmat12")
+    Z = gen.CSR(A.nrows, A.ncols, A.row_ptr, A.col, np.zeros_like(A.val), "zeros")
+    for thr, dl in PATHS.values():
+        sg.set_option(sg.SG_OPT_DENSE_LOG2, dl)
+        (rp, col, val), _ = _run(Z, thr)
+        R = oracle.spgemm(A, A)
+        assert np.array_equal(rp, R.row_ptr) and np.array_equal(col, R.col)
+        assert not val.any()
+
+
+def test_negative_zero_products_are_structural(options):
+    """-0.0 inputs: products are +-0.0, every entry exists and compares equal to 0."""
+    A = gen.config("C1")
+    N = gen.CSR(A.nrows, A.ncols, A.row_ptr, A.col, np.full_like(A.val, -0.0), "negzero")
+    for thr, dl in PATHS.values():
+        sg.set_option(sg.SG_OPT_DENSE_LOG2, dl)
+        (rp, col, val), _ = _run(N, thr)
+        R = oracle.spgemm(A, A)
+        assert np.array_equal(rp, R.row_ptr) and np.array_equal(col, R.col)
+        assert np.all(val == 0)

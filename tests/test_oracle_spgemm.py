@@ -209,3 +209,45 @@ def test_work_is_spmv_with_row_counts():
     pat = A.to_scipy().copy()
     pat.data[:] = 1.0
     assert np.array_equal((pat @ VB).astype(np.int64), w)
+
+
+def _struct_dense(A):
+    d = np.zeros((A.nrows, A.ncols), dtype=np.int64)
+    for i in range(A.nrows):
+        d[i, A.col[A.row_ptr[i]:A.row_ptr[i + 1]]] = 1
+    return d
+
+
+@pytest.mark.parametrize("mode", ["signed", "zeros"])
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_structural_zeros_and_exact_cancellation(mode, seed):
+    """Reading R9 (structural semantics): C has an entry wherever a product exists, kept when its
+    value is 0 — by exact cancellation (signed integers) or from explicitly stored zeros. Structure
+    = boolean product of the STORED patterns; values = the dense integer product, bit-exact."""
+    A = gen.random_pattern(48, 40, 0.15, seed, mode)
+    B = gen.random_pattern(40, 56, 0.15, seed + 50, mode)
+    R = oracle.spgemm(A, B)
+    _assert_canonical(R)
+    pat = _struct_dense(A) @ _struct_dense(B) > 0
+    assert np.array_equal(_pattern_of(R, 48, 56), pat)
+    assert np.array_equal(_dense_of(R, 48, 56), A.to_dense() @ B.to_dense())
+    zeros = int((R.val == 0).sum())
+    assert zeros > 0, "the fixture must produce structural zeros"
+    assert R.nnz == int(pat.sum())
+
+
+@pytest.mark.parametrize("name", ["C1", "rmat11"])
+def test_moments_digest_vs_scipy_structure(name):
+    """oracle.moments (per-row u, sum c, c^2, c^3 mod 2^64; the structure digest the C3 parity test
+    uses) equals the same sums over scipy.sparse's A@A pattern (an independent SpGEMM)."""
+    A = gen.config(name)
+    S = A.to_scipy()
+    P = (S @ S).tocsr()
+    P.sort_indices()
+    m = oracle.moments(A, A)
+    for i in range(A.nrows):
+        c = P.indices[P.indptr[i]:P.indptr[i + 1]].astype(np.uint64)
+        assert int(m[i, 0]) == len(c)
+        assert m[i, 1] == c.sum(dtype=np.uint64)
+        assert m[i, 2] == (c * c).sum(dtype=np.uint64)
+        assert m[i, 3] == (c * c * c).sum(dtype=np.uint64)
