@@ -301,6 +301,58 @@ __global__ void __launch_bounds__(D2_T, 1) k_num_dense2(
             D2_MARK(1);
             __syncthreads();  // window t accumulated
             D2_MARK(2);
+#ifndef SG_D2_EMIT
+#define SG_D2_EMIT 1
+#endif
+#if SG_D2_EMIT
+            // ---- emission, coalesced: warp w owns bitmap words [24w, 24w + 24) (768 columns); a warp scan
+            // of their popcounts and one exchange of warp totals place its entries; then output positions
+            // p = 32 r + lane are written by lane (word found by a 5-step shuffle search, bit by a popc
+            // bisection), so every store instruction covers 32 consecutive C entries (ncu: the
+            // per-thread scattered emission was 25 % of the kernel, profiles/r02_dense2_phases.txt) ----
+            static_assert(D2_WORDS == 24 * D2_NW, "emission: 24 bitmap words per warp");
+            const int wbase = 24 * wid;
+            const uint32_t wv = lane < 24 ? S.bm[wbase + lane] : 0u;
+            const int pcw = __popc(wv);
+            const int incl = warp_incl_scan(pcw);
+            const int excl = incl - pcw;
+            const int wt = __shfl_sync(FULL, incl, 31);
+            if (lane == 0) S.ws[wid] = wt;
+            __syncthreads();  // warp totals published; every bitmap word read
+            const int xw = S.ws[lane];
+            const int xi = warp_incl_scan(xw);
+            const int woff = __shfl_sync(FULL, xi - xw, wid);
+            const int wtot = __shfl_sync(FULL, xi, 31);
+            if (lane < 24) S.bm[wbase + lane] = 0u;
+            for (int p0 = 0; p0 < wt; p0 += 32) {
+                const int pp = p0 + lane;
+                int sw = 0;  // largest word index with excl <= pp (lanes >= 24 hold excl = wt > pp)
+                #pragma unroll
+                for (int b = 16; b; b >>= 1) {
+                    const int e2 = __shfl_sync(FULL, excl, sw + b);
+                    if (e2 <= pp) sw += b;
+                }
+                uint32_t x = __shfl_sync(FULL, wv, sw);
+                int k = pp - __shfl_sync(FULL, excl, sw);
+                if (pp < wt) {
+                    int bit = 0, c;  // k-th set bit of x (0-based)
+                    c = __popc(x & 0xFFFFu); if (k >= c) { k -= c; bit += 16; x >>= 16; }
+                    c = __popc(x & 0xFFu);   if (k >= c) { k -= c; bit += 8;  x >>= 8; }
+                    c = __popc(x & 0xFu);    if (k >= c) { k -= c; bit += 4;  x >>= 4; }
+                    c = __popc(x & 0x3u);    if (k >= c) { k -= c; bit += 2;  x >>= 2; }
+                    if (k >= (int)(x & 1u)) bit += 1;
+                    const int e = 32 * (wbase + sw) + bit;
+                    const int64_t at = pos + woff + pp;
+#if SG_D2_EXP == 4 || SG_D2_EXP == 5  // timing experiment: emission without the global stores (wrong C)
+                    if (S.vals[e] == 1234.5) st_out(C_col + at, (int32_t)(lo + e));
+#else
+                    st_out(C_col + at, (int32_t)(lo + e));
+                    st_out(C_val + at, (VT)S.vals[e]);
+#endif
+                    S.vals[e] = 0.0;
+                }
+            }
+#else
             // ---- emission: thread tid owns columns [D2_CPT*tid, +D2_CPT) of the window; one block scan of
             // their popcounts places every run; each thread writes its set bits in column order ----
             uint32_t hwb;
@@ -319,16 +371,13 @@ __global__ void __launch_bounds__(D2_T, 1) k_num_dense2(
                 while (m) {
                     const int e = ebase + __ffs(m) - 1;
                     m &= m - 1u;
-#if SG_D2_EXP == 4 || SG_D2_EXP == 5  // timing experiment: emission without the global stores (wrong C)
-                    if (S.vals[e] == 1234.5) st_out(C_col + at, (int32_t)(lo + e));
-#else
                     st_out(C_col + at, (int32_t)(lo + e));
                     st_out(C_val + at, (VT)S.vals[e]);
-#endif
                     S.vals[e] = 0.0;
                     ++at;
                 }
             }
+#endif
             pos += wtot;
             D2_MARK(3);
             __syncthreads();  // clears (and ws) ordered before the next window's products / scans

@@ -18,6 +18,7 @@
 // Per-k cursors advance monotonically across ranges; B rows longer than LONG_ROW locate their
 // segment through the tile-pointer table tp (one load), short rows by a bounded scan.
 #include "sg_device.cuh"
+#include <cstdio>
 
 namespace sg {
 
@@ -385,6 +386,13 @@ __device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.w
 __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 __device__ __forceinline__ void fence_proxy_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 
+#if defined(SG_HV_EXP) && SG_HV_EXP == 8  // timing experiment: per-phase cycle counters (lane 0 of each warp)
+__device__ unsigned long long g_hv_phase[10];
+#define HV_MARK(k) do { if ((threadIdx.x & 31) == 0) { long long _t = clock64(); hph[k] += _t - hv_last; hv_last = _t; } } while (0)
+#else
+#define HV_MARK(k) do { } while (0)
+#endif
+
 template <class VT>
 __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
     Mat A, Mat B, const int32_t* __restrict__ heavy, int64_t h0, int64_t nheavy, int64_t rb, const int64_t* __restrict__ range_off,
@@ -407,12 +415,17 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
 #endif
     constexpr bool kBulk = SG_BULK && sizeof(VT) == 8;  // fp64 output: accumulator copied out by bulk async copy
     int clear_n = 0;                          // accumulator entries still to be cleared (bulk path)
+#if defined(SG_HV_EXP) && SG_HV_EXP == 8
+    unsigned long long hph[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
+    long long hv_last = clock64();
+#endif
     while (true) {
         if (tid == 0) s_j = h0 + (long long)atomicAdd(counter, 1ull);
         __syncthreads();
         const int64_t h = s_j;
         __syncthreads();
         if (h >= nheavy) break;
+        HV_MARK(6);
         const int64_t li = heavy[h];
         const int64_t row = rb + li;
         const int64_t s0 = __ldg(A.rp + row), s1 = __ldg(A.rp + row + 1);
@@ -436,6 +449,10 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
             }
         }
         __syncthreads();
+        HV_MARK(0);
+#if defined(SG_HV_EXP) && SG_HV_EXP == 8
+        if (threadIdx.x == 0) { hph[8] += nr; }
+#endif
         RangeRec Rn;  // next range's record, loaded one range ahead
         if (nr > 0) Rn = rr[0];
         for (int ri = 0; ri < nr; ++ri) {
@@ -470,6 +487,10 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 }
                 int nk;
                 const int ctot = chunk_compact<NUM_T, int32_t>(len, beg, a, S.s_beg, S.s_off, S.s_a, &nk, S.wsll);
+                HV_MARK(1);
+#if defined(SG_HV_EXP) && SG_HV_EXP == 8
+                if (threadIdx.x == 0) hph[9] += ctot;
+#endif
                 const uint32_t bb = opaque_u32(a_bm - 4u * ((uint32_t)lo >> 5));  // &bm[(c - lo) >> 5] = bb + 4(c >> 5)
                 auto setbit = [&](int32_t c, double) {
                     if (c >= 0) red_or_s(bb + 4u * ((uint32_t)c >> 5), 1u << (c & 31));
@@ -493,6 +514,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 if (!single) __syncthreads();
             }
             __syncthreads();
+            HV_MARK(2);
             // ---- rank prefix over the range's words: thread t owns words [8t, 8t+8) (two 128-bit
             // loads, a sequential local prefix, one block scan, one 128-bit store of 8 uint16) ----
             {
@@ -518,6 +540,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 reinterpret_cast<uint4*>(S.pref)[tid] = o;  // words >= nwords are zero: harmless prefixes
             }
             __syncthreads();
+            HV_MARK(3);
             // ---- pass 2: every product accumulated at rank(c); the column is written on first arrival ----
             const int64_t base = crow + R.off;
             // vals[e + sh] and C_val[base + e] share 16 B alignment: sh from the ADDRESS (C_val is 8 B aligned,
@@ -560,6 +583,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
             }
             if (kBulk) fence_proxy_async_smem();  // accumulator writes visible to the bulk copy
             __syncthreads();
+            HV_MARK(4);
             // ---- values by rank; bitmap cleared for the next range ----
             const int cnt = R.cnt;
             if constexpr (kBulk) {
@@ -583,11 +607,16 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 bm4[2 * tid] = make_uint4(0, 0, 0, 0);
                 bm4[2 * tid + 1] = make_uint4(0, 0, 0, 0);
             }
+            HV_MARK(5);
             // no barrier here: the next range's first reads of the cleared bitmap / accumulator and its
             // rewrite of the packed chunk arrays all come after chunk_compact's barriers
         }
     }
     if (kBulk && tid == 0) bulk_wait_all();
+#if defined(SG_HV_EXP) && SG_HV_EXP == 8
+    if ((threadIdx.x & 31) == 0)
+        for (int k = 0; k < 10; ++k) atomicAdd(&g_hv_phase[k], hph[k]);
+#endif
 }
 
 cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, int64_t h0, int64_t nheavy, int64_t rb,
@@ -611,6 +640,19 @@ cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, i
                                         A, B, heavy, h0, nheavy, rb, range_off, nranges, ranges, long_id, tp, T, C_rp, C_col,
                                         (float*)C_val, counter, gscr, amax)));
     }
+#if defined(SG_HV_EXP) && SG_HV_EXP == 8
+    {
+        unsigned long long hh[10] = {0};
+        cudaStreamSynchronize(s);
+        cudaMemcpyFromSymbol(hh, g_hv_phase, sizeof(hh));
+        fprintf(stderr, "[rank phases, Gcycles summed over warps] row-setup %.2f seg+compact %.2f pass1 %.2f prefix %.2f "
+                "pass2 %.2f emit %.2f fetch %.2f | ranges %llu products %llu (thread-0 counts)\n",
+                hh[0] / 1e9, hh[1] / 1e9, hh[2] / 1e9, hh[3] / 1e9, hh[4] / 1e9, hh[5] / 1e9, hh[6] / 1e9,
+                hh[8], hh[9]);
+        unsigned long long z[10] = {0};
+        cudaMemcpyToSymbol(g_hv_phase, z, sizeof(z));
+    }
+#endif
     return cudaGetLastError();
 }
 
