@@ -39,6 +39,7 @@ struct sg_plan {
     int2* span = nullptr;           // light rows: [cmin, cmax] of the output columns
     int4* gscr = nullptr;           // heavy rows with more than KC entries: per-k cursor scratch
     void* pscr = nullptr;           // dense2: per-CTA part scratch for rows with many k entries
+    void* rscr = nullptr;           // rank2: per-CTA part scratch
     int64_t pscr_cap = 0;
     int variant = 0;
     int32_t* long_id = nullptr;
@@ -115,6 +116,11 @@ void init_options() {
         e = getenv("SG_DW_LOG2");
         if (e && *e) g_opt[SG_OPT_DENSE_LOG2] = atoll(e);
     });
+}
+
+int variant_bits() {
+    init_options();
+    return (int)g_opt[SG_OPT_VARIANT].load();
 }
 
 bool env_validate() {
@@ -231,10 +237,24 @@ sg_status row_stats(const Mat& A, const Mat& B, const int64_t* rows, int64_t nr,
     CK(launch_bin_scatter(rs.w, nr, cap, dbin + NBINS, lists, s));
     for (int b = 0; b < NBIN_LIGHT; ++b)
         CK(launch_sym_light(b, A, B, lists + off[b], cnt[b], rows, 0, rs.u, nullptr, nullptr, s));
-    unsigned long long* counter = (unsigned long long*)sc.get(sizeof(unsigned long long));
+    unsigned long long* counter = (unsigned long long*)sc.get(2 * sizeof(unsigned long long));
     if (!counter) return SG_ERR_OOM;
-    CK(launch_sym_heavy(A, B, lists + off[BIN_HEAVY], cnt[BIN_HEAVY], rows, 0, rs.u, nullptr, nullptr, nullptr,
-                        0, nullptr, nullptr, nullptr, 0, counter, s, cnt[BIN_HEAVY]));
+    if (cnt[BIN_HEAVY] == 0) return SG_OK;
+    if (variant_bits() & 2) {
+        CK(launch_sym_heavy(A, B, lists + off[BIN_HEAVY], cnt[BIN_HEAVY], rows, 0, rs.u, nullptr, nullptr, nullptr,
+                            0, nullptr, nullptr, nullptr, 0, counter, s, cnt[BIN_HEAVY]));
+        return SG_OK;
+    }
+    // largest a over the listed rows: part scratch of the lean symbolic (sg_sym2.cu)
+    unsigned long long amax = 0;
+    CK(launch_max_i64(rs.a, nr, counter + 1, s));
+    CK(cudaMemcpyAsync(&amax, counter + 1, sizeof(amax), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    const int64_t np = sym2_scratch_parts((int64_t)amax);
+    void* pscr = np > 0 ? sc.get(part_bytes() * (size_t)np) : nullptr;
+    if (np > 0 && !pscr) return SG_ERR_OOM;
+    CK(launch_sym_heavy2(A, B, lists + off[BIN_HEAVY], cnt[BIN_HEAVY], rows, 0, rs.w, rs.u, nullptr, nullptr, nullptr,
+                         0, nullptr, nullptr, nullptr, 0, counter, s, cnt[BIN_HEAVY], pscr, (int64_t)amax));
     return SG_OK;
 }
 
@@ -319,7 +339,7 @@ sg_status sg_set_option(int key, int64_t value) {
     if (key < 0 || key >= SG_OPT_COUNT) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_VALIDATE && value != 0 && value != 1) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_DENSE_LOG2 && (value < -1 || value > 62)) return SG_ERR_INVALID_ARG;
-    if (key == SG_OPT_VARIANT && (value < 0 || value > 1)) return SG_ERR_INVALID_ARG;
+    if (key == SG_OPT_VARIANT && (value < 0 || value > 7)) return SG_ERR_INVALID_ARG;
     g_opt[key] = value;
     return SG_OK;
 }
@@ -594,6 +614,7 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
     if (row_begin < 0 || row_end < row_begin || row_end > A->nrows) return SG_ERR_INVALID_ARG;
     sg_plan* pl = new sg_plan();
     pl->s = s;
+    pl->variant = variant_bits();
     pl->rb = row_begin; pl->re = row_end; pl->nr = row_end - row_begin; pl->thr = thr;
     pl->p = B->ncols; pl->m = B->nrows; pl->dt = (int)A->dtype;
     pl->C_rp = C_row_ptr;
@@ -675,11 +696,14 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
         pl->ranges = (RangeRec*)palloc(pl, sizeof(RangeRec) * (size_t)(pl->nslots > 0 ? pl->nslots : 1));
         pl->tp = (uint32_t*)palloc(pl, 4 * (size_t)(pl->nlong > 0 ? pl->nlong : 1) * (size_t)(pl->T + 1));
         if (!pl->ranges || !pl->tp) return fail(SG_ERR_OOM);
-        pl->variant = (int)g_opt[SG_OPT_VARIANT].load();
         if (pl->ndw > 0 && pl->amax + 32 > dense2_pcap()) {
             pl->pscr_cap = pl->amax + 32;
             pl->pscr = palloc(pl, dense2_part_bytes() * (size_t)pl->pscr_cap * 148);
             if (!pl->pscr) return fail(SG_ERR_OOM);
+        }
+        if (rank2_scratch_bytes(pl->amax) > 0) {
+            pl->rscr = palloc(pl, rank2_scratch_bytes(pl->amax));
+            if (!pl->rscr) return fail(SG_ERR_OOM);
         }
         if (pl->amax > heavy_kc() || pl->amax > dense_kc()) {
             pl->gscr = (int4*)palloc(pl, sizeof(int4) * (size_t)(heavy_grid() > dense_grid() ? heavy_grid() : dense_grid()) * (size_t)pl->amax);
@@ -691,9 +715,18 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
     for (int k = 0; k < NBIN_LIGHT; ++k)
         CKF(launch_sym_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], nullptr, row_begin, pl->u, pl->span,
                              (unsigned long long*)(pl->dbin + 2 * NBINS + 1), s));
-    CKF(launch_sym_heavy(a, b, pl->heavy, pl->nheavy, nullptr, row_begin, pl->u, pl->range_off, pl->ranges,
-                         pl->nranges, pl->ndw, pl->dtc, pl->long_id, pl->nlong > 0 ? pl->tp : nullptr, pl->T,
-                         pl->counter, s, pl->nbig));
+    if (pl->variant & 2) {
+        CKF(launch_sym_heavy(a, b, pl->heavy, pl->nheavy, nullptr, row_begin, pl->u, pl->range_off, pl->ranges,
+                             pl->nranges, pl->ndw, pl->dtc, pl->long_id, pl->nlong > 0 ? pl->tp : nullptr, pl->T,
+                             pl->counter, s, pl->nbig));
+    } else if (pl->nheavy > 0) {
+        const int64_t np = sym2_scratch_parts(pl->amax);
+        void* pscr = np > 0 ? palloc(pl, part_bytes() * (size_t)np) : nullptr;
+        if (np > 0 && !pscr) return fail(SG_ERR_OOM);
+        CKF(launch_sym_heavy2(a, b, pl->heavy, pl->nheavy, nullptr, row_begin, pl->w, pl->u, pl->range_off, pl->ranges,
+                              pl->nranges, pl->ndw, pl->dtc, pl->long_id, pl->nlong > 0 ? pl->tp : nullptr, pl->T,
+                              pl->counter, s, pl->nbig, pscr, pl->amax));
+    }
     CKF(scan_exclusive(pl->u, C_row_ptr, nr, stmp, s));
     CKF(cudaMemcpyAsync(&pl->nnz_c, C_row_ptr + nr, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     CKF(cudaMemcpyAsync(&pl->nskew, pl->dbin + 2 * NBINS + 1, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
@@ -727,8 +760,13 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
             CKP(pl, launch_num_dense2(a, b, pl->heavy, pl->ndw, pl->rb, pl->w, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
                                       C_val, pl->counter, pl->pscr, pl->pscr_cap, pl->dtc, pl->ditems,
                                       pl->ditem_off + pl->ndw, s));
-        CKP(pl, launch_num_heavy(a, b, pl->heavy, pl->ndw, pl->nheavy, pl->rb, pl->range_off, pl->nranges, pl->ranges,
-                                 pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter, pl->gscr, pl->amax, s));
+        if (pl->variant & 4)
+            CKP(pl, launch_num_heavy(a, b, pl->heavy, pl->ndw, pl->nheavy, pl->rb, pl->range_off, pl->nranges, pl->ranges,
+                                     pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter, pl->gscr, pl->amax, s));
+        else
+            CKP(pl, launch_num_rank2(a, b, pl->heavy, pl->ndw, pl->nheavy, pl->rb, pl->w, pl->range_off, pl->nranges,
+                                     pl->ranges, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter,
+                                     pl->rscr, pl->amax, s));
     }
     if (s != pl->s) {  // the plan's workspace frees (on pl->s) wait for this call's kernels
         cudaEvent_t ev;

@@ -27,11 +27,7 @@ constexpr int D2_CPT = D2_WD / D2_T;       // columns per thread in the emission
 constexpr int D2_PCAP = 1216;              // parts held in shared memory
 static_assert(D2_CPT * D2_T == D2_WD && D2_CPT <= 32, "emission: D2_CPT columns per thread");
 
-struct D2Part {       // one warp's share of one k entry: products B_k[cur .. end) still to come
-    int32_t cur, end; // B positions
-    int32_t q0, lid;  // start of the B row; its tile-pointer id (-1: short row, <= LONG_ROW entries)
-    double a;         // a_ik
-};
+using D2Part = Part;
 
 struct D2Smem {
     double vals[D2_WD];
@@ -46,82 +42,6 @@ static_assert(sizeof(D2Smem) + 64 <= 232448, "dense2 shared memory exceeds the s
 size_t dense2_part_bytes() { return sizeof(D2Part); }
 int dense2_pcap() { return D2_PCAP; }
 
-// first warp whose slice [bw(w), bw(w+1)) holds product x (bw(w) = floor(L w / 32), x < L)
-__device__ __forceinline__ int d2_warp_of(long long x, long long L) {
-    int w = (int)((x * D2_NW) / L);
-    while (w < D2_NW - 1 && ((L * (w + 1)) >> 5) <= x) ++w;  // one step unless L < D2_NW
-    return w;
-}
-
-// Streams one warp's 32 lane-held segments (beg, len, a) through acc(c, v). Segments of >= D2_LONG
-// products are swept lane-strided, 4 batches in flight, no search; all shorter ones are flattened
-// (one warp scan of their lengths, a 5-step shuffle search per batch) and streamed D2_UNR batches at a
-// time. (A software-pipelined variant that gathers the next D2_UNR batches during the accumulation of
-// the current ones measured slower: 33.4 vs 31.7 ms on C3 rows/2, profiles/r02_dense2_ab.txt.)
-constexpr int D2_LONG = 128;
-constexpr int D2_UNR = 4;
-template <class VT, class F>
-__device__ __forceinline__ void d2_segments(const Mat& B, int beg, int len, double a, F&& acc) {
-    const int lane = threadIdx.x & 31;
-    const int32_t* __restrict__ bcol = B.col;
-    const VT* __restrict__ bval = reinterpret_cast<const VT*>(B.val);
-#if defined(SG_D2_EXP) && SG_D2_EXP == 6  // timing experiment: gathers from a 3 MB, L2-resident footprint (wrong C)
-    beg &= 0x3FFFF;
-#endif
-    unsigned lm = __ballot_sync(FULL, len >= D2_LONG);
-    while (lm) {
-        const int L = __ffs(lm) - 1;
-        lm &= lm - 1u;
-        const int b = __shfl_sync(FULL, beg, L), n = __shfl_sync(FULL, len, L);
-        const double av = __shfl_sync(FULL, a, L);
-        for (int j = lane; j < n; j += 128) {
-            int c[4];
-            double v[4];
-            #pragma unroll
-            for (int r = 0; r < 4; ++r) {
-                const int jj = j + 32 * r;
-                c[r] = -1;
-                v[r] = 0.0;
-                if (jj < n) {
-                    c[r] = __ldg(bcol + b + jj);
-                    v[r] = av * (double)__ldg(bval + b + jj);
-                }
-            }
-            #pragma unroll
-            for (int r = 0; r < 4; ++r)
-                if (c[r] >= 0) acc(c[r], v[r]);
-        }
-    }
-    const int sl = len < D2_LONG ? len : 0;
-    const int inc = warp_incl_scan(sl);
-    const int tot = __shfl_sync(FULL, inc, 31);
-    const int off = inc - sl;
-    for (int j0 = 0; j0 < tot; j0 += 32 * D2_UNR) {
-        int c[D2_UNR];
-        double v[D2_UNR];
-        #pragma unroll
-        for (int r = 0; r < D2_UNR; ++r) {
-            const int j = j0 + 32 * r + lane;
-            int s = 0;
-            #pragma unroll
-            for (int bb = 16; bb; bb >>= 1) {
-                const int o = __shfl_sync(FULL, off, s + bb);
-                if (o <= j) s += bb;
-            }
-            const int q = __shfl_sync(FULL, beg, s) + (j - __shfl_sync(FULL, off, s));
-            const double as = __shfl_sync(FULL, a, s);
-            c[r] = -1;
-            v[r] = 0.0;
-            if (j < tot) {
-                c[r] = __ldg(bcol + q);
-                v[r] = as * (double)__ldg(bval + q);
-            }
-        }
-        #pragma unroll
-        for (int r = 0; r < D2_UNR; ++r)
-            if (c[r] >= 0) acc(c[r], v[r]);
-    }
-}
 
 #if defined(SG_D2_EXP) && SG_D2_EXP == 8  // timing experiment: per-phase cycle counters (lane 0 of each warp)
 __device__ unsigned long long g_d2_phase[8];
@@ -167,7 +87,6 @@ __global__ void __launch_bounds__(D2_T, 1) k_num_dense2(
         D2Part* P = na + D2_NW <= D2_PCAP ? S.parts : pscr + (int64_t)blockIdx.x * pscr_cap;
         const int64_t lo0 = (int64_t)ta * D2_WD;
         const int tlo = min(ta * D2_TILES, T);
-        for (int w = tid; w <= D2_NW; w += D2_T) S.wpart[w] = -1;
         // output offset of window ta inside the row: the row's tile counts below tile ta*D2_TILES
         long long off0 = 0;
         if (ta > 0) {
@@ -177,65 +96,7 @@ __global__ void __launch_bounds__(D2_T, 1) k_num_dense2(
             __syncthreads();  // wsll read by every warp before the part scans rewrite it
         }
         // ---- parts: the row's products cut into D2_NW equal slices (k entries split at boundaries) ----
-        long long carry_p = 0;
-        int carry_n = 0;
-        for (int c0 = 0; c0 < na; c0 += D2_T) {
-            const int i = c0 + tid;
-            int len = 0, q0 = 0, lid = -1;
-            double a = 0.0;
-            if (i < na) {
-                const int k = __ldg(A.col + s0 + i);
-                q0 = (int)__ldg(B.rp + k);
-                len = (int)(__ldg(B.rp + k + 1) - q0);
-                a = ldv<VT>(A.val, s0 + i);
-                if (len > LONG_ROW) lid = __ldg(long_id + k);
-            }
-            long long tot;
-            const long long ex = block_scan_ll<D2_T>((long long)len, &tot, S.wsll) + carry_p;
-            int wf = 0, wl = -1;
-            if (len > 0) {
-                wf = d2_warp_of(ex, L);
-                wl = d2_warp_of(ex + len - 1, L);
-            }
-            int ntot;
-            const int po = block_scan1<D2_T, int>(wl - wf + 1, &ntot, S.ws) + carry_n;
-            if (len > 0) {
-                // first entry of the item's first window (all parts of this k share it)
-                int first = q0;
-                if (ta > 0) {
-                    if (lid >= 0) {
-                        first = q0 + (int)__ldg(tp + (int64_t)lid * (T + 1) + tlo);
-                    } else {
-                        int n0 = 0;
-                        for (int q = 0; q < len; ++q) n0 += __ldg(B.col + q0 + q) < lo0;
-                        first = q0 + n0;
-                    }
-                }
-                for (int w = wf; w <= wl; ++w) {
-                    const long long bw = (L * w) >> 5, bw1 = (L * (w + 1)) >> 5;
-                    const int lo = (int)(max(ex, bw) - ex), hi = (int)(min(ex + len, bw1) - ex);
-                    D2Part pt;
-                    pt.cur = max(q0 + lo, first);
-                    pt.end = q0 + hi;
-                    pt.q0 = q0;
-                    pt.lid = lid;
-                    pt.a = a;
-                    P[po + (w - wf)] = pt;
-                    if (bw >= ex) S.wpart[w] = po + (w - wf);  // the part holding product bw(w) starts warp w
-                }
-            }
-            carry_p += tot;
-            carry_n += ntot;
-            __syncthreads();  // ws / wsll free for the next chunk's scans
-        }
-        if (wid == 0) {  // warps without products (only when L < D2_NW) start where the next one does
-            if (lane == 0) S.wpart[D2_NW] = carry_n;
-            __syncwarp();
-            if (lane == 0)
-                for (int w = D2_NW - 1; w >= 0; --w)
-                    if (S.wpart[w] < 0) S.wpart[w] = S.wpart[w + 1];
-        }
-        __syncthreads();
+        build_parts<D2_T, VT, true>(A, B, s0, na, L, long_id, tp, T, tlo, lo0, P, S.wpart, S.wsll, S.ws);
         D2_MARK(0);
         const int pw0 = S.wpart[wid], pw1 = S.wpart[wid + 1];
         int64_t pos = C_rp[li] + off0;
@@ -296,7 +157,7 @@ __global__ void __launch_bounds__(D2_T, 1) k_num_dense2(
                 }
                 if (g == pw0 && lid0 >= 0 && t + 1 < tb)
                     tpn = __ldg(tp + (int64_t)lid0 * (T + 1) + min((t + 2) * D2_TILES, T));
-                d2_segments<VT>(B, beg, len, a, acc);
+                seg_walk<true, VT>(B, beg, len, a, acc);
             }
             D2_MARK(1);
             __syncthreads();  // window t accumulated

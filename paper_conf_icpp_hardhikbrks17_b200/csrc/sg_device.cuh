@@ -488,4 +488,166 @@ __device__ __forceinline__ int seg_end(const Mat& B, int cur, int e1, int q0, bo
     return cur + n;
 }
 
+
+// ---- per-warp product slices ("parts"; sg_dense2.cu, sg_sym2.cu) --------------------------------
+// A row's products [0, L) (L = w_i = sum of its B row lengths, in A-column order) are cut into NW
+// equal contiguous slices, one per warp; warp w owns products [bw(w), bw(w+1)), bw(w) = floor(L w/NW).
+// A PART is one warp's share of one k entry: B_k[cur .. end). Parts are ordered by (k, warp), so each
+// warp's parts are contiguous; wpart[w] = first part of warp w, wpart[NW] = number of parts (<= na + NW).
+struct Part {
+    int32_t cur, end;  // B positions still to come
+    int32_t q0, lid;   // start of the B row; its tile-pointer id (-1: short row, <= LONG_ROW entries)
+    double a;          // a_ik (0 for structure-only walks)
+};
+
+template <int NW> __device__ __forceinline__ int part_warp_of(long long x, long long L) {
+    int w = (int)((x * NW) / L);
+    while (w < NW - 1 && (L * (w + 1)) / NW <= x) ++w;  // one step unless L < NW
+    return w;
+}
+
+// Block-wide (NT threads): builds the parts of row (s0, na) into P / wpart. Cursors start at the
+// first entry with column >= lo0 (tile tlo = lo0 / TW of the tile pointers; lo0 = 0 for a whole row).
+template <int NT, class VT, bool WITH_A>
+__device__ __forceinline__ void build_parts(const Mat& A, const Mat& B, int64_t s0, int na, long long L,
+                                            const int32_t* __restrict__ long_id, const uint32_t* __restrict__ tp,
+                                            int T, int tlo, int64_t lo0, Part* P, int32_t* wpart, long long* wsll,
+                                            int* ws) {
+    constexpr int NW = NT / 32;
+    const int tid = threadIdx.x;
+    for (int w = tid; w <= NW; w += NT) wpart[w] = -1;
+    long long carry_p = 0;
+    int carry_n = 0;
+    for (int c0 = 0; c0 < na; c0 += NT) {
+        const int i = c0 + tid;
+        int len = 0, q0 = 0, lid = -1;
+        double a = 0.0;
+        if (i < na) {
+            const int k = __ldg(A.col + s0 + i);
+            q0 = (int)__ldg(B.rp + k);
+            len = (int)(__ldg(B.rp + k + 1) - q0);
+            if (WITH_A) a = ldv<VT>(A.val, s0 + i);
+            if (len > LONG_ROW && tp) lid = __ldg(long_id + k);
+        }
+        long long tot;
+        const long long ex = block_scan_ll<NT>((long long)len, &tot, wsll) + carry_p;  // (barrier inside)
+        int wf = 0, wl = -1;
+        if (len > 0) {
+            wf = part_warp_of<NW>(ex, L);
+            wl = part_warp_of<NW>(ex + len - 1, L);
+        }
+        int ntot;
+        const int po = block_scan1<NT, int>(wl - wf + 1, &ntot, ws) + carry_n;
+        if (len > 0) {
+            int first = q0;  // first entry at or after column lo0 (all parts of this k share it)
+            if (lo0 > 0) {
+                if (lid >= 0) {
+                    first = q0 + (int)__ldg(tp + (int64_t)lid * (T + 1) + tlo);
+                } else {
+                    first = (int)lower_bound_col(B.col, q0, q0 + len, lo0);
+                }
+            }
+            for (int w = wf; w <= wl; ++w) {
+                const long long bw = (L * w) / NW, bw1 = (L * (w + 1)) / NW;
+                const int lo = (int)(max(ex, bw) - ex), hi = (int)(min(ex + len, bw1) - ex);
+                Part pt;
+                pt.cur = max(q0 + lo, first);
+                pt.end = q0 + hi;
+                pt.q0 = q0;
+                pt.lid = lid;
+                pt.a = a;
+                P[po + (w - wf)] = pt;
+                if (bw >= ex) wpart[w] = po + (w - wf);  // the part holding product bw(w) starts warp w
+            }
+        }
+        carry_p += tot;
+        carry_n += ntot;
+        __syncthreads();  // ws / wsll free for the next chunk's scans
+    }
+    if (tid == 0) {  // warps without products (only when L < NW) start where the next one does
+        wpart[NW] = carry_n;
+        for (int w = NW - 1; w >= 0; --w)
+            if (wpart[w] < 0) wpart[w] = wpart[w + 1];
+    }
+    __syncthreads();
+}
+
+// The end (exclusive B position) of part P's products below column hi: the tile pointer of tile th
+// (hi = th * TW, or p) for long B rows (tv = tp[lid][th], possibly prefetched), a bounded scan for short
+// ones; never before the cursor (a part may start past this window: its slice begins mid-row).
+__device__ __forceinline__ int part_seg_end(const Mat& B, const Part& pt, uint32_t tv, int64_t hi) {
+    if (pt.lid >= 0) return max(pt.cur, min(pt.end, pt.q0 + (int)tv));
+    if (pt.end - pt.cur > LONG_ROW) return (int)lower_bound_col(B.col, pt.cur, pt.end, hi);  // no tile pointers
+    int e = pt.cur;
+    while (e < pt.end && __ldg(B.col + e) < hi) ++e;  // <= LONG_ROW entries
+    return e;
+}
+
+// Streams one warp's 32 lane-held segments (beg, len, a) through acc(c, v) (v = a * b_kj if VAL). Segments of >= SEG_LONG
+// products are swept lane-strided, 4 batches in flight, no search; all shorter ones are flattened
+// (one warp scan of their lengths, a 5-step shuffle search per batch) and streamed SEG_UNR batches at a
+// time. (sg_dense2.cu; a software-pipelined variant that gathers the next SEG_UNR batches during the accumulation of
+// the current ones measured slower: 33.4 vs 31.7 ms on C3 rows/2, profiles/r02_dense2_ab.txt.)
+constexpr int SEG_LONG = 128;
+constexpr int SEG_UNR = 4;
+template <bool VAL, class VT, class F>
+__device__ __forceinline__ void seg_walk(const Mat& B, int beg, int len, double a, F&& acc) {
+    const int lane = threadIdx.x & 31;
+    const int32_t* __restrict__ bcol = B.col;
+    const VT* __restrict__ bval = reinterpret_cast<const VT*>(B.val);
+    unsigned lm = __ballot_sync(FULL, len >= SEG_LONG);
+    while (lm) {
+        const int L = __ffs(lm) - 1;
+        lm &= lm - 1u;
+        const int b = __shfl_sync(FULL, beg, L), n = __shfl_sync(FULL, len, L);
+        const double av = __shfl_sync(FULL, a, L);
+        for (int j = lane; j < n; j += 128) {
+            int c[4];
+            double v[4];
+            #pragma unroll
+            for (int r = 0; r < 4; ++r) {
+                const int jj = j + 32 * r;
+                c[r] = -1;
+                v[r] = 0.0;
+                if (jj < n) {
+                    c[r] = __ldg(bcol + b + jj);
+                    if (VAL) v[r] = av * (double)__ldg(bval + b + jj);
+                }
+            }
+            #pragma unroll
+            for (int r = 0; r < 4; ++r)
+                if (c[r] >= 0) acc(c[r], v[r]);
+        }
+    }
+    const int sl = len < SEG_LONG ? len : 0;
+    const int inc = warp_incl_scan(sl);
+    const int tot = __shfl_sync(FULL, inc, 31);
+    const int off = inc - sl;
+    for (int j0 = 0; j0 < tot; j0 += 32 * SEG_UNR) {
+        int c[SEG_UNR];
+        double v[SEG_UNR];
+        #pragma unroll
+        for (int r = 0; r < SEG_UNR; ++r) {
+            const int j = j0 + 32 * r + lane;
+            int s = 0;
+            #pragma unroll
+            for (int bb = 16; bb; bb >>= 1) {
+                const int o = __shfl_sync(FULL, off, s + bb);
+                if (o <= j) s += bb;
+            }
+            const int q = __shfl_sync(FULL, beg, s) + (j - __shfl_sync(FULL, off, s));
+            const double as = __shfl_sync(FULL, a, s);
+            c[r] = -1;
+            v[r] = 0.0;
+            if (j < tot) {
+                c[r] = __ldg(bcol + q);
+                if (VAL) v[r] = as * (double)__ldg(bval + q);
+            }
+        }
+        #pragma unroll
+        for (int r = 0; r < SEG_UNR; ++r)
+            if (c[r] >= 0) acc(c[r], v[r]);
+    }
+}
+
 }  // namespace sg

@@ -25,22 +25,8 @@ namespace sg {
 #ifndef SG_INREG
 #define SG_INREG 1
 #endif
-#ifndef SG_NUM_T
-#define SG_NUM_T 512
-#endif
-#ifndef SG_NUM_OCC
-#define SG_NUM_OCC 2
-#endif
-#ifndef SG_RCAP
-#define SG_RCAP 8192
-#endif
-constexpr int NUM_T = SG_NUM_T;       // numeric: threads per CTA
-constexpr int NUM_OCC = SG_NUM_OCC;   // numeric CTAs per SM (smem-bound)
 constexpr int KC = NUM_T;             // numeric k entries per chunk: one per thread
-constexpr int RW_TILES = NUM_T / 32;  // max tiles per numeric range (16 -> 128K columns, 16 KB bitmap)
 constexpr int RW_WORDS = RW_TILES * TW / 32;   // = 256 words per warp in the rank prefix
-constexpr int RCAP = SG_RCAP;         // max entries per numeric range (fp64 accumulator 64 KB)
-constexpr int RHALF = RCAP / 2;       // range key granularity (a range = run of tiles with equal key)
 static_assert(TW <= RCAP, "a single full tile must fit the numeric accumulator");
 
 // ------------------------------------------------------------------------------------------------

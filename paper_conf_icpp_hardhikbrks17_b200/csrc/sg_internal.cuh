@@ -35,6 +35,21 @@ constexpr int LONG_ROW = 8;       // B rows longer than this get per-tile pointe
 #ifndef SG_SYM_OCC
 #define SG_SYM_OCC 6
 #endif
+// rank-kernel (heavy numeric, sg_heavy.cu) geometry; the symbolic range plan depends on it
+#ifndef SG_NUM_T
+#define SG_NUM_T 512
+#endif
+#ifndef SG_NUM_OCC
+#define SG_NUM_OCC 2
+#endif
+#ifndef SG_RCAP
+#define SG_RCAP 8192
+#endif
+constexpr int NUM_T = SG_NUM_T;       // rank numeric: threads per CTA
+constexpr int NUM_OCC = SG_NUM_OCC;   // rank numeric CTAs per SM (smem-bound)
+constexpr int RW_TILES = NUM_T / 32;  // max tiles per numeric range (16 -> 128K columns, 16 KB bitmap)
+constexpr int RCAP = SG_RCAP;         // max entries per numeric range (fp64 accumulator 64 KB)
+constexpr int RHALF = RCAP / 2;       // range key granularity (a range = run of tiles with equal key)
 constexpr int WIN = 1 << SG_SYM_WIN_LOG2;  // heavy symbolic bitmap window (columns); WIN/8 bytes of smem
 constexpr int HEAVY_THREADS = SG_SYM_T;    // heavy symbolic threads per CTA
 constexpr int SYM_OCC = SG_SYM_OCC;        // heavy symbolic CTAs per SM
@@ -96,10 +111,25 @@ cudaError_t launch_sym_heavy(const Mat& A, const Mat& B, const int32_t* list, in
                              int64_t ndw, int32_t* dtc /*ndw x T tile counts, nullable*/, const int32_t* long_id /*nullable*/,
                              const uint32_t* tp /*nullable: binary search*/, int T, unsigned long long* counter,
                              cudaStream_t s, int64_t nbig /*rows [0, nbig) on the 1024-thread kernel*/);
+// lean heavy symbolic (sg_sym2.cu): same outputs as launch_sym_heavy; w = row work indexed like u;
+// pscr: sym2_scratch_parts(amax) Part records for rows of more than a few hundred k entries
+cudaError_t launch_sym_heavy2(const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, const int64_t* rowmap,
+                              int64_t rb, const int64_t* w, int64_t* u, const int64_t* range_off, RangeRec* ranges,
+                              int32_t* nranges, int64_t ndw, int32_t* dtc, const int32_t* long_id, const uint32_t* tp, int T,
+                              unsigned long long* counter, cudaStream_t s, int64_t nbig, void* pscr, int64_t amax);
+int64_t sym2_scratch_parts(int64_t amax);
+// lean rank numeric (sg_rank2.cu): same C as launch_num_heavy; pscr: rank2_scratch_bytes(amax) bytes
+cudaError_t launch_num_rank2(const Mat& A, const Mat& B, const int32_t* heavy, int64_t h0, int64_t nheavy, int64_t rb,
+                             const int64_t* w, const int64_t* range_off, const int32_t* nranges, const RangeRec* ranges,
+                             const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
+                             void* C_val, unsigned long long* counter, void* pscr, int64_t amax, cudaStream_t s);
+size_t rank2_scratch_bytes(int64_t amax);
+size_t part_bytes();
 cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, int64_t h0, int64_t nheavy, int64_t rb,
                              const int64_t* range_off, const int32_t* nranges, const RangeRec* ranges,
                              const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
                              void* C_val, unsigned long long* counter, int4* gscr, int64_t amax, cudaStream_t s);
+cudaError_t launch_max_i64(const int64_t* x, int64_t n, unsigned long long* out /*zeroed here*/, cudaStream_t s);
 cudaError_t launch_max_a(const Mat& A, const int32_t* list, int64_t cnt, int64_t rb, unsigned long long* out,
                          cudaStream_t s);
 // dense-window heavy rows (sg_dense.cu): heavy[0, ndw), all with w >= 2^dense_window_log2(p)

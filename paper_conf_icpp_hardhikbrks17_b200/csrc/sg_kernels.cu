@@ -74,6 +74,25 @@ cudaError_t launch_row_work_list(const Mat& A, const Mat& B, const int64_t* rows
     return cudaGetLastError();
 }
 
+// max of x[0..n) (non-negative values) into *out (zeroed by the caller)
+__global__ void k_max_i64(const int64_t* __restrict__ x, int64_t n, unsigned long long* out) {
+    unsigned long long m = 0;
+    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x) {
+        const unsigned long long v = (unsigned long long)x[j];
+        m = v > m ? v : m;
+    }
+    #pragma unroll
+    for (int o = 16; o; o >>= 1) { const unsigned long long y = __shfl_xor_sync(FULL, m, o); m = y > m ? y : m; }
+    if ((threadIdx.x & 31) == 0 && m) atomicMax(out, m);
+}
+
+cudaError_t launch_max_i64(const int64_t* x, int64_t n, unsigned long long* out, cudaStream_t s) {
+    cudaError_t e = cudaMemsetAsync(out, 0, sizeof(unsigned long long), s);
+    if (e != cudaSuccess || n <= 0) return e;
+    SG_LAUNCH("k_max_i64", s, k_max_i64<<<grid_for(n, 1024, 148 * 4), 256, 0, s>>>(x, n, out));
+    return cudaGetLastError();
+}
+
 // ------------------------------------------------------------------------------------------------
 // a2: exclusive scan (int64), three kernels per level, recursive over block sums
 // ------------------------------------------------------------------------------------------------
