@@ -39,7 +39,6 @@ struct sg_plan {
     int2* span = nullptr;           // light rows: [cmin, cmax] of the output columns
     int4* gscr = nullptr;           // heavy rows with more than KC entries: per-k cursor scratch
     void* pscr = nullptr;           // dense2: per-CTA part scratch for rows with many k entries
-    void* rscr = nullptr;           // rank2: per-CTA part scratch
     int64_t pscr_cap = 0;
     int variant = 0;
     int32_t* long_id = nullptr;
@@ -339,7 +338,7 @@ sg_status sg_set_option(int key, int64_t value) {
     if (key < 0 || key >= SG_OPT_COUNT) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_VALIDATE && value != 0 && value != 1) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_DENSE_LOG2 && (value < -1 || value > 62)) return SG_ERR_INVALID_ARG;
-    if (key == SG_OPT_VARIANT && (value < 0 || value > 7)) return SG_ERR_INVALID_ARG;
+    if (key == SG_OPT_VARIANT && (value < 0 || value > 3)) return SG_ERR_INVALID_ARG;
     g_opt[key] = value;
     return SG_OK;
 }
@@ -701,10 +700,6 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
             pl->pscr = palloc(pl, dense2_part_bytes() * (size_t)pl->pscr_cap * 148);
             if (!pl->pscr) return fail(SG_ERR_OOM);
         }
-        if (rank2_scratch_bytes(pl->amax) > 0) {
-            pl->rscr = palloc(pl, rank2_scratch_bytes(pl->amax));
-            if (!pl->rscr) return fail(SG_ERR_OOM);
-        }
         if (pl->amax > heavy_kc() || pl->amax > dense_kc()) {
             pl->gscr = (int4*)palloc(pl, sizeof(int4) * (size_t)(heavy_grid() > dense_grid() ? heavy_grid() : dense_grid()) * (size_t)pl->amax);
             if (!pl->gscr) return fail(SG_ERR_OOM);
@@ -760,13 +755,8 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
             CKP(pl, launch_num_dense2(a, b, pl->heavy, pl->ndw, pl->rb, pl->w, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
                                       C_val, pl->counter, pl->pscr, pl->pscr_cap, pl->dtc, pl->ditems,
                                       pl->ditem_off + pl->ndw, s));
-        if (pl->variant & 4)
-            CKP(pl, launch_num_heavy(a, b, pl->heavy, pl->ndw, pl->nheavy, pl->rb, pl->range_off, pl->nranges, pl->ranges,
-                                     pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter, pl->gscr, pl->amax, s));
-        else
-            CKP(pl, launch_num_rank2(a, b, pl->heavy, pl->ndw, pl->nheavy, pl->rb, pl->w, pl->range_off, pl->nranges,
-                                     pl->ranges, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter,
-                                     pl->rscr, pl->amax, s));
+        CKP(pl, launch_num_heavy(a, b, pl->heavy, pl->ndw, pl->nheavy, pl->rb, pl->range_off, pl->nranges, pl->ranges,
+                                 pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter, pl->gscr, pl->amax, s));
     }
     if (s != pl->s) {  // the plan's workspace frees (on pl->s) wait for this call's kernels
         cudaEvent_t ev;

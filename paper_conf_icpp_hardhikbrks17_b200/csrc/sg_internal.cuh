@@ -118,12 +118,6 @@ cudaError_t launch_sym_heavy2(const Mat& A, const Mat& B, const int32_t* list, i
                               int32_t* nranges, int64_t ndw, int32_t* dtc, const int32_t* long_id, const uint32_t* tp, int T,
                               unsigned long long* counter, cudaStream_t s, int64_t nbig, void* pscr, int64_t amax);
 int64_t sym2_scratch_parts(int64_t amax);
-// lean rank numeric (sg_rank2.cu): same C as launch_num_heavy; pscr: rank2_scratch_bytes(amax) bytes
-cudaError_t launch_num_rank2(const Mat& A, const Mat& B, const int32_t* heavy, int64_t h0, int64_t nheavy, int64_t rb,
-                             const int64_t* w, const int64_t* range_off, const int32_t* nranges, const RangeRec* ranges,
-                             const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
-                             void* C_val, unsigned long long* counter, void* pscr, int64_t amax, cudaStream_t s);
-size_t rank2_scratch_bytes(int64_t amax);
 size_t part_bytes();
 cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, int64_t h0, int64_t nheavy, int64_t rb,
                              const int64_t* range_off, const int32_t* nranges, const RangeRec* ranges,
