@@ -208,7 +208,7 @@ sg_status row_stats(const Mat& A, const Mat& B, const int64_t* rows, int64_t nr,
     rs.a = (int64_t*)sc.get(sizeof(int64_t) * (size_t)nr);
     rs.u = (int64_t*)sc.get(sizeof(int64_t) * (size_t)nr);
     int32_t* lists = (int32_t*)sc.get(sizeof(int32_t) * (size_t)nr);
-    int64_t* dbin = (int64_t*)sc.get(sizeof(int64_t) * 2 * NBINS);
+    int64_t* dbin = (int64_t*)sc.get(sizeof(int64_t) * (2 * NBINS + 1));
     int64_t* all_rows = nullptr;
     if (!rs.w || !rs.a || !rs.u || !lists || !dbin) return SG_ERR_OOM;
     if (!rows) {
@@ -224,11 +224,15 @@ sg_status row_stats(const Mat& A, const Mat& B, const int64_t* rows, int64_t nr,
     }
     CK(launch_row_work_list(A, B, rows, nr, rs.w, rs.a, s));
     CK(cudaMemsetAsync(rs.u, 0, sizeof(int64_t) * (size_t)nr, s));
-    CK(cudaMemsetAsync(dbin, 0, sizeof(int64_t) * 2 * NBINS, s));
+    CK(cudaMemsetAsync(dbin, 0, sizeof(int64_t) * (2 * NBINS + 1), s));
     CK(launch_bin_count(rs.w, nr, cap, dbin, nullptr, s));
-    int64_t cnt[NBINS];
+    // largest a over the listed rows (part scratch of the lean symbolic, sg_sym2.cu), read back with the
+    // bin counts in ONE copy + sync
+    CK(launch_max_i64(rs.a, nr, (unsigned long long*)(dbin + NBINS), s));
+    int64_t cnt[NBINS + 1];
     CK(cudaMemcpyAsync(cnt, dbin, sizeof(cnt), cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
+    const int64_t amax = cnt[NBINS];
     int64_t off[NBINS + 1];
     off[0] = 0;
     for (int b = 0; b < NBINS; ++b) off[b + 1] = off[b] + cnt[b];
@@ -244,16 +248,11 @@ sg_status row_stats(const Mat& A, const Mat& B, const int64_t* rows, int64_t nr,
                             0, nullptr, nullptr, nullptr, 0, counter, s, cnt[BIN_HEAVY]));
         return SG_OK;
     }
-    // largest a over the listed rows: part scratch of the lean symbolic (sg_sym2.cu)
-    unsigned long long amax = 0;
-    CK(launch_max_i64(rs.a, nr, counter + 1, s));
-    CK(cudaMemcpyAsync(&amax, counter + 1, sizeof(amax), cudaMemcpyDeviceToHost, s));
-    CK(cudaStreamSynchronize(s));
-    const int64_t np = sym2_scratch_parts((int64_t)amax);
+    const int64_t np = sym2_scratch_parts(amax);
     void* pscr = np > 0 ? sc.get(part_bytes() * (size_t)np) : nullptr;
     if (np > 0 && !pscr) return SG_ERR_OOM;
     CK(launch_sym_heavy2(A, B, lists + off[BIN_HEAVY], cnt[BIN_HEAVY], rows, 0, rs.w, rs.u, nullptr, nullptr, nullptr,
-                         0, nullptr, nullptr, nullptr, 0, counter, s, cnt[BIN_HEAVY], pscr, (int64_t)amax));
+                         0, nullptr, nullptr, nullptr, 0, counter, s, cnt[BIN_HEAVY], pscr, amax));
     return SG_OK;
 }
 
@@ -275,33 +274,34 @@ sg_status identify(const Mat& A, const Mat& B, const int64_t* rows, int64_t nr, 
     sg_status st = row_stats(A, B, rows, nr, c->cap_L, sc, rs, s);
     if (st != SG_OK) return st;
     CostModelD cm = cm_of(c);
-    if ((st = check_cost_bound(cm, rs, nr, sc, s)) != SG_OK) return st;
     size_t hb = sizeof(long long) * (size_t)(c->cap_L + 1);
     long long* hd = (long long*)sc.get(hb);
     long long* hc = (long long*)sc.get(hb);
     long long* hw = (long long*)sc.get(hb);
     long long* sums = (long long*)sc.get(4 * sizeof(long long));
     ThrResult* dres = (ThrResult*)sc.get(sizeof(ThrResult));
-    if (!hd || !hc || !hw || !sums || !dres) return SG_ERR_OOM;
+    // overflow bound (fp64 sum of c_L + c_H) and the per-class sums of u at the chosen threshold (the
+    // sample's compression, used by the cost-weighted split, R19): read back together with the
+    // threshold in one copy + sync
+    double* dm = (double*)sc.get(sizeof(double));
+    unsigned long long* us = (unsigned long long*)sc.get(2 * sizeof(unsigned long long));
+    if (!hd || !hc || !hw || !sums || !dres || !dm || !us) return SG_ERR_OOM;
+    CK(launch_cost_mag(cm, rs.w, rs.a, rs.u, nr, dm, s));
     CK(launch_cost_hist(cm, rs.w, rs.a, rs.u, nr, hd, hc, hw, sums, s));
     CK(launch_argmin(cm, hd, hc, hw, sums, dres, s));
-    CK(cudaMemcpyAsync(res, dres, sizeof(ThrResult), cudaMemcpyDeviceToHost, s));
-    CK(cudaStreamSynchronize(s));
-    // per-class sums of u over the rows at the chosen threshold (the sample's compression, used by
-    // the cost-weighted split, R19)
-    unsigned long long* us = (unsigned long long*)sc.get(2 * sizeof(unsigned long long));
-    if (!us) return SG_ERR_OOM;
+    CK(launch_class_usum_dev(rs.w, rs.u, nr, &dres->thr, us, s));
+    double hm = 0.0;
     unsigned long long hu[2] = {0, 0};
-    CK(launch_class_usum(rs.w, rs.u, nr, res->thr, us, s));
+    CK(cudaMemcpyAsync(res, dres, sizeof(ThrResult), cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(&hm, dm, sizeof(double), cudaMemcpyDeviceToHost, s));
     CK(cudaMemcpyAsync(hu, us, sizeof(hu), cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
+    if (hm >= kCostLimit) return SG_ERR_OVERFLOW;
     res->U_L = (long long)hu[0];
     res->U_H = (long long)hu[1];
     return SG_OK;
 }
 
-// Non-negative coefficients keep every cost prefix monotone (k_cuts' binary search relies on it) and
-// make the fp64 magnitude sum of check_cost_bound an upper bound of every integer sum.
 sg_status check_model(const sg_cost_model* c) {
     if (c->cap_L < 0 || c->cap_L > SG_CAP_L_MAX) return SG_ERR_INVALID_ARG;
     const int64_t co[] = {c->kappa_L, c->lambda_L, c->sigma_L, c->rho_L, c->kappa_H, c->lambda_H, c->tau_H, c->mu_H,

@@ -180,7 +180,10 @@ __device__ __forceinline__ int acc_insert(int32_t* keys, double* vals, int32_t c
     uint32_t h;
     if (ident) {
         h = d;
-        if (keys[h] != c) keys[h] = c;  // idempotent: every writer stores the same key
+        // every writer of slot d stores the same key c into a slot that starts at EMPTY_KEY (-1, all bits
+        // set): an atomic AND installs it race-free (a native shared atomic; compute-sanitizer racecheck
+        // flagged the earlier plain idempotent store, profiles/r02_sanitizer_racecheck.log)
+        atomicAnd(&keys[h], c);
     } else {
         h = (uint32_t)(((uint64_t)d * mult) >> 32);
         while (true) {

@@ -168,6 +168,8 @@ cudaError_t launch_cost_mag(const CostModelD& cm, const int64_t* w, const int64_
 constexpr double kCostLimit = 4611686018427387904.0;  // 2^62: a cost bound at or above it -> SG_ERR_OVERFLOW
 cudaError_t launch_class_usum(const int64_t* w, const int64_t* u, int64_t nr, int64_t thr, unsigned long long* out,
                               cudaStream_t s);
+cudaError_t launch_class_usum_dev(const int64_t* w, const int64_t* u, int64_t nr, const long long* thr_dev,
+                                  unsigned long long* out, cudaStream_t s);
 cudaError_t launch_gather_rows(const int64_t* src, const int64_t* rows, int64_t nr, int64_t* dst, cudaStream_t s);
 cudaError_t launch_add_offset(int64_t* x, int64_t n, int64_t off, cudaStream_t s);
 cudaError_t launch_check_rows(const int64_t* rows, int64_t nr, int64_t n, unsigned long long* bad, cudaStream_t s);

@@ -379,6 +379,32 @@ __global__ void k_class_usum(const int64_t* __restrict__ w, const int64_t* __res
     }
 }
 
+// the same with the threshold read from device memory (k_argmin's result; no host round trip)
+__global__ void k_class_usum_dev(const int64_t* __restrict__ w, const int64_t* __restrict__ u, int64_t nr,
+                                 const long long* __restrict__ thr_dev, unsigned long long* out) {
+    const long long thr = *thr_dev;
+    unsigned long long sl = 0, sh = 0;
+    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < nr; j += (int64_t)gridDim.x * blockDim.x) {
+        const long long wj = w[j];
+        if (wj == 0) continue;
+        if (wj <= thr) sl += (unsigned long long)u[j]; else sh += (unsigned long long)u[j];
+    }
+    sl = warp_sum(sl);
+    sh = warp_sum(sh);
+    if ((threadIdx.x & 31) == 0) {
+        if (sl) atomicAdd(&out[0], sl);
+        if (sh) atomicAdd(&out[1], sh);
+    }
+}
+
+cudaError_t launch_class_usum_dev(const int64_t* w, const int64_t* u, int64_t nr, const long long* thr_dev,
+                                  unsigned long long* out, cudaStream_t s) {
+    cudaError_t e = cudaMemsetAsync(out, 0, 2 * sizeof(unsigned long long), s);
+    if (e != cudaSuccess || nr <= 0) return e;
+    SG_LAUNCH("k_class_usum", s, k_class_usum_dev<<<grid_for(nr, 256, 148 * 4), 256, 0, s>>>(w, u, nr, thr_dev, out));
+    return cudaGetLastError();
+}
+
 cudaError_t launch_class_usum(const int64_t* w, const int64_t* u, int64_t nr, int64_t thr, unsigned long long* out,
                               cudaStream_t s) {
     cudaError_t e = cudaMemsetAsync(out, 0, 2 * sizeof(unsigned long long), s);
