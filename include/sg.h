@@ -213,6 +213,34 @@ sg_status sg_gather(sg_plan* plan, void* nccl_comm, int gather_values,
                     int32_t* C_col_global /*nullable*/, void* C_val_global /*nullable*/, int64_t nnz_cap,
                     int64_t* nnz_total_out /*host*/, void* stream);
 
+/* ---- assembly through NCCL symmetric memory (Alg. 2 l.7) --------
+ * The assembled C lives in NCCL symmetric windows on every rank (ncclMemAlloc + ncclCommWindowRegister,
+ * NCCL_WIN_COLL_SYMMETRIC; NCCL >= 2.28 device API). Flow per rank: sg_symbolic -> sg_sym_c_layout
+ * (where this rank's rows go) -> sg_numeric with C_col / C_val = the window buffers + that offset (the
+ * numeric kernels write the rank's rows straight into its own window) -> sg_sym_c_assemble (one kernel
+ * stores the rank's rows into every LSA peer's window over NVLink through ncclGetLsaPointer, then an
+ * LSA barrier). No NCCL collective moves C. */
+typedef struct sg_sym_c sg_sym_c;
+/* Collective over nccl_comm: every rank passes the same n_rows (rows of the global C) and nnz_cap
+ * (capacity of col / val). Errors: INVALID_ARG, OOM (ncclMemAlloc), NCCL. */
+sg_status sg_sym_c_create(void* nccl_comm, int64_t n_rows, int64_t nnz_cap, sg_dtype dtype, sg_sym_c** out /*host*/);
+/* This rank's copy of the assembled C: row_ptr int64[n_rows+1], col int32[nnz_cap], val dtype[nnz_cap]
+ * (device; owned by the sg_sym_c, valid until sg_sym_c_destroy). Any output pointer may be NULL. */
+sg_status sg_sym_c_buffers(const sg_sym_c* S, int64_t** row_ptr, int32_t** col, void** val);
+/* Collective (one ncclAllGather of (row_begin, row_end, nnz) per rank; synchronises): this rank's first
+ * global C entry (host) and the total nnz (host, nullable). Errors: SHAPE (blocks not contiguous from row
+ * 0, rows != n_rows, or total > nnz_cap; the same on every rank), DTYPE, NCCL. */
+sg_status sg_sym_c_layout(sg_sym_c* S, sg_plan* plan, int64_t* c_offset_out /*host*/, int64_t* nnz_total_out /*host*/,
+                          void* stream);
+/* Collective: pushes this rank's rows (local_row_ptr = the plan's sg_symbolic prefix, plus the global
+ * offset; col / val from its window at the offset, written there by sg_numeric) into every LSA peer's
+ * window, then an LSA barrier; on return every rank's buffers hold the whole C. Synchronises. */
+sg_status sg_sym_c_assemble(sg_sym_c* S, sg_plan* plan, const int64_t* local_row_ptr, void* stream);
+void sg_sym_c_destroy(sg_sym_c* S);
+/* Stream-ordered device-to-device copy of `bytes` bytes (plumbing for bindings that hold raw device
+ * pointers, e.g. copying out of a sg_sym_c window). Errors: INVALID_ARG, CUDA. */
+sg_status sg_copy_device(void* dst, const void* src, int64_t bytes, void* stream);
+
 /* The host-only arithmetic of sg_gather (no device work, usable without a GPU): lay holds the
  * per-rank (row_begin, row_end, nnz) triples in rank order. Checks that the blocks are contiguous
  * from row 0 (SHAPE otherwise) and writes begin[r] (first row of rank r, nranks entries), off[r]

@@ -70,6 +70,13 @@ def _L():
         lib.oracle_row_work.argtypes = [i64, P, P, P, P]
         lib.oracle_spgemm_count.argtypes = [P, P, P, P, i64, P, P]
         lib.oracle_spgemm_moments.argtypes = [P, P, P, P, i64, P, P]
+        lib.oracle_hh_block_count.argtypes = [P, P, P, P, i64, ctypes.c_int, ctypes.c_int, i64, P, P]
+        lib.oracle_hh_block_fill.argtypes = [P, P, P, ctypes.c_int, P, P, P, ctypes.c_int, i64, ctypes.c_int,
+                                             ctypes.c_int, i64, P, P, P, P]
+        lib.oracle_hh_sample.restype = i64
+        lib.oracle_hh_sample.argtypes = [i64, P, P, u64, ctypes.c_double, P, P, P, P]
+        lib.oracle_hh_extrapolate.restype = i64
+        lib.oracle_hh_extrapolate.argtypes = [i64]
         lib.oracle_spgemm_fill.argtypes = [P, P, P, ctypes.c_int, P, P, P, ctypes.c_int, i64, P, P, P, P, P]
         lib.oracle_sample_rows.restype = i64
         lib.oracle_sample_rows.argtypes = [i64, i64, u64, ctypes.c_double, P]
@@ -239,6 +246,62 @@ def exhaustive_threshold(A, B, cm: CostModel, w_all=None, u_all=None) -> tuple[i
     w_all = row_work(A, B) if w_all is None else w_all
     u_all = counts(A, B) if u_all is None else u_all
     return threshold(cm, w_all, np.diff(A.row_ptr), u_all)
+
+
+# ---- HH four-block variant (NEXT #4; Alg. 3) ----------------------------------
+
+def hh_block(A, B, t: int, xa: int, yb: int, rows=None) -> RowsResult:
+    """Block A_X B_Y of the HH-CPU decomposition (X = xa, Y = yb; 1 = high: more than t non-zeros)."""
+    rows = np.arange(A.nrows, dtype=np.int64) if rows is None else np.ascontiguousarray(rows, dtype=np.int64)
+    L = _L()
+    u = np.zeros(rows.shape[0], dtype=np.int64)
+    if rows.shape[0]:
+        L.oracle_hh_block_count(_p(A.row_ptr), _p(A.col), _p(B.row_ptr), _p(B.col), t, xa, yb, rows.shape[0], _p(rows), _p(u))
+    rp = np.zeros(rows.shape[0] + 1, dtype=np.int64)
+    np.cumsum(u, out=rp[1:])
+    col = np.empty(int(rp[-1]), dtype=np.int32)
+    val = np.empty(int(rp[-1]), dtype=np.float64)
+    if rows.shape[0]:
+        L.oracle_hh_block_fill(_p(A.row_ptr), _p(A.col), _p(A.val), int(A.val.dtype == np.float32), _p(B.row_ptr),
+                               _p(B.col), _p(B.val), int(B.val.dtype == np.float32), t, xa, yb, rows.shape[0],
+                               _p(rows), _p(rp), _p(col), _p(val))
+    return RowsResult(rows, rp, col, val, None, B.ncols)
+
+
+def hh_combine(blocks) -> RowsResult:
+    """Phase IV: the four blocks added row by row (same row list in every block)."""
+    rows = blocks[0].rows
+    out_rp = [0]
+    cols, vals = [], []
+    for s in range(len(rows)):
+        acc = {}
+        for R in blocks:
+            for c, v in zip(R.col[R.row_ptr[s]:R.row_ptr[s + 1]], R.val[R.row_ptr[s]:R.row_ptr[s + 1]]):
+                acc[int(c)] = acc.get(int(c), 0.0) + float(v)
+        ks = sorted(acc)
+        cols.extend(ks)
+        vals.extend(acc[k] for k in ks)
+        out_rp.append(len(cols))
+    return RowsResult(rows, np.array(out_rp, dtype=np.int64), np.array(cols, dtype=np.int32),
+                      np.array(vals, dtype=np.float64), None, blocks[0].ncols)
+
+
+def hh_sample(A, seed: int, f: float | None = None):
+    """Phase I Sample (L285-L287): returns (kept row ids, A' as (row_ptr, col, source positions)); f
+    defaults to 1/sqrt(n)."""
+    n = A.nrows
+    f = 1.0 / max(1.0, np.sqrt(n)) if f is None else f
+    rows = np.empty(max(n, 1), dtype=np.int64)
+    rp = np.empty(max(n, 1) + 1, dtype=np.int64)
+    col = np.empty(max(A.nnz, 1), dtype=np.int32)
+    pos = np.empty(max(A.nnz, 1), dtype=np.int64)
+    s = int(_L().oracle_hh_sample(n, _p(A.row_ptr), _p(A.col), seed, f, _p(rows), _p(rp), _p(col), _p(pos)))
+    m = int(rp[s])
+    return rows[:s].copy(), rp[:s + 1].copy(), col[:m].copy(), pos[:m].copy()
+
+
+def hh_extrapolate(t_s: int) -> int:
+    return int(_L().oracle_hh_extrapolate(int(t_s)))
 
 
 # ---- O3 -------------------------------------------------------------------------------------

@@ -36,6 +36,10 @@
  *        (heavy iff "more than t", L272-L274; equality -> light, reading R13), candidates
  *        {0} u {w_i > 0} clipped to t <= cap_L, thr = smallest minimiser. "Extrapolate" is the
  *        identity (L236 r = r'; whole rows sampled, reading R3).
+ *   HH oracle_hh_block_count / oracle_hh_block_fill / oracle_hh_sample / oracle_hh_extrapolate
+ *        The HH-CPU four-block decomposition (Alg. 3): C = sum over (X, Y) in {H, L}^2 of
+ *        A_X B_Y, high iff more than t non-zeros (L274); the sqrt(n)-row sampler with relabelled columns
+ *        (L285-L287; reading R20) and the extrapolation t_A = t_s^2 (L291).
  *   O6 oracle_heavy_share
  *        r(t) = 100 * sum_{w_i > t} w_i / W, the split percentage of Alg. 2 (L204, L208).
  */
@@ -302,6 +306,80 @@ void oracle_partition_cost(const oracle_cost_model* cm, int64_t thr, const int64
     oracle_partition(n, c.data(), G, cuts);
     if (cost_total) *cost_total = (int64_t)tot;
 }
+
+// ---- HH (Alg. 3 "HH-CPU") ---------------------------------
+// A row is HIGH dense iff it has MORE than t non-zeros (L274). With A_H / A_L the high / low rows of A
+// and B_H / B_L those of B, C = A B = A_H B_H + A_H B_L + A_L B_H + A_L B_L where X_Y (X, Y in {H, L})
+// restricts row i to class X and its k entries to B rows of class Y (Alg. 3 Phases II-III), and Phase IV
+// adds the blocks. oracle_hh_block_fill writes block (xa, yb) (0 = L, 1 = H) of the listed rows with
+// the same sorted-map accumulator as O1: rows of the other class, and k entries of the other class,
+// contribute nothing (an empty row stays empty).
+void oracle_hh_block_count(const int64_t* Arp, const int32_t* Acol, const int64_t* Brp, const int32_t* Bcol,
+                           int64_t t, int xa, int yb, int64_t nsel, const int64_t* rows, int64_t* u) {
+    #pragma omp parallel for schedule(dynamic, 1)
+    for (int64_t s = 0; s < nsel; ++s) {
+        int64_t i = rows[s];
+        std::map<int32_t, double> acc;
+        if (((Arp[i + 1] - Arp[i]) > t) == (xa == 1)) {
+            for (int64_t p = Arp[i]; p < Arp[i + 1]; ++p) {
+                int32_t k = Acol[p];
+                if (((Brp[k + 1] - Brp[k]) > t) != (yb == 1)) continue;
+                for (int64_t q = Brp[k]; q < Brp[k + 1]; ++q) acc[Bcol[q]] += 0.0;
+            }
+        }
+        u[s] = (int64_t)acc.size();
+    }
+}
+
+void oracle_hh_block_fill(const int64_t* Arp, const int32_t* Acol, const void* Aval, int A_f32,
+                          const int64_t* Brp, const int32_t* Bcol, const void* Bval, int B_f32,
+                          int64_t t, int xa, int yb, int64_t nsel, const int64_t* rows, const int64_t* out_ptr,
+                          int32_t* col_out, double* val_out) {
+    #pragma omp parallel for schedule(dynamic, 1)
+    for (int64_t s = 0; s < nsel; ++s) {
+        int64_t i = rows[s];
+        std::map<int32_t, double> acc;
+        if (((Arp[i + 1] - Arp[i]) > t) == (xa == 1)) {
+            for (int64_t p = Arp[i]; p < Arp[i + 1]; ++p) {
+                int32_t k = Acol[p];
+                if (((Brp[k + 1] - Brp[k]) > t) != (yb == 1)) continue;
+                double a = load_val(Aval, A_f32, p);
+                for (int64_t q = Brp[k]; q < Brp[k + 1]; ++q) acc[Bcol[q]] += a * load_val(Bval, B_f32, q);
+            }
+        }
+        int64_t o = out_ptr[s];
+        for (const auto& kv : acc) { col_out[o] = kv.first; val_out[o] = kv.second; ++o; }
+    }
+}
+
+// Phase I Sample of Section V-A (L285-L287): A' keeps ~sqrt(n) rows of A chosen uniformly at random
+// (Bernoulli(1/sqrt(n)) per row through the sampler hash, reading R4) and, in each kept row, the
+// elements whose column is itself a kept row index, relabelled by rank so that A' is s x s with
+// s = |kept rows| ("column indices transformed so that the column indices are within 1 to sqrt(n)";
+// DESIGN.md reading R20). Writes the kept rows' ids (rows_out, s entries) and A' (rp_out s+1; col_out,
+// pos_out = source position in A, up to nnz(A) entries). Returns s.
+int64_t oracle_hh_sample(int64_t n, const int64_t* Arp, const int32_t* Acol, uint64_t seed, double f,
+                         int64_t* rows_out, int64_t* rp_out, int32_t* col_out, int64_t* pos_out) {
+    const uint64_t Tf = f >= 1.0 ? ~0ull : (uint64_t)std::ldexp(f, 64);
+    std::vector<int64_t> rank(n, -1);
+    int64_t s = 0;
+    for (int64_t i = 0; i < n; ++i)
+        if (f >= 1.0 || hash3(seed, TAG_SAMPLE, (uint64_t)i) < Tf) { rank[i] = s; rows_out[s++] = i; }
+    int64_t o = 0;
+    rp_out[0] = 0;
+    for (int64_t r = 0; r < s; ++r) {
+        int64_t i = rows_out[r];
+        for (int64_t p = Arp[i]; p < Arp[i + 1]; ++p) {
+            int32_t j = Acol[p];
+            if (j < n && rank[j] >= 0) { col_out[o] = (int32_t)rank[j]; pos_out[o] = p; ++o; }
+        }
+        rp_out[r + 1] = o;
+    }
+    return s;
+}
+
+// Phase I Extrapolate (L291): the off-line relation the paper found for spmm, t_A = t_s * t_s.
+int64_t oracle_hh_extrapolate(int64_t t_s) { return t_s * t_s; }
 
 // ---- O6: r(t) = 100 * sum_{w_i > t} w_i / W  (split percentage) -------
 double oracle_heavy_share(int64_t n, const int64_t* w, int64_t t) {

@@ -38,7 +38,9 @@ EXPORTS = ["sg_status_string", "sg_version", "sg_default_cost_model", "sg_row_wo
            "sg_exhaustive_threshold", "sg_cost_curve", "sg_partition", "sg_symbolic", "sg_numeric", "sg_gather",
            "sg_plan_get_info", "sg_plan_get_classes", "sg_plan_get_work", "sg_plan_destroy", "sg_sample_rows",
            "sg_profile_enable", "sg_launch_count", "sg_profile_count", "sg_profile_read", "sg_profile_reset",
-           "sg_gather_layout", "sg_threshold_on_rows", "sg_set_option", "sg_get_option"]
+           "sg_gather_layout", "sg_threshold_on_rows", "sg_set_option", "sg_get_option",
+           "sg_sym_c_create", "sg_sym_c_buffers", "sg_sym_c_layout", "sg_sym_c_assemble", "sg_sym_c_destroy",
+           "sg_copy_device"]
 
 SG_OPT_VALIDATE, SG_OPT_DENSE_LOG2, SG_OPT_VARIANT = 0, 1, 2
 
@@ -125,6 +127,12 @@ def load(build_if_missing: bool = True):
         "sg_numeric": (st, [P, V, V, P, P, P]),
         "sg_gather": (st, [P, P, ctypes.c_int, P, P, P, P, i64, P, P, i64, pi64, P]),
         "sg_set_option": (st, [ctypes.c_int, i64]),
+        "sg_sym_c_create": (st, [P, i64, i64, ctypes.c_int, ctypes.POINTER(P)]),
+        "sg_sym_c_buffers": (st, [P, ctypes.POINTER(P), ctypes.POINTER(P), ctypes.POINTER(P)]),
+        "sg_sym_c_layout": (st, [P, P, pi64, pi64, P]),
+        "sg_sym_c_assemble": (st, [P, P, P, P]),
+        "sg_sym_c_destroy": (None, [P]),
+        "sg_copy_device": (st, [P, P, i64, P]),
         "sg_get_option": (i64, [ctypes.c_int]),
         "sg_plan_get_info": (st, [P, ctypes.POINTER(PlanInfo)]),
         "sg_plan_get_classes": (st, [P, P, P]),
@@ -432,6 +440,61 @@ class profile:
 
 def launch_count() -> int:
     return int(lib().sg_launch_count())
+
+
+class SymC:
+    """C assembled in NCCL symmetric windows (NEXT #3; include/sg.h sg_sym_c_*). Collective over the
+    communicator: every rank creates it with the same (n_rows, nnz_cap, dtype)."""
+
+    def __init__(self, comm_ptr: int, n_rows: int, nnz_cap: int, dtype=torch.float64):
+        _require_cuda()
+        self.n, self.cap, self.dtype = int(n_rows), int(nnz_cap), dtype
+        h = ctypes.c_void_p()
+        _check(lib().sg_sym_c_create(ctypes.c_void_p(comm_ptr), self.n, self.cap,
+                                     0 if dtype == torch.float64 else 1, ctypes.byref(h)), "sg_sym_c_create")
+        self.handle = h
+        rp, col, val = ctypes.c_void_p(), ctypes.c_void_p(), ctypes.c_void_p()
+        _check(lib().sg_sym_c_buffers(h, ctypes.byref(rp), ctypes.byref(col), ctypes.byref(val)), "sg_sym_c_buffers")
+        self._ptrs = (rp.value, col.value, val.value)
+        self.offset = None
+        self.total = None
+
+    def layout(self, plan: "Plan"):
+        off, tot = ctypes.c_int64(0), ctypes.c_int64(0)
+        _check(lib().sg_sym_c_layout(self.handle, plan.handle, ctypes.byref(off), ctypes.byref(tot), _stream()),
+               "sg_sym_c_layout")
+        self.offset, self.total = int(off.value), int(tot.value)
+        return self.offset, self.total
+
+    def numeric_into(self, plan: "Plan", A: "DeviceCSR", B: "DeviceCSR"):
+        """sg_numeric writing this rank's rows straight into its window at the layout offset."""
+        vs = 8 if self.dtype == torch.float64 else 4
+        _check(lib().sg_numeric(plan.handle, ctypes.byref(A.view()), ctypes.byref(B.view()),
+                                ctypes.c_void_p(self._ptrs[1] + 4 * self.offset),
+                                ctypes.c_void_p(self._ptrs[2] + vs * self.offset), _stream()), "sg_numeric")
+
+    def assemble(self, plan: "Plan"):
+        _check(lib().sg_sym_c_assemble(self.handle, plan.handle, _ptr(plan.row_ptr), _stream()), "sg_sym_c_assemble")
+
+    def tensors(self):
+        """(row_ptr, col, val) of the assembled C as host-owned copies (the windows stay with the SymC)."""
+        import numpy as np
+        L = lib()
+        out = []
+        for ptr, n, dt in ((self._ptrs[0], self.n + 1, torch.int64), (self._ptrs[1], self.total, torch.int32),
+                           (self._ptrs[2], self.total, self.dtype)):
+            t = torch.empty(n, dtype=dt, device="cuda")
+            nbytes = n * t.element_size()
+            if nbytes:
+                _check(L.sg_copy_device(ctypes.c_void_p(t.data_ptr()), ctypes.c_void_p(ptr), nbytes, _stream()),
+                       "sg_copy_device")
+            out.append(t)
+        return tuple(out)
+
+    def destroy(self):
+        if self.handle:
+            lib().sg_sym_c_destroy(self.handle)
+            self.handle = None
 
 
 def set_option(key: int, value: int) -> None:

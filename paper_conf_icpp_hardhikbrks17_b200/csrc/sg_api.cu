@@ -811,6 +811,13 @@ sg_status sg_plan_get_work(const sg_plan* pl, int64_t* w_out, void* stream) {
     return SG_OK;
 }
 
+sg_status sg_copy_device(void* dst, const void* src, int64_t bytes, void* stream) {
+    if (bytes < 0 || (bytes > 0 && (!dst || !src))) return SG_ERR_INVALID_ARG;
+    if (bytes == 0) return SG_OK;
+    CK(cudaMemcpyAsync(dst, src, (size_t)bytes, cudaMemcpyDeviceToDevice, (cudaStream_t)stream));
+    return SG_OK;
+}
+
 void sg_plan_destroy(sg_plan* pl) {
     if (!pl) return;
     for (void* p : pl->allocs) cudaFreeAsync(p, pl->s);
