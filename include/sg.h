@@ -241,6 +241,32 @@ void sg_sym_c_destroy(sg_sym_c* S);
  * pointers, e.g. copying out of a sg_sym_c window). Errors: INVALID_ARG, CUDA. */
 sg_status sg_copy_device(void* dst, const void* src, int64_t bytes, void* stream);
 
+/* ---- the HH-CPU four-block variant (PAPER Alg. 3, Section V-A) ------
+ * A row is HIGH dense iff it has more than t non-zeros (L274). C = A_H B_H + A_H B_L + A_L B_H + A_L B_L:
+ * the four products run on the hot path (sg_symbolic / sg_numeric); Phase IV adds two results P + Q as
+ * the product [P Q] * [I; I] (the accumulators add equal columns, structural zeros kept). The Python
+ * binding's spgemm_hh() / hh_threshold() drive the whole algorithm. */
+/* Phase I: keeps the rows of M with (nnz > t) == (high != 0), empties the others (row ids unchanged).
+ * rp_out int64[nrows+1]; col_out / val_out capacity M.nnz (device, caller-owned); nnz_out (host).
+ * Synchronises. Errors: INVALID_ARG, DTYPE, OVERFLOW. */
+sg_status sg_hh_filter(const sg_csr_view* M, int64_t t, int high, int64_t* rp_out, int32_t* col_out, void* val_out,
+                       int64_t* nnz_out /*host*/, void* stream);
+/* [P Q]: nrows x (P.ncols + Q.ncols), row i = P_i then Q_i with columns shifted by P.ncols. Outputs:
+ * rp_out int64[nrows+1], col_out / val_out capacity P.nnz + Q.nnz. Errors: SHAPE (row counts), DTYPE,
+ * OVERFLOW (P.ncols + Q.ncols > INT32_MAX). */
+sg_status sg_hh_hstack(const sg_csr_view* P, const sg_csr_view* Q, int64_t* rp_out, int32_t* col_out, void* val_out,
+                       void* stream);
+/* [I; I] (2p x p): row k holds (k mod p, 1). rp_out int64[2p+1], col_out int32[2p], val_out dtype[2p]. */
+sg_status sg_hh_identity2(int64_t p, sg_dtype dtype, int64_t* rp_out, int32_t* col_out, void* val_out, void* stream);
+/* Phase I Sample (L285-L287; reading R20): the principal sub-matrix A' = A[S, S] of a square A on
+ * S = { i : h(seed, SAMPLE, i) < floor(f 2^64) } (f = 1/sqrt(n): the paper's sqrt(n) x sqrt(n) sample),
+ * columns relabelled by rank. Outputs (device, capacity n / n+1 / A.nnz): rows_out = S ascending, rp_out
+ * (s+1), col_out (relabelled), pos_out (each entry's position in A), val_out (its value; nullable);
+ * s_out, nnz_out (host). Synchronises. Errors: SHAPE (A not square), INVALID_ARG. */
+sg_status sg_hh_sample(const sg_csr_view* A, uint64_t seed, double f, int64_t* rows_out, int64_t* rp_out,
+                       int32_t* col_out, int64_t* pos_out, void* val_out /*nullable*/, int64_t* s_out /*host*/,
+                       int64_t* nnz_out /*host*/, void* stream);
+
 /* The host-only arithmetic of sg_gather (no device work, usable without a GPU): lay holds the
  * per-rank (row_begin, row_end, nnz) triples in rank order. Checks that the blocks are contiguous
  * from row 0 (SHAPE otherwise) and writes begin[r] (first row of rank r, nranks entries), off[r]

@@ -40,7 +40,7 @@ EXPORTS = ["sg_status_string", "sg_version", "sg_default_cost_model", "sg_row_wo
            "sg_profile_enable", "sg_launch_count", "sg_profile_count", "sg_profile_read", "sg_profile_reset",
            "sg_gather_layout", "sg_threshold_on_rows", "sg_set_option", "sg_get_option",
            "sg_sym_c_create", "sg_sym_c_buffers", "sg_sym_c_layout", "sg_sym_c_assemble", "sg_sym_c_destroy",
-           "sg_copy_device"]
+           "sg_copy_device", "sg_hh_filter", "sg_hh_hstack", "sg_hh_identity2", "sg_hh_sample"]
 
 SG_OPT_VALIDATE, SG_OPT_DENSE_LOG2, SG_OPT_VARIANT = 0, 1, 2
 
@@ -133,6 +133,10 @@ def load(build_if_missing: bool = True):
         "sg_sym_c_assemble": (st, [P, P, P, P]),
         "sg_sym_c_destroy": (None, [P]),
         "sg_copy_device": (st, [P, P, i64, P]),
+        "sg_hh_filter": (st, [P, i64, ctypes.c_int, P, P, P, pi64, P]),
+        "sg_hh_hstack": (st, [P, P, P, P, P, P]),
+        "sg_hh_identity2": (st, [i64, ctypes.c_int, P, P, P, P]),
+        "sg_hh_sample": (st, [P, ctypes.c_uint64, ctypes.c_double, P, P, P, P, P, pi64, pi64, P]),
         "sg_get_option": (i64, [ctypes.c_int]),
         "sg_plan_get_info": (st, [P, ctypes.POINTER(PlanInfo)]),
         "sg_plan_get_classes": (st, [P, P, P]),
@@ -495,6 +499,127 @@ class SymC:
         if self.handle:
             lib().sg_sym_c_destroy(self.handle)
             self.handle = None
+
+
+# ---- NEXT #4: the HH-CPU four-block variant (PAPER Alg. 3, Section V-A) ----------
+
+def sg_hh_filter(M: DeviceCSR, t: int, high: bool) -> DeviceCSR:
+    """Phase I: the rows of M whose class is `high` (more than t non-zeros); others emptied."""
+    _require_cuda()
+    dev = M.row_ptr.device
+    rp = torch.empty(M.nrows + 1, dtype=torch.int64, device=dev)
+    col = torch.empty(max(M.nnz, 1), dtype=torch.int32, device=dev)
+    val = torch.empty(max(M.nnz, 1), dtype=M.val.dtype, device=dev)
+    nz = ctypes.c_int64(0)
+    _check(lib().sg_hh_filter(ctypes.byref(M.view()), int(t), int(bool(high)), _ptr(rp), _ptr(col), _ptr(val),
+                              ctypes.byref(nz), _stream()), "sg_hh_filter")
+    return DeviceCSR(M.nrows, M.ncols, rp, col[: nz.value], val[: nz.value])
+
+
+def sg_hh_add(P: DeviceCSR, Q: DeviceCSR, thr: int | None = None) -> DeviceCSR:
+    """Phase IV: P + Q (same shape) as the product [P Q] * [I; I] on the hot path (equal columns added,
+    union sorted, structural zeros kept)."""
+    _require_cuda()
+    dev = P.row_ptr.device
+    n = P.nrows
+    rp = torch.empty(n + 1, dtype=torch.int64, device=dev)
+    col = torch.empty(max(P.nnz + Q.nnz, 1), dtype=torch.int32, device=dev)
+    val = torch.empty(max(P.nnz + Q.nnz, 1), dtype=P.val.dtype, device=dev)
+    _check(lib().sg_hh_hstack(ctypes.byref(P.view()), ctypes.byref(Q.view()), _ptr(rp), _ptr(col), _ptr(val), _stream()),
+           "sg_hh_hstack")
+    PQ = DeviceCSR(n, P.ncols + Q.ncols, rp, col[: P.nnz + Q.nnz], val[: P.nnz + Q.nnz])
+    p = P.ncols
+    irp = torch.empty(2 * p + 1, dtype=torch.int64, device=dev)
+    icol = torch.empty(max(2 * p, 1), dtype=torch.int32, device=dev)
+    ival = torch.empty(max(2 * p, 1), dtype=P.val.dtype, device=dev)
+    _check(lib().sg_hh_identity2(p, 0 if P.val.dtype == torch.float64 else 1, _ptr(irp), _ptr(icol), _ptr(ival),
+                                 _stream()), "sg_hh_identity2")
+    I2 = DeviceCSR(2 * p, p, irp, icol[: 2 * p], ival[: 2 * p])
+    C, _ = spgemm(PQ, I2, thr=thr if thr is not None else SG_CAP_L_MAX)
+    return C
+
+
+def spgemm_hh(A: DeviceCSR, B: DeviceCSR, t: int, sample_frac: float = 0.01, seed: int = 1):
+    """HH-CPU (Alg. 3) at density threshold t: Phase I splits A and B into high / low dense rows, Phases
+    II-III compute A_X B_Y for X, Y in {H, L} on the hot path, Phase IV adds them. Returns (C, info)."""
+    AH, AL = sg_hh_filter(A, t, True), sg_hh_filter(A, t, False)
+    BH, BL = (AH, AL) if B is A else (sg_hh_filter(B, t, True), sg_hh_filter(B, t, False))
+    info = {"t": int(t), "blocks": {}}
+    sums = []
+    for xa, AX in (("H", AH), ("L", AL)):
+        parts = []
+        for yb, BY in (("H", BH), ("L", BL)):
+            Cxy, inf = spgemm(AX, BY, sample_frac, seed) if AX.nnz and BY.nnz else (None, None)
+            if Cxy is None:
+                Cxy = DeviceCSR(A.nrows, B.ncols, torch.zeros(A.nrows + 1, dtype=torch.int64, device=A.row_ptr.device),
+                                torch.empty(0, dtype=torch.int32, device=A.row_ptr.device),
+                                torch.empty(0, dtype=A.val.dtype, device=A.row_ptr.device))
+            info["blocks"][xa + yb] = Cxy.nnz
+            parts.append(Cxy)
+        sums.append(sg_hh_add(parts[0], parts[1]))
+    return sg_hh_add(sums[0], sums[1]), info
+
+
+def sg_hh_sample(A: DeviceCSR, seed: int, f: float | None = None):
+    """Phase I Sample (L285-L287, reading R20): the principal sub-matrix A[S, S], |S| ~ f n (f = 1/sqrt(n)
+    by default). Returns (rows S, A' as DeviceCSR, positions of A' entries in A)."""
+    _require_cuda()
+    import math
+    n = A.nrows
+    f = 1.0 / max(1.0, math.sqrt(n)) if f is None else f
+    dev = A.row_ptr.device
+    rows = torch.empty(max(n, 1), dtype=torch.int64, device=dev)
+    rp = torch.empty(n + 1, dtype=torch.int64, device=dev)
+    col = torch.empty(max(A.nnz, 1), dtype=torch.int32, device=dev)
+    pos = torch.empty(max(A.nnz, 1), dtype=torch.int64, device=dev)
+    val = torch.empty(max(A.nnz, 1), dtype=A.val.dtype, device=dev)
+    sn, nz = ctypes.c_int64(0), ctypes.c_int64(0)
+    _check(lib().sg_hh_sample(ctypes.byref(A.view()), seed, f, _ptr(rows), _ptr(rp), _ptr(col), _ptr(pos), _ptr(val),
+                              ctypes.byref(sn), ctypes.byref(nz), _stream()), "sg_hh_sample")
+    s_, m = int(sn.value), int(nz.value)
+    return rows[:s_], DeviceCSR(s_, s_, rp[: s_ + 1], col[:m], val[:m]), pos[:m]
+
+
+def hh_threshold(A: DeviceCSR, seed: int = 1, f: float | None = None, reps: int = 3):
+    """Sample -> Identify -> Extrapolate for HH-CPU (Section V-A): A' = sg_hh_sample(A); Identify = a descent
+    over thresholds t' on the measured time of spgemm_hh(A', A', t') (the paper's "gradient descent based
+    approach", L289: doubling steps from the median row density while the time drops, then one refining
+    step of sqrt(2) each way); Extrapolate t_A = t_s^2 (L291). Returns (t_A, info)."""
+    import math
+    _, As, _ = sg_hh_sample(A, seed, f)
+    dens = torch.diff(As.row_ptr).float()
+    cache = {}
+
+    def T(t):
+        t = int(max(0, t))
+        if t not in cache:
+            ms = []
+            for _ in range(reps):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record()
+                spgemm_hh(As, As, t, sample_frac=0.05, seed=seed)
+                e1.record()
+                torch.cuda.synchronize()
+                ms.append(e0.elapsed_time(e1))
+            cache[t] = sorted(ms)[len(ms) // 2]
+        return cache[t]
+
+    t = max(1, int(dens[dens > 0].median().item()) if bool((dens > 0).any()) else 1)
+    best = t
+    for step in (2.0, 0.5):  # walk up, then down, while the time keeps dropping
+        cur = best
+        while True:
+            nxt = int(round(cur * step))
+            if nxt == cur or nxt < 0 or nxt > 1 << 20 or T(nxt) >= T(cur):
+                break
+            cur = nxt
+        if T(cur) < T(best):
+            best = cur
+    for nxt in (int(round(best * math.sqrt(2))), int(round(best / math.sqrt(2)))):
+        if T(nxt) < T(best):
+            best = nxt
+    return best * best, {"t_s": best, "sample_rows": As.nrows, "sample_nnz": As.nnz,
+                         "curve": {str(k): v for k, v in sorted(cache.items())}}
 
 
 def set_option(key: int, value: int) -> None:

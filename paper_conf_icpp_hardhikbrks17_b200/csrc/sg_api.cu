@@ -179,11 +179,13 @@ CostModelD cm_of(const sg_cost_model* c) {
 }
 
 // Default model: calibrated from the measured kernels (profiles/).
-// Fitted by tools/sweep.py (non-negative least squares of per-class kernel times over the
-// threshold grid on ER 2^18 and R-MAT 18; profiles/r01_sweep_calibration.json), in ps of SM time.
+// Refitted in round 2 on the round-2 kernels (sg_sym2.cu, sg_dense2.cu) by tools/sweep.py: non-negative
+// least squares of the per-class kernel times over the threshold grid on ER 2^18, R-MAT 18 and
+// un-permuted R-MAT 18 (profiles/r02_sweep_precal.json "fit"), in ps of SM time. (Round 1's constants,
+// fitted before the heavy kernels changed: 33399, 7915, 0, 0, 17907513, 1102, 68338, 209.)
 const sg_cost_model kDefaultModel = {
-    /*kappa_L*/ 33399, /*lambda_L*/ 7915, /*sigma_L*/ 0, /*rho_L*/ 0,
-    /*kappa_H*/ 17907513, /*lambda_H*/ 1102, /*tau_H*/ 68338, /*mu_H*/ 209,
+    /*kappa_L*/ 0, /*lambda_L*/ 10450, /*sigma_L*/ 0, /*rho_L*/ 0,
+    /*kappa_H*/ 5498663, /*lambda_H*/ 989, /*tau_H*/ 40554, /*mu_H*/ 0,
     /*tiles_fixed*/ 1, /*capu*/ 12288, /*cap_L*/ SG_CAP_L_MAX};
 
 // Partition model (reading R19): fitted by tools/fit_partition_model.py to 88 measured
@@ -808,6 +810,97 @@ sg_status sg_plan_get_work(const sg_plan* pl, int64_t* w_out, void* stream) {
     if (pl->poisoned) return SG_ERR_CUDA;
     if (pl->nr > 0)
         CK(cudaMemcpyAsync(w_out, pl->w, 8 * (size_t)pl->nr, cudaMemcpyDeviceToDevice, (cudaStream_t)stream));
+    return SG_OK;
+}
+
+// ---- NEXT #4: HH-CPU four blocks (PAPER Alg. 3, Section V-A; sg_hh.cu) --------
+sg_status sg_hh_filter(const sg_csr_view* M, int64_t t, int high, int64_t* rp_out, int32_t* col_out, void* val_out,
+                       int64_t* nnz_out, void* stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    init_pool();
+    sg_status st = validate_one(M, s);
+    if (st != SG_OK) return st;
+    if (!rp_out || !nnz_out || (M->nnz > 0 && (!col_out || !val_out))) return SG_ERR_INVALID_ARG;
+    Mat m = mat_of(M);
+    const int64_t n = M->nrows;
+    Scratch sc(s);
+    int64_t* len = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(n > 0 ? n : 1));
+    void* tmp = sc.get(scan_tmp_bytes(n));
+    if (!len || !tmp) return SG_ERR_OOM;
+    CK(launch_hh_len(m, t, high, len, s));
+    CK(scan_exclusive(len, rp_out, n, tmp, s));
+    CK(launch_hh_copy(m, rp_out, col_out, val_out, s));
+    int64_t nnz = 0;
+    CK(cudaMemcpyAsync(&nnz, rp_out + n, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    *nnz_out = nnz;
+    return SG_OK;
+}
+
+sg_status sg_hh_hstack(const sg_csr_view* P, const sg_csr_view* Q, int64_t* rp_out, int32_t* col_out, void* val_out,
+                       void* stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    init_pool();
+    sg_status st;
+    if ((st = validate_one(P, s)) != SG_OK || (st = validate_one(Q, s)) != SG_OK) return st;
+    if (P->nrows != Q->nrows) return SG_ERR_SHAPE;
+    if (P->dtype != Q->dtype) return SG_ERR_DTYPE;
+    if (P->ncols + Q->ncols > INT32_MAX) return SG_ERR_OVERFLOW;
+    if (!rp_out || (P->nnz + Q->nnz > 0 && (!col_out || !val_out))) return SG_ERR_INVALID_ARG;
+    Mat mp = mat_of(P), mq = mat_of(Q);
+    const int64_t n = P->nrows;
+    Scratch sc(s);
+    int64_t* len = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(n > 0 ? n : 1));
+    void* tmp = sc.get(scan_tmp_bytes(n));
+    if (!len || !tmp) return SG_ERR_OOM;
+    CK(launch_hh_hstack(mp, mq, len, nullptr, nullptr, 0, s));
+    CK(scan_exclusive(len, rp_out, n, tmp, s));
+    CK(launch_hh_hstack(mp, mq, rp_out, col_out, val_out, 1, s));
+    return SG_OK;
+}
+
+sg_status sg_hh_identity2(int64_t p, sg_dtype dtype, int64_t* rp_out, int32_t* col_out, void* val_out, void* stream) {
+    if (p < 0 || 2 * p > INT32_MAX || !rp_out || (p > 0 && (!col_out || !val_out))) return SG_ERR_INVALID_ARG;
+    if (dtype != SG_F64 && dtype != SG_F32) return SG_ERR_DTYPE;
+    init_pool();
+    CK(launch_hh_identity2(p, (int)dtype, rp_out, col_out, val_out, (cudaStream_t)stream));
+    return SG_OK;
+}
+
+sg_status sg_hh_sample(const sg_csr_view* A, uint64_t seed, double f, int64_t* rows_out, int64_t* rp_out,
+                       int32_t* col_out, int64_t* pos_out, void* val_out, int64_t* s_out, int64_t* nnz_out, void* stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    init_pool();
+    sg_status st = validate_one(A, s);
+    if (st != SG_OK) return st;
+    if (A->nrows != A->ncols) return SG_ERR_SHAPE;  // a principal sub-matrix needs a square A
+    if (!(f > 0.0 && f <= 1.0) || !rows_out || !rp_out || !s_out || !nnz_out ||
+        (A->nnz > 0 && (!col_out || !pos_out)))
+        return SG_ERR_INVALID_ARG;
+    Mat m = mat_of(A);
+    const int64_t n = A->nrows;
+    Scratch sc(s);
+    int64_t* keep = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(n > 0 ? n : 1));
+    int64_t* rank = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(n + 1));
+    int64_t* cnt = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(n > 0 ? n : 1));
+    void* tmp = sc.get(scan_tmp_bytes(n));
+    if (!keep || !rank || !cnt || !tmp) return SG_ERR_OOM;
+    const bool all = f >= 1.0;
+    const uint64_t Tf = all ? 0 : (uint64_t)std::ldexp(f, 64);
+    CK(launch_hh_mask(n, seed, Tf, all ? 1 : 0, keep, s));
+    CK(scan_exclusive(keep, rank, n, tmp, s));
+    int64_t sr = 0;
+    CK(cudaMemcpyAsync(&sr, rank + n, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    CK(launch_hh_rows_of_rank(n, keep, rank, rows_out, s));
+    CK(launch_hh_sub(m, keep, rank, rows_out, sr, cnt, nullptr, nullptr, nullptr, 0, s));
+    CK(scan_exclusive(cnt, rp_out, sr, tmp, s));
+    CK(launch_hh_sub(m, keep, rank, rows_out, sr, rp_out, col_out, pos_out, val_out, 1, s));
+    int64_t nz = 0;
+    CK(cudaMemcpyAsync(&nz, rp_out + sr, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    *s_out = sr;
+    *nnz_out = nz;
     return SG_OK;
 }
 

@@ -170,6 +170,16 @@ cudaError_t launch_class_usum(const int64_t* w, const int64_t* u, int64_t nr, in
                               cudaStream_t s);
 cudaError_t launch_class_usum_dev(const int64_t* w, const int64_t* u, int64_t nr, const long long* thr_dev,
                                   unsigned long long* out, cudaStream_t s);
+// HH four-block variant (sg_hh.cu)
+cudaError_t launch_hh_len(const Mat& M, int64_t t, int high, int64_t* len, cudaStream_t s);
+cudaError_t launch_hh_copy(const Mat& M, const int64_t* out_rp, int32_t* col, void* val, cudaStream_t s);
+cudaError_t launch_hh_hstack(const Mat& P, const Mat& Q, int64_t* rp, int32_t* col, void* val, int pass, cudaStream_t s);
+cudaError_t launch_hh_identity2(int64_t p, int dt, int64_t* rp, int32_t* col, void* val, cudaStream_t s);
+cudaError_t launch_hh_mask(int64_t n, uint64_t seed, uint64_t Tf, int all, int64_t* keep, cudaStream_t s);
+cudaError_t launch_hh_rows_of_rank(int64_t n, const int64_t* keep, const int64_t* rank, int64_t* rows_of_rank,
+                                   cudaStream_t s);
+cudaError_t launch_hh_sub(const Mat& M, const int64_t* keep, const int64_t* rank, const int64_t* rows_of_rank, int64_t s_rows,
+                          int64_t* cnt_or_rp, int32_t* col, int64_t* pos, void* val /*nullable*/, int pass, cudaStream_t s);
 cudaError_t launch_gather_rows(const int64_t* src, const int64_t* rows, int64_t nr, int64_t* dst, cudaStream_t s);
 cudaError_t launch_add_offset(int64_t* x, int64_t n, int64_t off, cudaStream_t s);
 cudaError_t launch_check_rows(const int64_t* rows, int64_t nr, int64_t n, unsigned long long* bad, cudaStream_t s);

@@ -216,6 +216,7 @@ CONFIGS = {
     "C3": "R-MAT scale 20, edge factor 16 (a=0.57,b=c=0.19), C=A*A",
     "C4": "R-MAT scale 22, 8xB200 sharded",
     "R18": "R-MAT scale 18 (threshold sweep, config 5)",
+    "R18u": "R-MAT scale 18, un-permuted labels (config 5 ablation)",
 }
 
 
@@ -230,6 +231,8 @@ def config(name: str, seed: int = 1, mode: str = "real", dtype: str = "f64") -> 
         return rmat(22, 16, seed=seed, mode=mode, dtype=dtype)
     if name == "R18":
         return rmat(18, 16, seed=seed, mode=mode, dtype=dtype)
+    if name == "R18u":  # config 5's un-permuted variant (hubs at low ids; the Fig. 7 randomness ablation)
+        return rmat(18, 16, seed=seed, permute=False, mode=mode, dtype=dtype)
     if name.startswith("rmat"):
         return rmat(int(name[4:]), 16, seed=seed, mode=mode, dtype=dtype)
     raise KeyError(name)

@@ -11,7 +11,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 def _declared():
     src = open(os.path.join(ROOT, "include", "sg.h")).read()
     src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
-    return sorted(set(re.findall(r"\b(sg_[a-z_]+)\s*\(", src)))
+    return sorted(set(re.findall(r"\b(sg_[a-z_0-9]+)\s*\(", src)))
 
 
 def test_header_declares_the_north_star_calls():
