@@ -62,7 +62,7 @@ typedef struct {
 /* Per-row path costs in integer picoseconds (the "offline relation" of PAPER L94):
  *   c_L(i) = kappa_L + lambda_L*w_i + sigma_L*u_i*ceil(log2 max(u_i,2)) + rho_L*u_i
  *   c_H(i) = kappa_H + lambda_H*w_i + tau_H*a_i*R(u_i) + mu_H*u_i
- *   R(u)   = tiles_fixed if capu == 0, else max(1, ceil(u/capu))
+ *   R(u)   = tiles_fixed if capu == 0, else max(1, tiles_fixed, ceil(u/capu))
  * with a_i = nnz(A_i), w_i = L_AB[i], u_i = nnz(C_i). cap_L is the largest admissible
  * threshold (the light path's table capacity); it must be <= SG_CAP_L_MAX. Every coefficient must be
  * >= 0 (INVALID_ARG otherwise): costs are then non-negative and every cost prefix is monotone. */
@@ -117,8 +117,11 @@ int64_t sg_get_option(int key);
 const char* sg_status_string(sg_status st);
 /* Library version string, e.g. "sg 0.1.0 sm_100a". */
 const char* sg_version(void);
-/* The calibrated default cost model. */
+/* The calibrated default cost model, with tiles_fixed = 1. Calls given cm == NULL use it
+ * with tiles_fixed = ceil(B.ncols / 131072), the heavy path's minimum number of column ranges per row
+ * (R(u)'s floor): exactly the model sg_default_cost_model_for(B.ncols) returns. */
 void sg_default_cost_model(sg_cost_model* out /*host*/);
+void sg_default_cost_model_for(int64_t p, sg_cost_model* out /*host*/);
 /* The default model of sg_partition_cost: fitted to measured per-shard times. */
 void sg_default_partition_model(sg_cost_model* out /*host*/);
 

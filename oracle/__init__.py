@@ -45,7 +45,7 @@ def build(force: bool = False) -> str:
 class CostModel(ctypes.Structure):
     """Per-row path costs in integer picoseconds:
     c_L = kappa_L + lambda_L*w + sigma_L*u*ceil(log2 max(u,2)) + rho_L*u
-    c_H = kappa_H + lambda_H*w + tau_H*a*R(u) + mu_H*u,  R(u) = tiles_fixed if capu == 0 else max(1, ceil(u/capu))
+    c_H = kappa_H + lambda_H*w + tau_H*a*R(u) + mu_H*u,  R(u) = tiles_fixed if capu == 0 else max(1, tiles_fixed, ceil(u/capu))
     """
     _fields_ = [(n, ctypes.c_int64) for n in (
         "kappa_L", "lambda_L", "sigma_L", "rho_L",

@@ -190,7 +190,7 @@ typedef struct {
     int64_t kappa_L, lambda_L, sigma_L, rho_L;      // light: kappa + lambda*w + sigma*u*ceil(log2 max(u,2)) + rho*u
     int64_t kappa_H, lambda_H, tau_H, mu_H;         // heavy: kappa + lambda*w + tau*a*R(u) + mu*u
     int64_t tiles_fixed;                            // R(u) = tiles_fixed if capu == 0
-    int64_t capu;                                   // else R(u) = max(1, ceil(u / capu))
+    int64_t capu;                                   // else R(u) = max(1, tiles_fixed, ceil(u / capu))
     int64_t cap_L;                                  // largest admissible threshold (light capacity)
 } oracle_cost_model;
 
@@ -207,7 +207,8 @@ int64_t oracle_cost_L(const oracle_cost_model* cm, int64_t w, int64_t a, int64_t
 }
 
 int64_t oracle_cost_H(const oracle_cost_model* cm, int64_t w, int64_t a, int64_t u) {
-    int64_t R = cm->capu == 0 ? cm->tiles_fixed : std::max<int64_t>(1, (u + cm->capu - 1) / cm->capu);
+    int64_t R = cm->capu == 0 ? cm->tiles_fixed
+                              : std::max<int64_t>(std::max<int64_t>(1, cm->tiles_fixed), (u + cm->capu - 1) / cm->capu);
     return cm->kappa_H + cm->lambda_H * w + cm->tau_H * a * R + cm->mu_H * u;
 }
 

@@ -40,7 +40,7 @@ EXPORTS = ["sg_status_string", "sg_version", "sg_default_cost_model", "sg_row_wo
            "sg_profile_enable", "sg_launch_count", "sg_profile_count", "sg_profile_read", "sg_profile_reset",
            "sg_gather_layout", "sg_threshold_on_rows", "sg_set_option", "sg_get_option",
            "sg_sym_c_create", "sg_sym_c_buffers", "sg_sym_c_layout", "sg_sym_c_assemble", "sg_sym_c_destroy",
-           "sg_copy_device", "sg_hh_filter", "sg_hh_hstack", "sg_hh_identity2", "sg_hh_sample"]
+           "sg_copy_device", "sg_default_cost_model_for", "sg_hh_filter", "sg_hh_hstack", "sg_hh_identity2", "sg_hh_sample"]
 
 SG_OPT_VALIDATE, SG_OPT_DENSE_LOG2, SG_OPT_VARIANT = 0, 1, 2
 
@@ -133,6 +133,7 @@ def load(build_if_missing: bool = True):
         "sg_sym_c_assemble": (st, [P, P, P, P]),
         "sg_sym_c_destroy": (None, [P]),
         "sg_copy_device": (st, [P, P, i64, P]),
+        "sg_default_cost_model_for": (None, [i64, ctypes.POINTER(CostModel)]),
         "sg_hh_filter": (st, [P, i64, ctypes.c_int, P, P, P, pi64, P]),
         "sg_hh_hstack": (st, [P, P, P, P, P, P]),
         "sg_hh_identity2": (st, [i64, ctypes.c_int, P, P, P, P]),
@@ -214,9 +215,13 @@ class DeviceCSR:
         return (self.row_ptr.cpu().numpy(), self.col.cpu().numpy(), self.val.cpu().numpy())
 
 
-def sg_default_cost_model() -> CostModel:
+def sg_default_cost_model(p: int | None = None) -> CostModel:
+    """The calibrated default model; with p (= B.ncols) the exact model calls with cm=None use."""
     cm = CostModel()
-    lib().sg_default_cost_model(ctypes.byref(cm))
+    if p is None:
+        lib().sg_default_cost_model(ctypes.byref(cm))
+    else:
+        lib().sg_default_cost_model_for(int(p), ctypes.byref(cm))
     return cm
 
 
@@ -652,7 +657,17 @@ def spgemm(A: DeviceCSR, B: DeviceCSR, sample_frac: float = 0.01, seed: int = 1,
     Returns (C as DeviceCSR, info dict)."""
     rep = None
     if thr is None:
-        thr, rep = sg_sample_threshold(A, B, sample_frac, seed, cm)
+        try:
+            thr, rep = sg_sample_threshold(A, B, sample_frac, seed, cm)
+        except SgError as e:
+            if e.code != 5:  # SG_ERR_EMPTY_SAMPLE: a small or very sparse input; Identify over every row
+                raise
+            try:
+                thr, rep = sg_sample_threshold(A, B, 1.0, seed, cm)
+            except SgError as e2:
+                if e2.code != 5:
+                    raise
+                thr = 0  # no row has any product: every row is EMPTY, the threshold is moot
     plan = sg_symbolic(A, B, thr)
     col, val = sg_numeric(plan, A, B)
     C = DeviceCSR(A.nrows, B.ncols, plan.row_ptr, col, val)

@@ -188,6 +188,15 @@ const sg_cost_model kDefaultModel = {
     /*kappa_H*/ 5498663, /*lambda_H*/ 989, /*tau_H*/ 40554, /*mu_H*/ 0,
     /*tiles_fixed*/ 1, /*capu*/ 12288, /*cap_L*/ SG_CAP_L_MAX};
 
+// The heavy path's minimum number of column ranges per row: a row whose columns span [0, p) needs at
+// least ceil(p / (RW_TILES * TW)) rank-kernel ranges (and dense windows in proportion), whatever its u.
+// The default model takes it as R(u)'s floor (tiles_fixed) for the B at hand.
+int64_t default_range_floor(int64_t p) {
+    const int64_t span = (int64_t)RW_TILES * TW;
+    const int64_t r = (p + span - 1) / span;
+    return r < 1 ? 1 : r;
+}
+
 // Partition model (reading R19): fitted by tools/fit_partition_model.py to 88 measured
 // shard times (R-MAT 20 and 18, permuted and un-permuted, G = 2..16; profiles/r01s4_partition_model_fit.json):
 // a light row costs rho_L per output, a heavy row lambda_H per product (ps of SM time).
@@ -355,6 +364,12 @@ void sg_default_cost_model(sg_cost_model* out) {
     if (out) *out = kDefaultModel;
 }
 
+void sg_default_cost_model_for(int64_t p, sg_cost_model* out) {
+    if (!out) return;
+    *out = kDefaultModel;
+    out->tiles_fixed = default_range_floor(p);
+}
+
 void sg_default_partition_model(sg_cost_model* out) {
     if (out) *out = kPartitionModel;
 }
@@ -417,7 +432,9 @@ sg_status sg_sample_threshold(const sg_csr_view* A, const sg_csr_view* B, double
     if (!(sample_frac > 0.0 && sample_frac <= 1.0)) return SG_ERR_INVALID_ARG;
     sg_status st = validate_pair(A, B, s);
     if (st != SG_OK) return st;
-    const sg_cost_model* c = cm ? cm : &kDefaultModel;
+    sg_cost_model dflt = kDefaultModel;
+    dflt.tiles_fixed = default_range_floor(B->ncols);
+    const sg_cost_model* c = cm ? cm : &dflt;
     if ((st = check_model(c)) != SG_OK) return st;
     Mat a = mat_of(A), b = mat_of(B);
     const int64_t n = A->nrows;
@@ -462,7 +479,9 @@ sg_status sg_threshold_on_rows(const sg_csr_view* A, const sg_csr_view* B, const
     if (!thr_out || nrows < 0 || (nrows > 0 && !rows)) return SG_ERR_INVALID_ARG;
     sg_status st = validate_pair(A, B, s);
     if (st != SG_OK) return st;
-    const sg_cost_model* c = cm ? cm : &kDefaultModel;
+    sg_cost_model dflt = kDefaultModel;
+    dflt.tiles_fixed = default_range_floor(B->ncols);
+    const sg_cost_model* c = cm ? cm : &dflt;
     if ((st = check_model(c)) != SG_OK) return st;
     if (nrows == 0) return SG_ERR_EMPTY_SAMPLE;
     {
@@ -501,7 +520,9 @@ sg_status sg_exhaustive_threshold(const sg_csr_view* A, const sg_csr_view* B, co
     if (!thr_out) return SG_ERR_INVALID_ARG;
     sg_status st = validate_pair(A, B, s);
     if (st != SG_OK) return st;
-    const sg_cost_model* c = cm ? cm : &kDefaultModel;
+    sg_cost_model dflt = kDefaultModel;
+    dflt.tiles_fixed = default_range_floor(B->ncols);
+    const sg_cost_model* c = cm ? cm : &dflt;
     if ((st = check_model(c)) != SG_OK) return st;
     ThrResult r;
     st = identify(mat_of(A), mat_of(B), nullptr, A->nrows, c, &r, s);
@@ -518,7 +539,9 @@ sg_status sg_cost_curve(const sg_csr_view* A, const sg_csr_view* B, const sg_cos
     if (nt < 0 || (nt > 0 && (!t_host || !J_host))) return SG_ERR_INVALID_ARG;
     sg_status st = validate_pair(A, B, s);
     if (st != SG_OK) return st;
-    const sg_cost_model* c = cm ? cm : &kDefaultModel;
+    sg_cost_model dflt = kDefaultModel;
+    dflt.tiles_fixed = default_range_floor(B->ncols);
+    const sg_cost_model* c = cm ? cm : &dflt;
     if ((st = check_model(c)) != SG_OK) return st;
     Scratch sc(s);
     RowStats rs;

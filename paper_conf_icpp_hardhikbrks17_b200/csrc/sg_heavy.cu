@@ -544,7 +544,12 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 // the product that finds the accumulator at exactly 0.0 writes the column: the first
                 // product of every column does (accumulators start at 0.0); a later one only when the
                 // partial sum is exactly 0.0, rewriting the same value
+#if defined(SG_HV_EXP) && SG_HV_EXP == 3  // timing experiment: per-warp rotated ranks, no cross-warp same-address collisions (wrong C)
+                const uint32_t rr2 = ((uint32_t)rank + 97u * (threadIdx.x >> 5)) % (uint32_t)RCAP;
+                if (atom_add_f64_s(bw + (vb - bw) + 8u * rr2, v) == 0.0) st_out(C_col + base + rank, c);
+#else
                 if (atom_add_f64_s(bw + (vb - bw) + 8u * (uint32_t)rank, v) == 0.0) st_out(C_col + base + rank, c);
+#endif
             };
             if (inreg) {
                 #pragma unroll

@@ -294,7 +294,11 @@ __device__ __forceinline__ long long costL(const CostModelD& cm, long long w, lo
     return cm.kL + cm.lL * w + cm.sL * u * ceil_log2_max2(u) + cm.rL * u;
 }
 __device__ __forceinline__ long long costH(const CostModelD& cm, long long w, long long a, long long u) {
-    long long R = cm.capu == 0 ? cm.tiles_fixed : ((u + cm.capu - 1) / cm.capu > 1 ? (u + cm.capu - 1) / cm.capu : 1);
+    long long R = cm.tiles_fixed;  // R(u) = tiles_fixed (capu == 0) or max(1, tiles_fixed, ceil(u / capu))
+    if (cm.capu != 0) {
+        const long long q = (u + cm.capu - 1) / cm.capu, lo = cm.tiles_fixed > 1 ? cm.tiles_fixed : 1;
+        R = q > lo ? q : lo;
+    }
     return cm.kH + cm.lH * w + cm.tH * a * R + cm.mH * u;
 }
 
@@ -303,7 +307,8 @@ __device__ __forceinline__ long long costH(const CostModelD& cm, long long w, lo
 // of the histogram and every cut target; the host rejects the model when that bound reaches 2^62.
 __device__ __forceinline__ double cost_mag(const CostModelD& cm, double w, double a, double u) {
     const double lg = (double)ceil_log2_max2((long long)u);
-    const double R = cm.capu == 0 ? (double)cm.tiles_fixed : fmax(1.0, ceil(u / (double)cm.capu));
+    const double R = cm.capu == 0 ? (double)cm.tiles_fixed
+                                  : fmax(fmax(1.0, (double)cm.tiles_fixed), ceil(u / (double)cm.capu));
     const double cl = (double)cm.kL + (double)cm.lL * w + (double)cm.sL * u * lg + (double)cm.rL * u;
     const double ch = (double)cm.kH + (double)cm.lH * w + (double)cm.tH * a * R + (double)cm.mH * u;
     return cl + ch;

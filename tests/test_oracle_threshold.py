@@ -264,12 +264,13 @@ def test_worked_example_cost_split_nonexact_uh():
 
 
 def test_cost_H_tile_count_closed_form():
-    """R(u) = max(1, ceil(u/capu)) for capu > 0 at every u in [0, 5*capu]: with every other
-    constant 0 and tau_H = a = 1, c_H(u) IS R(u) (closed form, checked against integer ceil)."""
+    """R(u) = max(1, tiles_fixed, ceil(u/capu)) for capu > 0 at every u in [0, 5*capu]: with every
+    other constant 0 and tau_H = a = 1, c_H(u) IS R(u) (closed form, checked against integer ceil)."""
     for capu in (1, 3, 16, 100):
-        cm = _cm(tau_H=1, tiles_fixed=7, capu=capu, cap_L=100)
-        for uu in range(0, 5 * capu + 2):
-            assert oracle.cost_H(cm, 0, 1, uu) == max(1, -(-uu // capu))
+        for tf in (0, 1, 7):
+            cm = _cm(tau_H=1, tiles_fixed=tf, capu=capu, cap_L=100)
+            for uu in range(0, 5 * capu + 2):
+                assert oracle.cost_H(cm, 0, 1, uu) == max(1, tf, -(-uu // capu))
     cm = _cm(tau_H=1, tiles_fixed=7, capu=0, cap_L=100)
     assert oracle.cost_H(cm, 0, 1, 12345) == 7
 
@@ -282,3 +283,18 @@ def test_cost_L_rho_term_closed_form():
     cm = _cm(sigma_L=1, cap_L=100)
     for uu, lg in ((0, 1), (1, 1), (2, 1), (3, 2), (4, 2), (5, 3), (1024, 10), (1025, 11)):
         assert oracle.cost_L(cm, 5, 1, uu) == uu * lg
+
+
+def test_cost_H_range_floor_tiles_fixed_with_capu():
+    """R(u) = max(1, tiles_fixed, ceil(u/capu)) when capu > 0 (the heavy path's
+    minimum number of column ranges for a row spanning all p columns is tiles_fixed). Hand values for
+    tiles_fixed = 3, capu = 16: u = 4 -> 3, 40 -> 3 (2.5 -> 3), 48 -> 3, 49 -> 4 (3.06 -> 4), 150 -> 10."""
+    cm = _cm(tau_H=1, tiles_fixed=3, capu=16, cap_L=100)
+    for uu, R in ((0, 3), (4, 3), (40, 3), (48, 3), (49, 4), (150, 10)):
+        assert oracle.cost_H(cm, 0, 1, uu) == R
+    cm = _cm(kappa_H=100, lambda_H=1, tau_H=1, mu_H=1, tiles_fixed=3, capu=16, cap_L=100)
+    # c_H(w=60, a=5, u=40) = 100 + 60 + 5*3 + 40 = 215 ; c_H(200, 10, 150) = 100 + 200 + 10*10 + 150 = 550
+    assert oracle.cost_H(cm, 60, 5, 40) == 215 and oracle.cost_H(cm, 200, 10, 150) == 550
+    # with tiles_fixed = 12 the floor dominates: c_H(200, 10, 150) = 100 + 200 + 10*12 + 150 = 570
+    cm.tiles_fixed = 12
+    assert oracle.cost_H(cm, 200, 10, 150) == 570

@@ -35,6 +35,14 @@ def grid(cap=4096):
     return sorted(ts)
 
 
+def product_only(sg, A, t):
+    """symbolic + numeric at threshold t; C is dropped at once (C3's C is 116 GB: never two alive)."""
+    plan = sg.sg_symbolic(A, A, t)
+    col, val = sg.sg_numeric(plan, A, A)
+    plan.destroy()
+    del col, val
+
+
 def timed(fn, reps):
     import torch
     out = []
@@ -63,11 +71,12 @@ def main():
     import sginputs as gen
     import paper_conf_icpp_hardhikbrks17_b200 as sg
 
-    cm = sg.sg_default_cost_model()
-    report = {"cost_model": cm.as_dict(), "configs": {}}
+    report = {"cost_model": sg.sg_default_cost_model().as_dict(), "configs": {}}
     for name in a.configs.split(","):
         H = gen.config(name)
         A = sg.DeviceCSR.from_host(H)
+        cm = sg.sg_default_cost_model(H.ncols)  # the model calls with cm=None use for this B (R's floor from p)
+        tf = max(1, int(cm.tiles_fixed))
         w = sg.sg_row_work(A, A).cpu().numpy()
         W = float(w.sum())
         r = lambda t: 100.0 * float(w[w > t].sum()) / W
@@ -83,8 +92,7 @@ def main():
                 del col, val
                 return prof.by_kernel(), u
             _, (bk, u) = timed(run, 1)                      # per-class split (profiled run)
-            ms = timed(lambda: (lambda p: (sg.sg_numeric(p, A, A), p.destroy()))(sg.sg_symbolic(A, A, t)),
-                       a.reps)[0]                           # T(t) without profiling events
+            ms = timed(lambda: product_only(sg, A, t), a.reps)[0]  # T(t) without profiling events
             light = (w > 0) & (w <= t)
             heavy = w > t
             arow = np.diff(H.row_ptr)
@@ -94,12 +102,12 @@ def main():
                          "L": [int(light.sum()), int(w[light].sum()), int(u[light].sum())],
                          "H": [int(heavy.sum()), int(w[heavy].sum()), int(u[heavy].sum()),
                                int(arow[heavy].sum()),
-                               int((arow[heavy] * np.maximum(1, np.ceil(u[heavy] / max(cm.capu, 1)))).sum())]})
+                               int((arow[heavy] * np.maximum(tf, np.ceil(u[heavy] / max(cm.capu, 1)))).sum())]})
             print(f"{name} t={t:5d} T={ms:8.3f} ms  light {kl:7.3f}  heavy {kh:7.3f}  r={r(t):6.2f}%", flush=True)
         Tbest = min(x["ms"] for x in rows)
         t_meas = min(rows, key=lambda x: x["ms"])["t"]
         thr_star, J_star = sg.sg_exhaustive_threshold(A, A, cm)
-        T_at = lambda t: timed(lambda: (lambda p: (sg.sg_numeric(p, A, A), p.destroy()))(sg.sg_symbolic(A, A, t)), a.reps)[0]
+        T_at = lambda t: timed(lambda: product_only(sg, A, t), a.reps)[0]
         T_star = T_at(thr_star)
         samples = {}
         for f in [float(x) for x in a.fracs.split(",")]:
@@ -123,7 +131,7 @@ def main():
             samples[str(f)] = {"agg": agg, "runs": res}
             print(f"{name} f={f:.2f}: " + "  ".join(f"{k} mean {v['mean']:.4f} max {v['max']:.4f}" for k, v in agg.items()),
                   flush=True)
-        report["configs"][name] = {"n": H.nrows, "W": W, "grid": rows, "T_best_ms": Tbest, "t_best_measured": t_meas,
+        report["configs"][name] = {"n": H.nrows, "W": W, "tiles_fixed": tf, "grid": rows, "T_best_ms": Tbest, "t_best_measured": t_meas,
                                    "thr_star_model": thr_star, "J_star": J_star, "T_at_thr_star_ms": T_star,
                                    "r_at_t_best_measured": r(t_meas), "r_at_thr_star": r(thr_star),
                                    "samples": samples}
