@@ -39,6 +39,8 @@ struct sg_plan {
     int2* span = nullptr;           // light rows: [cmin, cmax] of the output columns
     int4* gscr = nullptr;           // heavy rows with more than KC entries: per-k cursor scratch
     void* pscr = nullptr;           // dense2: per-CTA part scratch for rows with many k entries
+    int32_t* bcol_tag = nullptr;    // dense2: B.col with hot columns tagged (nullptr: privatisation off)
+    int32_t* hotcols = nullptr;     // dense2: the hot column of every (window, slot)
     int64_t pscr_cap = 0;
     int variant = 0;
     int32_t* long_id = nullptr;
@@ -180,12 +182,14 @@ CostModelD cm_of(const sg_cost_model* c) {
 
 // Default model: calibrated from the measured kernels (profiles/).
 // Refitted in round 2 on the round-2 kernels (sg_sym2.cu, sg_dense2.cu) by tools/sweep.py: non-negative
-// least squares of the per-class kernel times over the threshold grid on ER 2^18, R-MAT 18 and
-// un-permuted R-MAT 18 (profiles/r02_sweep_precal.json "fit"), in ps of SM time. (Round 1's constants,
-// fitted before the heavy kernels changed: 33399, 7915, 0, 0, 17907513, 1102, 68338, 209.)
+// least squares of the per-class kernel times over the threshold grids of ER 2^18, R-MAT 18, un-permuted
+// R-MAT 18 and R-MAT 20 (C3) together, with R(u)'s floor tiles_fixed = ceil(p / 131072) per matrix
+// (profiles/r02_sweep_fitall.json "fit"), in ps of SM time. tiles_fixed here is the p <= 131072 value;
+// calls with cm == NULL use default_range_floor(B.ncols). (Round 1's constants, fitted before the heavy
+// kernels changed: 33399, 7915, 0, 0, 17907513, 1102, 68338, 209 with R(u) = max(1, ceil(u/12288)).)
 const sg_cost_model kDefaultModel = {
-    /*kappa_L*/ 0, /*lambda_L*/ 10450, /*sigma_L*/ 0, /*rho_L*/ 0,
-    /*kappa_H*/ 5498663, /*lambda_H*/ 989, /*tau_H*/ 40554, /*mu_H*/ 0,
+    /*kappa_L*/ 0, /*lambda_L*/ 9315, /*sigma_L*/ 0, /*rho_L*/ 0,
+    /*kappa_H*/ 5016705, /*lambda_H*/ 0, /*tau_H*/ 74786, /*mu_H*/ 1854,
     /*tiles_fixed*/ 1, /*capu*/ 12288, /*cap_L*/ SG_CAP_L_MAX};
 
 // The heavy path's minimum number of column ranges per row: a row whose columns span [0, p) needs at
@@ -349,7 +353,7 @@ sg_status sg_set_option(int key, int64_t value) {
     if (key < 0 || key >= SG_OPT_COUNT) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_VALIDATE && value != 0 && value != 1) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_DENSE_LOG2 && (value < -1 || value > 62)) return SG_ERR_INVALID_ARG;
-    if (key == SG_OPT_VARIANT && (value < 0 || value > 3)) return SG_ERR_INVALID_ARG;
+    if (key == SG_OPT_VARIANT && (value < 0 || value > 7)) return SG_ERR_INVALID_ARG;
     g_opt[key] = value;
     return SG_OK;
 }
@@ -725,6 +729,32 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
             pl->pscr = palloc(pl, dense2_part_bytes() * (size_t)pl->pscr_cap * 148);
             if (!pl->pscr) return fail(SG_ERR_OOM);
         }
+        // dense2 hot-column privatisation (sg_dense2.cu): columns of B whose in-degree is in the top
+        // ~40 per 24576-column window (and >= 64) get per-warp partial sums. Needs columns < 2^24.
+        if (pl->ndw > 0 && pl->p <= (1 << 24) && !(pl->variant & 4)) {
+            unsigned int* cnt = (unsigned int*)palloc(pl, sizeof(unsigned int) * (size_t)pl->p);
+            unsigned long long* hist = (unsigned long long*)palloc(pl, sizeof(unsigned long long) * 33);
+            if (!cnt || !hist) return fail(SG_ERR_OOM);
+            CKF(launch_dense2_hot(b, cnt, hist, 0, 0, nullptr, nullptr, nullptr, s));
+            unsigned long long hh2[33];
+            CKF(cudaMemcpyAsync(hh2, hist, sizeof(hh2), cudaMemcpyDeviceToHost, s));
+            CKF(cudaStreamSynchronize(s));
+            const int64_t nwin2 = (pl->p + dense2_window() - 1) / dense2_window();
+            int bsel = -1;
+            unsigned long long above = 0;
+            for (int bb2 = 32; bb2 >= 6; --bb2) {  // smallest 2^bb2 (>= 64) with <= 40 columns per window above it
+                above += hh2[bb2];
+                if (above > (unsigned long long)(40 * nwin2)) break;
+                if (above > 0) bsel = bb2;
+            }
+            if (bsel >= 0) {
+                int8_t* slot_of = (int8_t*)palloc(pl, (size_t)pl->p);
+                pl->hotcols = (int32_t*)palloc(pl, sizeof(int32_t) * (size_t)nwin2 * dense2_hot_slots());
+                pl->bcol_tag = (int32_t*)palloc(pl, sizeof(int32_t) * (size_t)(b.nnz > 0 ? b.nnz : 1));
+                if (!slot_of || !pl->hotcols || !pl->bcol_tag) return fail(SG_ERR_OOM);
+                CKF(launch_dense2_hot(b, cnt, hist, 1, 1u << bsel, slot_of, pl->hotcols, pl->bcol_tag, s));
+            }
+        }
         if (pl->amax > heavy_kc() || pl->amax > dense_kc()) {
             pl->gscr = (int4*)palloc(pl, sizeof(int4) * (size_t)(heavy_grid() > dense_grid() ? heavy_grid() : dense_grid()) * (size_t)pl->amax);
             if (!pl->gscr) return fail(SG_ERR_OOM);
@@ -779,7 +809,7 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
         else
             CKP(pl, launch_num_dense2(a, b, pl->heavy, pl->ndw, pl->rb, pl->w, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
                                       C_val, pl->counter, pl->pscr, pl->pscr_cap, pl->dtc, pl->ditems,
-                                      pl->ditem_off + pl->ndw, s));
+                                      pl->ditem_off + pl->ndw, pl->bcol_tag, pl->hotcols, s));
         CKP(pl, launch_num_heavy(a, b, pl->heavy, pl->ndw, pl->nheavy, pl->rb, pl->range_off, pl->nranges, pl->ranges,
                                  pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter, pl->gscr, pl->amax, s));
     }

@@ -592,6 +592,7 @@ __device__ __forceinline__ int part_seg_end(const Mat& B, const Part& pt, uint32
 // time. (sg_dense2.cu; a software-pipelined variant that gathers the next SEG_UNR batches during the accumulation of
 // the current ones measured slower: 33.4 vs 31.7 ms on C3 rows/2, profiles/r02_dense2_ab.txt.)
 constexpr int SEG_LONG = 128;
+constexpr int32_t SEG_NONE = INT_MAX;  // no product (a column is < INT32_MAX; tagged columns are negative)
 constexpr int SEG_UNR = 4;
 template <bool VAL, class VT, class F>
 __device__ __forceinline__ void seg_walk(const Mat& B, int beg, int len, double a, F&& acc) {
@@ -610,7 +611,7 @@ __device__ __forceinline__ void seg_walk(const Mat& B, int beg, int len, double 
             #pragma unroll
             for (int r = 0; r < 4; ++r) {
                 const int jj = j + 32 * r;
-                c[r] = -1;
+                c[r] = SEG_NONE;
                 v[r] = 0.0;
                 if (jj < n) {
                     c[r] = __ldg(bcol + b + jj);
@@ -619,7 +620,7 @@ __device__ __forceinline__ void seg_walk(const Mat& B, int beg, int len, double 
             }
             #pragma unroll
             for (int r = 0; r < 4; ++r)
-                if (c[r] >= 0) acc(c[r], v[r]);
+                if (c[r] != SEG_NONE) acc(c[r], v[r]);
         }
     }
     const int sl = len < SEG_LONG ? len : 0;
@@ -640,7 +641,7 @@ __device__ __forceinline__ void seg_walk(const Mat& B, int beg, int len, double 
             }
             const int q = __shfl_sync(FULL, beg, s) + (j - __shfl_sync(FULL, off, s));
             const double as = __shfl_sync(FULL, a, s);
-            c[r] = -1;
+            c[r] = SEG_NONE;
             v[r] = 0.0;
             if (j < tot) {
                 c[r] = __ldg(bcol + q);
@@ -649,7 +650,7 @@ __device__ __forceinline__ void seg_walk(const Mat& B, int beg, int len, double 
         }
         #pragma unroll
         for (int r = 0; r < SEG_UNR; ++r)
-            if (c[r] >= 0) acc(c[r], v[r]);
+            if (c[r] != SEG_NONE) acc(c[r], v[r]);
     }
 }
 
