@@ -39,8 +39,6 @@ struct sg_plan {
     int2* span = nullptr;           // light rows: [cmin, cmax] of the output columns
     int4* gscr = nullptr;           // heavy rows with more than KC entries: per-k cursor scratch
     void* pscr = nullptr;           // dense2: per-CTA part scratch for rows with many k entries
-    int32_t* bcol_tag = nullptr;    // dense2: B.col with hot columns tagged (nullptr: privatisation off)
-    int32_t* hotcols = nullptr;     // dense2: the hot column of every (window, slot)
     int64_t pscr_cap = 0;
     int variant = 0;
     int32_t* long_id = nullptr;
@@ -353,7 +351,7 @@ sg_status sg_set_option(int key, int64_t value) {
     if (key < 0 || key >= SG_OPT_COUNT) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_VALIDATE && value != 0 && value != 1) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_DENSE_LOG2 && (value < -1 || value > 62)) return SG_ERR_INVALID_ARG;
-    if (key == SG_OPT_VARIANT && (value < 0 || value > 7)) return SG_ERR_INVALID_ARG;
+    if (key == SG_OPT_VARIANT && (value < 0 || value > 3)) return SG_ERR_INVALID_ARG;
     g_opt[key] = value;
     return SG_OK;
 }
@@ -729,32 +727,6 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
             pl->pscr = palloc(pl, dense2_part_bytes() * (size_t)pl->pscr_cap * 148);
             if (!pl->pscr) return fail(SG_ERR_OOM);
         }
-        // dense2 hot-column privatisation (sg_dense2.cu): columns of B whose in-degree is in the top
-        // ~40 per 24576-column window (and >= 64) get per-warp partial sums. Needs columns < 2^24.
-        if (pl->ndw > 0 && pl->p <= (1 << 24) && !(pl->variant & 4)) {
-            unsigned int* cnt = (unsigned int*)palloc(pl, sizeof(unsigned int) * (size_t)pl->p);
-            unsigned long long* hist = (unsigned long long*)palloc(pl, sizeof(unsigned long long) * 33);
-            if (!cnt || !hist) return fail(SG_ERR_OOM);
-            CKF(launch_dense2_hot(b, cnt, hist, 0, 0, nullptr, nullptr, nullptr, s));
-            unsigned long long hh2[33];
-            CKF(cudaMemcpyAsync(hh2, hist, sizeof(hh2), cudaMemcpyDeviceToHost, s));
-            CKF(cudaStreamSynchronize(s));
-            const int64_t nwin2 = (pl->p + dense2_window() - 1) / dense2_window();
-            int bsel = -1;
-            unsigned long long above = 0;
-            for (int bb2 = 32; bb2 >= 6; --bb2) {  // smallest 2^bb2 (>= 64) with <= 40 columns per window above it
-                above += hh2[bb2];
-                if (above > (unsigned long long)(40 * nwin2)) break;
-                if (above > 0) bsel = bb2;
-            }
-            if (bsel >= 0) {
-                int8_t* slot_of = (int8_t*)palloc(pl, (size_t)pl->p);
-                pl->hotcols = (int32_t*)palloc(pl, sizeof(int32_t) * (size_t)nwin2 * dense2_hot_slots());
-                pl->bcol_tag = (int32_t*)palloc(pl, sizeof(int32_t) * (size_t)(b.nnz > 0 ? b.nnz : 1));
-                if (!slot_of || !pl->hotcols || !pl->bcol_tag) return fail(SG_ERR_OOM);
-                CKF(launch_dense2_hot(b, cnt, hist, 1, 1u << bsel, slot_of, pl->hotcols, pl->bcol_tag, s));
-            }
-        }
         if (pl->amax > heavy_kc() || pl->amax > dense_kc()) {
             pl->gscr = (int4*)palloc(pl, sizeof(int4) * (size_t)(heavy_grid() > dense_grid() ? heavy_grid() : dense_grid()) * (size_t)pl->amax);
             if (!pl->gscr) return fail(SG_ERR_OOM);
@@ -809,7 +781,7 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
         else
             CKP(pl, launch_num_dense2(a, b, pl->heavy, pl->ndw, pl->rb, pl->w, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
                                       C_val, pl->counter, pl->pscr, pl->pscr_cap, pl->dtc, pl->ditems,
-                                      pl->ditem_off + pl->ndw, pl->bcol_tag, pl->hotcols, s));
+                                      pl->ditem_off + pl->ndw, s));
         CKP(pl, launch_num_heavy(a, b, pl->heavy, pl->ndw, pl->nheavy, pl->rb, pl->range_off, pl->nranges, pl->ranges,
                                  pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter, pl->gscr, pl->amax, s));
     }

@@ -24,8 +24,7 @@ constexpr int D2_TILES = 3;                // TW-column tiles per window
 constexpr int D2_WD = D2_TILES * TW;       // 24576 columns per window (192 KB fp64 accumulator)
 constexpr int D2_WORDS = D2_WD / 32;       // occupancy words
 constexpr int D2_CPT = D2_WD / D2_T;       // columns per thread in the emission
-constexpr int D2_PCAP = 560;               // parts held in shared memory
-constexpr int D2_HOT = 64;                 // privatised hot columns per window (see k_num_dense2)
+constexpr int D2_PCAP = 1216;              // parts held in shared memory
 static_assert(D2_CPT * D2_T == D2_WD && D2_CPT <= 32, "emission: D2_CPT columns per thread");
 
 using D2Part = Part;
@@ -34,8 +33,6 @@ struct D2Smem {
     double vals[D2_WD];
     uint32_t bm[D2_WORDS + 1];  // +1 pad word for the two-word emission read
     D2Part parts[D2_PCAP];
-    double priv[D2_NW][D2_HOT];         // per-warp partial sums of the window's hot columns
-    uint32_t touched[D2_NW][D2_HOT / 32];  // which of them received a product
     int32_t wpart[D2_NW + 1];   // warp w owns parts [wpart[w], wpart[w+1])
     long long wsll[33];
     int ws[33];
@@ -59,7 +56,7 @@ __global__ void __launch_bounds__(D2_T, 1) k_num_dense2(
     const int32_t* __restrict__ long_id, const uint32_t* __restrict__ tp, int T, const int64_t* __restrict__ C_rp,
     int32_t* __restrict__ C_col, VT* __restrict__ C_val, unsigned long long* counter, D2Part* __restrict__ pscr,
     int64_t pscr_cap, const int32_t* __restrict__ dtc, const int4* __restrict__ items,
-    const int64_t* __restrict__ nitems, const int32_t* __restrict__ bcol_tag, const int32_t* __restrict__ hotcols) {
+    const int64_t* __restrict__ nitems) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     D2Smem& S = *reinterpret_cast<D2Smem*>(smem_raw);
     __shared__ long long s_j;
@@ -68,16 +65,6 @@ __global__ void __launch_bounds__(D2_T, 1) k_num_dense2(
     const uint32_t a_vals = smem_addr(S.vals), a_bm = smem_addr(S.bm);
     for (int q = tid; q < D2_WD; q += D2_T) S.vals[q] = 0.0;
     for (int q = tid; q < D2_WORDS + 1; q += D2_T) S.bm[q] = 0u;
-    for (int q = tid; q < D2_NW * D2_HOT; q += D2_T) (&S.priv[0][0])[q] = 0.0;
-    for (int q = tid; q < D2_NW * D2_HOT / 32; q += D2_T) (&S.touched[0][0])[q] = 0u;
-    // hot-column privatisation (bcol_tag != nullptr): B.col with bit 31 set and the column's slot in
-    // bits 24-29 for the <= D2_HOT most in-demand columns of each window (in-degree in B at or above a
-    // threshold; sg_symbolic builds it). Their products go to a per-warp partial sum instead of the
-    // shared accumulator (profiles/r02_dense2_ab.txt — same-column CAS contention across the
-    // 32 warps cost 26 % of this kernel: hub columns take up to 14540 products in one row).
-    Mat Bt = B;
-    if (bcol_tag) Bt.col = bcol_tag;
-    const uint32_t a_priv = smem_addr(&S.priv[wid][0]), a_touch = smem_addr(&S.touched[wid][0]);
     const int64_t n_items = *nitems;
 #if defined(SG_D2_EXP) && SG_D2_EXP == 8
     unsigned long long ph[6] = {0, 0, 0, 0, 0, 0};
@@ -142,12 +129,6 @@ __global__ void __launch_bounds__(D2_T, 1) k_num_dense2(
                 const uint32_t cc = (uint32_t)(c - (int)lo + 97 * (int)(threadIdx.x >> 5)) % (uint32_t)D2_WD;
                 if (atom_add_f64_s_nc(a_vals + 8u * cc, v) == 0.0) red_or_s_nc(bb + 4u * ((uint32_t)c >> 5), 1u << (c & 31));
 #else
-                if (c < 0) {  // tagged hot column: the warp's private partial sum (folded at the window end)
-                    const uint32_t sl = ((uint32_t)c >> 24) & (D2_HOT - 1);
-                    atom_add_f64_s(a_priv + 8u * sl, v);
-                    red_or_s(a_touch + 4u * (sl >> 5), 1u << (sl & 31));
-                    return;
-                }
                 if (atom_add_f64_s(vb + 8u * (uint32_t)c, v) == 0.0) red_or_s(bb + 4u * ((uint32_t)c >> 5), 1u << (c & 31));
 #endif
             };
@@ -176,24 +157,10 @@ __global__ void __launch_bounds__(D2_T, 1) k_num_dense2(
                 }
                 if (g == pw0 && lid0 >= 0 && t + 1 < tb)
                     tpn = __ldg(tp + (int64_t)lid0 * (T + 1) + min((t + 2) * D2_TILES, T));
-                seg_walk<true, VT>(Bt, beg, len, a, acc);
+                seg_walk<true, VT>(B, beg, len, a, acc);
             }
             D2_MARK(1);
             __syncthreads();  // window t accumulated
-            if (bcol_tag) {
-                // fold the per-warp hot partial sums into the accumulator (at most D2_NW adds per column)
-                for (int q = tid; q < D2_NW * D2_HOT; q += D2_T) {
-                    const int w2 = q / D2_HOT, sl = q % D2_HOT;
-                    if (S.touched[w2][sl >> 5] & (1u << (sl & 31))) {
-                        const int c = hotcols[(int64_t)t * D2_HOT + sl];
-                        atom_add_f64_s(vb + 8u * (uint32_t)c, S.priv[w2][sl]);
-                        red_or_s(bb + 4u * ((uint32_t)c >> 5), 1u << (c & 31));  // the column has a product
-                        S.priv[w2][sl] = 0.0;
-                    }
-                }
-                __syncthreads();  // every fold done (and every touched word read) before the emission
-                for (int q = tid; q < D2_NW * D2_HOT / 32; q += D2_T) (&S.touched[0][0])[q] = 0u;
-            }
             D2_MARK(2);
 #ifndef SG_D2_EMIT
 #define SG_D2_EMIT 1
@@ -287,8 +254,7 @@ __global__ void __launch_bounds__(D2_T, 1) k_num_dense2(
 cudaError_t launch_num_dense2(const Mat& A, const Mat& B, const int32_t* heavy, int64_t ndw, int64_t rb,
                               const int64_t* w, const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp,
                               int32_t* C_col, void* C_val, unsigned long long* counter, void* pscr, int64_t pscr_cap,
-                              const int32_t* dtc, const int4* items, const int64_t* nitems, const int32_t* bcol_tag,
-                              const int32_t* hotcols, cudaStream_t s) {
+                              const int32_t* dtc, const int4* items, const int64_t* nitems, cudaStream_t s) {
     if (ndw <= 0) return cudaSuccess;
     const int smem = (int)sizeof(D2Smem);
     cudaError_t e = cudaMemsetAsync(counter, 0, sizeof(unsigned long long), s);  // item counter
@@ -298,12 +264,12 @@ cudaError_t launch_num_dense2(const Mat& A, const Mat& B, const int32_t* heavy, 
         if ((e = cudaFuncSetAttribute(k_num_dense2<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
         SG_LAUNCH("k_num_dense", s, (k_num_dense2<double><<<grid, D2_T, smem, s>>>(A, B, heavy, rb, w, long_id, tp, T, C_rp, C_col,
                                                                                  (double*)C_val, counter, (D2Part*)pscr,
-                                                                                 pscr_cap, dtc, items, nitems, bcol_tag, hotcols)));
+                                                                                 pscr_cap, dtc, items, nitems)));
     } else {
         if ((e = cudaFuncSetAttribute(k_num_dense2<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
         SG_LAUNCH("k_num_dense", s, (k_num_dense2<float><<<grid, D2_T, smem, s>>>(A, B, heavy, rb, w, long_id, tp, T, C_rp, C_col,
                                                                                 (float*)C_val, counter, (D2Part*)pscr,
-                                                                                pscr_cap, dtc, items, nitems, bcol_tag, hotcols)));
+                                                                                pscr_cap, dtc, items, nitems)));
     }
 #if defined(SG_D2_EXP) && SG_D2_EXP == 8
     {
@@ -318,77 +284,5 @@ cudaError_t launch_num_dense2(const Mat& A, const Mat& B, const int32_t* heavy, 
 #endif
     return cudaGetLastError();
 }
-
-// ---- hot columns of the dense-window kernel ------------------------------------------------------
-__global__ void k_colcount(Mat B, unsigned int* __restrict__ cnt) {
-    for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < B.nnz; q += (int64_t)gridDim.x * blockDim.x)
-        atomicAdd(&cnt[__ldg(B.col + q)], 1u);
-}
-
-__global__ void k_cnt_hist(const unsigned int* __restrict__ cnt, int64_t p, unsigned long long* hist /*33*/) {
-    __shared__ unsigned int sh[33];
-    if (threadIdx.x < 33) sh[threadIdx.x] = 0;
-    __syncthreads();
-    for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < p; c += (int64_t)gridDim.x * blockDim.x) {
-        const unsigned int v = cnt[c];
-        if (v) atomicAdd(&sh[31 - __clz(v)], 1u);
-    }
-    __syncthreads();
-    if (threadIdx.x < 33 && sh[threadIdx.x]) atomicAdd(&hist[threadIdx.x], (unsigned long long)sh[threadIdx.x]);
-}
-
-// one 1024-thread block per window: the window's columns with in-degree >= H get slots 0, 1, ... in column
-// order (the first D2_HOT of them; the rest stay on the shared accumulator)
-__global__ void __launch_bounds__(D2_T) k_hot_slots(const unsigned int* __restrict__ cnt, int64_t p, unsigned int H,
-                                                    int8_t* __restrict__ slot_of, int32_t* __restrict__ hotcols) {
-    __shared__ int ws[33];
-    const int64_t lo = (int64_t)blockIdx.x * D2_WD;
-    const int64_t c0 = lo + (int64_t)threadIdx.x * D2_CPT;
-    uint32_t m = 0;
-    for (int k = 0; k < D2_CPT; ++k)
-        if (c0 + k < p && cnt[c0 + k] >= H) m |= 1u << k;
-    int tot;
-    int r = block_scan1<D2_T, int>(__popc(m), &tot, ws);
-    for (int k = 0; k < D2_CPT; ++k) {
-        if (c0 + k >= p) break;
-        int8_t sl = -1;
-        if (m & (1u << k)) {
-            if (r < D2_HOT) {
-                sl = (int8_t)r;
-                hotcols[(int64_t)blockIdx.x * D2_HOT + r] = (int32_t)(c0 + k);
-            }
-            ++r;
-        }
-        slot_of[c0 + k] = sl;
-    }
-}
-
-__global__ void k_tag_cols(Mat B, const int8_t* __restrict__ slot_of, int32_t* __restrict__ tag) {
-    for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < B.nnz; q += (int64_t)gridDim.x * blockDim.x) {
-        const int32_t c = __ldg(B.col + q);
-        const int sl = slot_of[c];
-        tag[q] = sl >= 0 ? (int32_t)(0x80000000u | ((uint32_t)sl << 24) | (uint32_t)c) : c;
-    }
-}
-
-cudaError_t launch_dense2_hot(const Mat& B, unsigned int* cnt, unsigned long long* hist, int stage, unsigned int H,
-                              int8_t* slot_of, int32_t* hotcols, int32_t* tag, cudaStream_t s) {
-    const int64_t p = B.ncols;
-    cudaError_t e;
-    if (stage == 0) {  // in-degrees and their log2 histogram
-        if ((e = cudaMemsetAsync(cnt, 0, sizeof(unsigned int) * (size_t)p, s)) != cudaSuccess) return e;
-        if ((e = cudaMemsetAsync(hist, 0, sizeof(unsigned long long) * 33, s)) != cudaSuccess) return e;
-        if (B.nnz > 0) SG_LAUNCH("k_colcount", s, (k_colcount<<<grid_for(B.nnz, 256, 148 * 8), 256, 0, s>>>(B, cnt)));
-        SG_LAUNCH("k_cnt_hist", s, (k_cnt_hist<<<grid_for(p, 256, 148 * 4), 256, 0, s>>>(cnt, p, hist)));
-        return cudaGetLastError();
-    }
-    const int nwin = (int)((p + D2_WD - 1) / D2_WD);  // stage 1: slots and the tagged B.col
-    SG_LAUNCH("k_hot_slots", s, (k_hot_slots<<<nwin, D2_T, 0, s>>>(cnt, p, H, slot_of, hotcols)));
-    if (B.nnz > 0) SG_LAUNCH("k_tag_cols", s, (k_tag_cols<<<grid_for(B.nnz, 256, 148 * 8), 256, 0, s>>>(B, slot_of, tag)));
-    return cudaGetLastError();
-}
-
-int dense2_hot_slots() { return D2_HOT; }
-int dense2_window() { return D2_WD; }
 
 }  // namespace sg

@@ -136,15 +136,7 @@ cudaError_t launch_num_dense(const Mat& A, const Mat& B, const int32_t* heavy, i
 cudaError_t launch_num_dense2(const Mat& A, const Mat& B, const int32_t* heavy, int64_t ndw, int64_t rb,
                               const int64_t* w, const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp,
                               int32_t* C_col, void* C_val, unsigned long long* counter, void* pscr, int64_t pscr_cap,
-                              const int32_t* dtc, const int4* items, const int64_t* nitems,
-                              const int32_t* bcol_tag /*nullable: no hot-column privatisation*/, const int32_t* hotcols,
-                              cudaStream_t s);
-// hot columns of the dense-window kernel: stage 0 = in-degrees of B + log2 histogram (hist: 33 entries),
-// stage 1 = per-window slots of the columns with in-degree >= H and the tagged copy of B.col
-cudaError_t launch_dense2_hot(const Mat& B, unsigned int* cnt, unsigned long long* hist, int stage, unsigned int H,
-                              int8_t* slot_of, int32_t* hotcols, int32_t* tag, cudaStream_t s);
-int dense2_hot_slots();
-int dense2_window();
+                              const int32_t* dtc, const int4* items, const int64_t* nitems, cudaStream_t s);
 size_t dense2_part_bytes();
 int dense2_pcap();
 // dense-window work items (row, window range): at most dense_items_bound(ndw, p); off[ndw] = count
