@@ -51,7 +51,10 @@ def main():
         tot = sum(v[1] for v in bk.values())
         rows = torch.repeat_interleave(torch.arange(re, device=col.device, dtype=torch.int64),
                                        torch.diff(plan.row_ptr)) if plan.nnz < 2**31 else None
-        dig = {"nnz": plan.nnz, "colsum": int(col.sum(dtype=torch.int64)), "valsum": float(val.double().sum())}
+        step = 1 << 29  # chunked: C3's C has 9.7e9 entries
+        dig = {"nnz": plan.nnz,
+               "colsum": sum(int(col[i:i + step].sum(dtype=torch.int64)) for i in range(0, col.numel(), step)),
+               "valsum": sum(float(val[i:i + step].double().sum()) for i in range(0, val.numel(), step))}
         if rows is not None:
             dig["hash"] = int(((rows * 1000003 + col.long()) * 0x9E3779B1 % (2**61 - 1)).sum())
         print(f"variant={var} dense_log2={dl} (n_dense {info['n_dense']}) rows [0,{re}) thr={thr} wall {t*1e3:.1f} ms "
