@@ -106,7 +106,8 @@ typedef struct sg_plan sg_plan;   /* opaque; owns only its workspace */
  *                      dense-window numeric kernel; 62 disables that path.
  *   SG_OPT_VARIANT     kernel variant bits for A/B measurements (0 = the default kernels; bit 0: the
  *                      previous dense-window kernel, sg_dense.cu; bit 1: the previous heavy symbolic
- *                      kernel, k_sym_heavy in sg_heavy.cu). Every variant computes the same C.
+ *                      kernel, k_sym_heavy in sg_heavy.cu; bit 2: row-major dense-window work items
+ *                      instead of window-major ones). Every variant computes the same C.
  * The environment seeds them once, at the library's first call (SG_VALIDATE=1, SG_DW_LOG2=m).
  * Errors: INVALID_ARG (unknown key or value out of range). sg_get_option: INT64_MIN if unknown. */
 typedef enum { SG_OPT_VALIDATE = 0, SG_OPT_DENSE_LOG2 = 1, SG_OPT_VARIANT = 2, SG_OPT_COUNT = 3 } sg_option;

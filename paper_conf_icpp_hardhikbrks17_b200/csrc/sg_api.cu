@@ -351,7 +351,7 @@ sg_status sg_set_option(int key, int64_t value) {
     if (key < 0 || key >= SG_OPT_COUNT) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_VALIDATE && value != 0 && value != 1) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_DENSE_LOG2 && (value < -1 || value > 62)) return SG_ERR_INVALID_ARG;
-    if (key == SG_OPT_VARIANT && (value < 0 || value > 3)) return SG_ERR_INVALID_ARG;
+    if (key == SG_OPT_VARIANT && (value < 0 || value > 7)) return SG_ERR_INVALID_ARG;
     g_opt[key] = value;
     return SG_OK;
 }
@@ -715,7 +715,10 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
             int64_t* dcnt = (int64_t*)palloc(pl, sizeof(int64_t) * (size_t)pl->ndw);
             void* t3 = palloc(pl, scan_tmp_bytes(pl->ndw));
             if (!pl->dtc || !pl->ditems || !pl->ditem_off || !dcnt || !t3) return fail(SG_ERR_OOM);
-            CKF(launch_dense_items(pl->heavy, pl->ndw, pl->w, pl->p, dcnt, pl->ditem_off, t3, pl->ditems, s));
+            if (pl->variant & 4)  // round-1 items: row chunks of <= 2^19 products, row-major
+                CKF(launch_dense_items(pl->heavy, pl->ndw, pl->w, pl->p, dcnt, pl->ditem_off, t3, pl->ditems, s));
+            else  // window-major blocks (sg_dense.cu); the item count goes where the kernels read it
+                CKF(launch_dense_items_wm(pl->ndw, pl->p, pl->ditems, pl->ditem_off + pl->ndw, s));
         }
         pl->nslots = hb[0];
         pl->amax = hb[1];

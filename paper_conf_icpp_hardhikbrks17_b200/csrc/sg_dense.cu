@@ -340,6 +340,32 @@ __global__ void k_dense_items(const int32_t* __restrict__ heavy, int64_t ndw, co
         items[off[h] + c] = make_int4((int)h, (int)(c * nwin / nc), (int)((c + 1) * nwin / nc), 0);
 }
 
+// Window-major items [r2]: every dense row is cut into blocks of DW_BLOCK consecutive windows and the
+// items are ordered block by block (item blk * ndw + h = row h's block blk; rows heaviest first inside a
+// block). The persistent CTAs take items in that order, so at any time they all sweep the same one or
+// two window blocks: the slab of B they gather (~193 MB / 43 windows per window at C3) stays L2-resident
+// instead of every CTA streaming its own part of B through L2 (round 1: dense-kernel DRAM traffic ~4x
+// its algorithmic bytes, profiles/r02f_ncu_traffic.txt).
+constexpr int DW_BLOCK = 3;
+
+__global__ void k_dense_items_wm(int64_t ndw, int nwin, int nblk, int4* __restrict__ items, int64_t* __restrict__ nitems) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i == 0) *nitems = ndw * nblk;
+    if (i >= ndw * nblk) return;
+    const int blk = (int)(i / ndw);
+    const int64_t h = i % ndw;
+    items[i] = make_int4((int)h, blk * DW_BLOCK, min(nwin, (blk + 1) * DW_BLOCK), 0);
+}
+
+cudaError_t launch_dense_items_wm(int64_t ndw, int64_t p, int4* items, int64_t* nitems, cudaStream_t s) {
+    if (ndw <= 0) return cudaSuccess;
+    const int nwin = (int)((p + WD - 1) / WD);
+    const int nblk = (nwin + DW_BLOCK - 1) / DW_BLOCK;
+    const int64_t n = ndw * nblk;
+    SG_LAUNCH("k_dense_items", s, (k_dense_items_wm<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(ndw, nwin, nblk, items, nitems)));
+    return cudaGetLastError();
+}
+
 int64_t dense_items_bound(int64_t ndw, int64_t p) {
     const int64_t nwin = (p + WD - 1) / WD;
     return ndw * (nwin < 1 ? 1 : nwin);

@@ -141,6 +141,8 @@ size_t dense2_part_bytes();
 int dense2_pcap();
 // dense-window work items (row, window range): at most dense_items_bound(ndw, p); off[ndw] = count
 int64_t dense_items_bound(int64_t ndw, int64_t p);
+// window-major items (blocks of consecutive windows, ordered block by block); *nitems (device) = count
+cudaError_t launch_dense_items_wm(int64_t ndw, int64_t p, int4* items, int64_t* nitems, cudaStream_t s);
 cudaError_t launch_dense_items(const int32_t* heavy, int64_t ndw, const int64_t* w, int64_t p, int64_t* cnt,
                                int64_t* off, void* scan_tmp, int4* items, cudaStream_t s);
 int dense_window_cols();
