@@ -378,6 +378,9 @@ __device__ unsigned long long g_hv_phase[10];
 #else
 #define HV_MARK(k) do { } while (0)
 #endif
+#if defined(SG_HV_EXP) && SG_HV_EXP == 9  // timing experiment: per-range cycles binned by log2(products)
+__device__ unsigned long long g_hv_rng[24][4];
+#endif
 
 template <class VT>
 __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
@@ -444,6 +447,9 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
         for (int ri = 0; ri < nr; ++ri) {
             const RangeRec R = Rn;
             if (ri + 1 < nr) Rn = rr[ri + 1];
+#if defined(SG_HV_EXP) && SG_HV_EXP == 9
+            const long long hv_t0 = clock64();
+#endif
             const int64_t lo = (int64_t)R.t0 * TW, hi = min(p, (int64_t)R.t1 * TW);
             int tot1 = 0, nk1 = 0;
             bool inreg = false;
@@ -599,6 +605,15 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 bm4[2 * tid + 1] = make_uint4(0, 0, 0, 0);
             }
             HV_MARK(5);
+#if defined(SG_HV_EXP) && SG_HV_EXP == 9
+            if (tid == 0) {
+                const int bn = 32 - __clz(tot1 | 1);
+                atomicAdd(&g_hv_rng[bn][0], 1ull);
+                atomicAdd(&g_hv_rng[bn][1], (unsigned long long)(clock64() - hv_t0));
+                atomicAdd(&g_hv_rng[bn][2], (unsigned long long)tot1);
+                atomicAdd(&g_hv_rng[bn][3], (unsigned long long)R.cnt);
+            }
+#endif
             // no barrier here: the next range's first reads of the cleared bitmap / accumulator and its
             // rewrite of the packed chunk arrays all come after chunk_compact's barriers
         }
@@ -642,6 +657,19 @@ cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, i
                 hh[8], hh[9]);
         unsigned long long z[10] = {0};
         cudaMemcpyToSymbol(g_hv_phase, z, sizeof(z));
+    }
+#endif
+#if defined(SG_HV_EXP) && SG_HV_EXP == 9
+    {
+        unsigned long long hh[24][4] = {{0}};
+        cudaStreamSynchronize(s);
+        cudaMemcpyFromSymbol(hh, g_hv_rng, sizeof(hh));
+        for (int b = 0; b < 24; ++b)
+            if (hh[b][0])
+                fprintf(stderr, "[rank ranges] products<2^%d: ranges %llu  cycles/range %.0f  products/range %.0f  out/range %.0f\n",
+                        b, hh[b][0], (double)hh[b][1] / hh[b][0], (double)hh[b][2] / hh[b][0], (double)hh[b][3] / hh[b][0]);
+        unsigned long long z[24][4] = {{0}};
+        cudaMemcpyToSymbol(g_hv_rng, z, sizeof(z));
     }
 #endif
     return cudaGetLastError();
