@@ -375,11 +375,21 @@ __device__ __forceinline__ void fence_proxy_async_smem() { asm volatile("fence.p
 #if defined(SG_HV_EXP) && SG_HV_EXP == 8  // timing experiment: per-phase cycle counters (lane 0 of each warp)
 __device__ unsigned long long g_hv_phase[10];
 #define HV_MARK(k) do { if ((threadIdx.x & 31) == 0) { long long _t = clock64(); hph[k] += _t - hv_last; hv_last = _t; } } while (0)
+#elif defined(SG_HV_EXP) && SG_HV_EXP == 9
+#define HV_MARK(k) HV_MARK9_##k
+#define HV_MARK9_0 do { } while (0)
+#define HV_MARK9_6 do { } while (0)
+#define HV_MARK9_1 do { if (tid == 0) hv_ts[1] = clock64(); } while (0)
+#define HV_MARK9_2 do { if (tid == 0) hv_ts[2] = clock64(); } while (0)
+#define HV_MARK9_3 do { if (tid == 0) hv_ts[3] = clock64(); } while (0)
+#define HV_MARK9_4 do { if (tid == 0) hv_ts[4] = clock64(); } while (0)
+#define HV_MARK9_5 do { if (tid == 0) hv_ts[5] = clock64(); } while (0)
 #else
 #define HV_MARK(k) do { } while (0)
 #endif
-#if defined(SG_HV_EXP) && SG_HV_EXP == 9  // timing experiment: per-range cycles binned by log2(products)
+#if defined(SG_HV_EXP) && SG_HV_EXP == 9  // timing experiment: per-range cycles (and per phase) binned by log2(products)
 __device__ unsigned long long g_hv_rng[24][4];
+__device__ unsigned long long g_hv_ph[24][5];
 #endif
 
 template <class VT>
@@ -449,6 +459,8 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
             if (ri + 1 < nr) Rn = rr[ri + 1];
 #if defined(SG_HV_EXP) && SG_HV_EXP == 9
             const long long hv_t0 = clock64();
+            long long hv_ts[6];
+            hv_ts[0] = hv_t0;
 #endif
             const int64_t lo = (int64_t)R.t0 * TW, hi = min(p, (int64_t)R.t1 * TW);
             int tot1 = 0, nk1 = 0;
@@ -612,6 +624,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 atomicAdd(&g_hv_rng[bn][1], (unsigned long long)(clock64() - hv_t0));
                 atomicAdd(&g_hv_rng[bn][2], (unsigned long long)tot1);
                 atomicAdd(&g_hv_rng[bn][3], (unsigned long long)R.cnt);
+                for (int k = 0; k < 5; ++k) atomicAdd(&g_hv_ph[bn][k], (unsigned long long)(hv_ts[k + 1] - hv_ts[k]));
             }
 #endif
             // no barrier here: the next range's first reads of the cleared bitmap / accumulator and its
@@ -661,15 +674,20 @@ cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, i
 #endif
 #if defined(SG_HV_EXP) && SG_HV_EXP == 9
     {
-        unsigned long long hh[24][4] = {{0}};
+        unsigned long long hh[24][4] = {{0}}, ph[24][5] = {{0}};
         cudaStreamSynchronize(s);
         cudaMemcpyFromSymbol(hh, g_hv_rng, sizeof(hh));
+        cudaMemcpyFromSymbol(ph, g_hv_ph, sizeof(ph));
         for (int b = 0; b < 24; ++b)
             if (hh[b][0])
-                fprintf(stderr, "[rank ranges] products<2^%d: ranges %llu  cycles/range %.0f  products/range %.0f  out/range %.0f\n",
-                        b, hh[b][0], (double)hh[b][1] / hh[b][0], (double)hh[b][2] / hh[b][0], (double)hh[b][3] / hh[b][0]);
-        unsigned long long z[24][4] = {{0}};
+                fprintf(stderr, "[rank ranges] products<2^%d: ranges %llu  cycles/range %.0f  products/range %.0f  out/range %.0f"
+                        " | seg+compact %.0f pass1 %.0f prefix %.0f pass2 %.0f emit %.0f\n",
+                        b, hh[b][0], (double)hh[b][1] / hh[b][0], (double)hh[b][2] / hh[b][0], (double)hh[b][3] / hh[b][0],
+                        (double)ph[b][0] / hh[b][0], (double)ph[b][1] / hh[b][0], (double)ph[b][2] / hh[b][0],
+                        (double)ph[b][3] / hh[b][0], (double)ph[b][4] / hh[b][0]);
+        unsigned long long z[24][4] = {{0}}, z5[24][5] = {{0}};
         cudaMemcpyToSymbol(g_hv_rng, z, sizeof(z));
+        cudaMemcpyToSymbol(g_hv_ph, z5, sizeof(z5));
     }
 #endif
     return cudaGetLastError();
