@@ -269,6 +269,44 @@ __device__ __forceinline__ void emit_slots(int32_t* keys, double* vals, int nslo
         if (keys[s] != EMPTY_KEY) { keys[s] = EMPTY_KEY; vals[s] = 0.0; }
 }
 
+// ---- occupancy-driven emission of the light accumulator ------------------------------------------
+// acc_insert with an occupancy bitmap: the product that installs a key in an empty slot also sets the
+// slot's bit (one native 32-bit shared atomic per distinct column), so that emission visits the
+// occupied slots only instead of scanning every slot of the table.
+__device__ __forceinline__ int acc_insert_occ(int32_t* keys, double* vals, uint32_t* occ, int32_t c, double v, uint32_t d,
+                                              bool ident, uint64_t mult) {
+    uint32_t h;
+    if (ident) {
+        h = d;
+        if (atomicAnd(&keys[h], c) == EMPTY_KEY) atomicOr(&occ[h >> 5], 1u << (h & 31));  // see acc_insert
+    } else {
+        h = (uint32_t)(((uint64_t)d * mult) >> 32);
+        while (true) {
+            int32_t old = keys[h];
+            if (old == c) break;
+            if (old == EMPTY_KEY) {
+                old = atomicCAS(&keys[h], EMPTY_KEY, c);
+                if (old == EMPTY_KEY) { atomicOr(&occ[h >> 5], 1u << (h & 31)); break; }
+                if (old == c) break;
+            }
+            ++h;
+        }
+    }
+    atomicAdd(&vals[h], v);
+    return (int)h;
+}
+
+// index of the r-th (0-based) set bit of m (r < popc(m)), by popcount bisection
+__device__ __forceinline__ int select_bit(uint32_t m, int r) {
+    int pos = 0;
+    #pragma unroll
+    for (int sh = 16; sh; sh >>= 1) {
+        const int c = __popc(m & ((1u << sh) - 1u));
+        if (r >= c) { r -= c; m >>= sh; pos += sh; }
+    }
+    return pos;
+}
+
 // ---- block-level product flattening (heavy path; light rows with U >= 1024) ----------------------
 __device__ __forceinline__ int64_t lower_bound_col(const int32_t* __restrict__ col, int64_t lo, int64_t hi, int64_t x) {
     while (lo < hi) {
@@ -329,6 +367,91 @@ __device__ __forceinline__ int find_k(const int* off, int nk, int j) {
 template <int NT>
 __device__ __forceinline__ long long block_scan_ll(long long v, long long* total, long long* ws) {
     return block_scan1<NT, long long>(v, total, ws);
+}
+
+// Group-wide emission of the occupied slots of [0, nslots) (bits of occ) in slot order into C at
+// `base`; clears the slots and the bits. wp: >= ceil(nslots/32) + 1 ints of group-private shared
+// memory (word prefix), ws: >= G/32 ints (block scan). Entry e (the e-th occupied slot, s) goes to
+// e when slot order is column order (identity map), else (ranked: order-preserving hash, runs mutually
+// ordered but not sorted inside) to e - (s - run start) + (its rank inside the run).
+template <int G, int BLK, class VT>
+__device__ __forceinline__ void emit_occ(int32_t* keys, double* vals, uint32_t* occ, int* wp, int nslots, int64_t base,
+                                         int32_t* __restrict__ C_col, VT* __restrict__ C_val, int* ws, bool ranked) {
+    const int t = threadIdx.x % G, lane = threadIdx.x & 31;
+    const int W = (nslots + 31) >> 5;
+    int u;
+    if constexpr (G == 32) {
+        int carry = 0;
+        for (int w0 = 0; w0 < W; w0 += 32) {
+            const int w = w0 + lane;
+            const int c = w < W ? __popc(occ[w]) : 0;
+            const int inc = warp_incl_scan(c);
+            if (w < W) wp[w] = carry + inc - c;
+            carry += __shfl_sync(FULL, inc, 31);
+        }
+        u = carry;
+        if (lane == 0) wp[W] = u;
+        __syncwarp();
+    } else {
+        // W <= G: one word per thread (P / 32 <= G for the block bins)
+        const int c = t < W ? __popc(occ[t]) : 0;
+        int tot;
+        const int ex = block_scan<G>(c, &tot, ws);
+        if (t < W) wp[t] = ex;
+        if (t == 0) wp[W] = tot;
+        u = tot;
+        group_bar<G, BLK>();
+    }
+    for (int e0 = t - lane; e0 < u; e0 += G) {
+        const int e = e0 + lane;
+        if (e < u) {
+            int lo = 0, hi = W - 1;  // largest w with wp[w] <= e (that word holds entry e)
+            while (lo < hi) {
+                const int mid = (lo + hi + 1) >> 1;
+                if (wp[mid] <= e) lo = mid; else hi = mid - 1;
+            }
+            const uint32_t m = occ[lo];
+            const int bit = select_bit(m, e - wp[lo]);
+            const int s = 32 * lo + bit;
+            const int32_t k = keys[s];
+            int o = e;
+            if (ranked) {
+                int rs, re;
+                const uint32_t below = ~m & ((1u << bit) - 1u);
+                if (below) rs = 32 * lo + (31 - __clz(below)) + 1;
+                else {
+                    int ww = lo - 1;
+                    while (ww >= 0 && occ[ww] == 0xFFFFFFFFu) --ww;
+                    rs = ww < 0 ? 0 : 32 * ww + (31 - __clz(~occ[ww])) + 1;
+                }
+                const uint32_t above = bit == 31 ? 0u : (~m & (~0u << (bit + 1)));
+                if (above) re = 32 * lo + __ffs(above) - 1;
+                else {
+                    int ww = lo + 1;
+                    while (ww < W && occ[ww] == 0xFFFFFFFFu) ++ww;
+                    re = ww >= W ? 32 * W : 32 * ww + __ffs(~occ[ww]) - 1;
+                }
+                if (re - rs > 1) {
+                    int rank = 0;
+                    for (int j = rs; j < re; ++j) rank += keys[j] < k;
+                    o = e - (s - rs) + rank;
+                }
+            }
+            st_out(C_col + base + o, k);
+            st_out(C_val + base + o, (VT)vals[s]);
+        }
+    }
+    group_bar<G, BLK>();  // every rank computed before any slot is cleared
+    for (int w = t; w < W; w += G) {
+        uint32_t m = occ[w];
+        while (m) {
+            const int b = __ffs(m) - 1;
+            m &= m - 1u;
+            keys[32 * w + b] = EMPTY_KEY;
+            vals[32 * w + b] = 0.0;
+        }
+        occ[w] = 0u;
+    }
 }
 
 // First packed entry of every warp's product slice (see SliceCursor): written by the entry whose

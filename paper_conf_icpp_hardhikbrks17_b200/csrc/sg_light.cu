@@ -305,10 +305,16 @@ __device__ __forceinline__ void sorted_emit(int32_t* keys, double* vals, int* cn
     group_bar<G, BLK>();
 }
 
+#ifndef SG_LIGHT_OCC
+#define SG_LIGHT_OCC 1  // emission driven by an occupancy bitmap (0: scan every slot)
+#endif
 template <int U>
 struct LightTable {
     static constexpr int H = 2 * U;  // home range (load <= 1/2)
     static constexpr int P = H + U;  // + overflow room: probing never passes the end (u <= U)
+    static constexpr int OW = (P + 31) / 32;  // occupancy words
+    // per-row shared memory: vals, keys, occupancy bits, word prefix (+1)
+    static constexpr int BYTES = P * 12 + (SG_LIGHT_OCC ? (OW * 4 + (OW + 1) * 4) : 0);
 };
 
 template <int U, int R, class VT>
@@ -316,13 +322,18 @@ __global__ void __launch_bounds__(32 * R) k_num_light(Mat A, Mat B, const int32_
                                                       int64_t rb, const int2* __restrict__ span,
                                                       const int64_t* __restrict__ C_rp, int32_t* __restrict__ C_col,
                                                       VT* __restrict__ C_val) {
-    constexpr int H = LightTable<U>::H, P = LightTable<U>::P;
+    constexpr int H = LightTable<U>::H, P = LightTable<U>::P, OW = LightTable<U>::OW;
     extern __shared__ double smem_d[];
     __shared__ int s_cnt[R];
     const int g = threadIdx.x / 32, lane = threadIdx.x & 31;
     double* vals = smem_d + g * P;
     int32_t* keys = reinterpret_cast<int32_t*>(smem_d + R * P) + g * P;
+    uint32_t* occ = reinterpret_cast<uint32_t*>(reinterpret_cast<int32_t*>(smem_d + R * P) + R * P) + g * OW;
+    int* wp = reinterpret_cast<int*>(reinterpret_cast<uint32_t*>(reinterpret_cast<int32_t*>(smem_d + R * P) + R * P) + R * OW) +
+              g * (OW + 1);
     for (int s = lane; s < P; s += 32) { keys[s] = EMPTY_KEY; vals[s] = 0.0; }
+    if (SG_LIGHT_OCC)
+        for (int s = lane; s < OW; s += 32) occ[s] = 0u;
     if (lane == 0) s_cnt[g] = 0;
     __syncwarp();
     for (int64_t j = (int64_t)blockIdx.x * R + g; j < cnt; j += (int64_t)gridDim.x * R) {
@@ -348,13 +359,16 @@ __global__ void __launch_bounds__(32 * R) k_num_light(Mat A, Mat B, const int32_
         for (int64_t pb = s0; pb < s1; pb += 32) {
             chunk_products<true, VT, 2>(A, B, pb, min(pb + 32, s1), [](int, int64_t&, int&) {},
                                         [&](int32_t c, double v) {
-                                            int h = acc_insert(keys, vals, c, v, (uint32_t)(c - cmin), ident, mult);
+                                            const int h = SG_LIGHT_OCC
+                                                ? acc_insert_occ(keys, vals, occ, c, v, (uint32_t)(c - cmin), ident, mult)
+                                                : acc_insert(keys, vals, c, v, (uint32_t)(c - cmin), ident, mult);
                                             hmax = max(hmax, h);
                                         });
         }
         hmax = warp_max(hmax);
         __syncwarp();
-        emit_slots<32, 32 * R, VT>(keys, vals, hmax + 1, C_rp[li], C_col, C_val, nullptr, !ident);
+        if (SG_LIGHT_OCC) emit_occ<32, 32 * R, VT>(keys, vals, occ, wp, hmax + 1, C_rp[li], C_col, C_val, nullptr, !ident);
+        else emit_slots<32, 32 * R, VT>(keys, vals, hmax + 1, C_rp[li], C_col, C_val, nullptr, !ident);
         __syncwarp();
     }
 }
@@ -364,7 +378,8 @@ __global__ void __launch_bounds__(NT) k_num_light_blk(Mat A, Mat B, const int32_
                                                       int64_t rb, const int2* __restrict__ span,
                                                       const int64_t* __restrict__ C_rp, int32_t* __restrict__ C_col,
                                                       VT* __restrict__ C_val) {
-    constexpr int H = LightTable<U>::H, P = LightTable<U>::P;
+    constexpr int H = LightTable<U>::H, P = LightTable<U>::P, OW = LightTable<U>::OW;
+    static_assert(!SG_LIGHT_OCC || OW <= NT, "emit_occ: one occupancy word per thread");
     extern __shared__ double smem_d[];
     __shared__ int64_t s_beg[NT];
     __shared__ int s_off[NT];
@@ -375,7 +390,11 @@ __global__ void __launch_bounds__(NT) k_num_light_blk(Mat A, Mat B, const int32_
     const int tid = threadIdx.x, lane = tid & 31;
     double* vals = smem_d;
     int32_t* keys = reinterpret_cast<int32_t*>(smem_d + P);
+    uint32_t* occ = reinterpret_cast<uint32_t*>(keys + P);
+    int* wp = reinterpret_cast<int*>(occ + OW);
     for (int s = tid; s < P; s += NT) { keys[s] = EMPTY_KEY; vals[s] = 0.0; }
+    if (SG_LIGHT_OCC)
+        for (int s = tid; s < OW; s += NT) occ[s] = 0u;
     if (tid == 0) { s_hmax = -1; s_cnt = 0; }
     __syncthreads();
     for (int64_t j = blockIdx.x; j < cnt; j += gridDim.x) {
@@ -425,7 +444,8 @@ __global__ void __launch_bounds__(NT) k_num_light_blk(Mat A, Mat B, const int32_
             const int tot = chunk_compact<NT, int64_t>(len, beg, a, s_beg, s_off, s_a, &nk, wsll);
             warp_slice<NT, true, VT, int64_t>(s_beg, s_off, s_a, nk, tot, B, [&](int32_t c, double v) {
                 if (c < 0) return;
-                const int h = acc_insert(keys, vals, c, v, (uint32_t)(c - cmin), ident, mult);
+                const int h = SG_LIGHT_OCC ? acc_insert_occ(keys, vals, occ, c, v, (uint32_t)(c - cmin), ident, mult)
+                                           : acc_insert(keys, vals, c, v, (uint32_t)(c - cmin), ident, mult);
                 hmax = max(hmax, h);
             });
             __syncthreads();
@@ -436,7 +456,8 @@ __global__ void __launch_bounds__(NT) k_num_light_blk(Mat A, Mat B, const int32_
         const int nslots = s_hmax + 1;
         __syncthreads();
         if (tid == 0) s_hmax = -1;
-        emit_slots<NT, NT, VT>(keys, vals, nslots, C_rp[li], C_col, C_val, ws, !ident);
+        if (SG_LIGHT_OCC) emit_occ<NT, NT, VT>(keys, vals, occ, wp, nslots, C_rp[li], C_col, C_val, ws, !ident);
+        else emit_slots<NT, NT, VT>(keys, vals, nslots, C_rp[li], C_col, C_val, ws, !ident);
         __syncthreads();
     }
 }
@@ -448,7 +469,7 @@ static cudaError_t num_light_V(int b, const Mat& A, const Mat& B, const int32_t*
 #define X(B_, U_, R_)                                                                                         \
     case B_: {                                                                                                \
         auto kern = k_num_light<U_, R_, VT>;                                                                  \
-        const int smem = R_ * LightTable<U_>::P * 12;                                                         \
+        const int smem = R_ * LightTable<U_>::BYTES;                                                          \
         if (smem > 48 * 1024) {                                                                               \
             cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);     \
             if (e != cudaSuccess) return e;                                                                   \
@@ -462,7 +483,7 @@ static cudaError_t num_light_V(int b, const Mat& A, const Mat& B, const int32_t*
 #define X(B_, U_, NT_)                                                                                        \
     case B_: {                                                                                                \
         auto kern = k_num_light_blk<U_, NT_, VT>;                                                             \
-        const int smem = LightTable<U_>::P * 12;                                                              \
+        const int smem = LightTable<U_>::BYTES;                                                               \
         if (smem > 48 * 1024) {                                                                               \
             cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);     \
             if (e != cudaSuccess) return e;                                                                   \
