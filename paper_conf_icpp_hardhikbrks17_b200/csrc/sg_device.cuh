@@ -523,7 +523,9 @@ struct SliceCursor {
         i0 = j_lo < j_hi ? sg_wstart[wid] : 0;  // written by the packing (chunk_compact)
     }
     // batch [j0, j0 + 32): lane's (column, a_ik * b_kj), c = -1 beyond the slice
-    __device__ __forceinline__ void fetch(const Mat& B, int j0, int& c, double& v) {
+    __device__ __forceinline__ void fetch(const Mat& B, int j0, int& c, double& v) { fetchv<VAL>(B, j0, c, v); }
+    template <bool V>
+    __device__ __forceinline__ void fetchv(const Mat& B, int j0, int& c, double& v) {
         const int lane = threadIdx.x & 31;
         const int e0 = i0 + 1 < nk ? off_at(i0 + 1) : tot;
         if (j0 + 31 < e0) {  // fast path: the whole batch lies inside entry i0 (hub rows of B)
@@ -533,7 +535,7 @@ struct SliceCursor {
             if (j < j_hi) {
                 const int64_t q = (int64_t)beg_at(i0) + (j - off_at(i0));
                 c = __ldg(B.col + q);
-                if (VAL) v = a_at(i0) * ldv<VT>(B.val, q);
+                if (V) v = a_at(i0) * ldv<VT>(B.val, q);
             }
             return;
         }
@@ -553,45 +555,49 @@ struct SliceCursor {
         if (j < j_hi) {
             const int64_t q = (int64_t)beg_at(kk) + (j - os);
             c = __ldg(B.col + q);
-            if (VAL) v = a_at(kk) * ldv<VT>(B.val, q);
+            if (V) v = a_at(kk) * ldv<VT>(B.val, q);
         }
         i0 = __shfl_sync(FULL, kk, 31);
     }
 };
 
-// Streams the warp's slice through f, four batches in flight (fetch(j + 96) is issued before batch
-// j is consumed). f is called by every lane (c < 0: no product) so it may use warp collectives.
+// Streams the warp's slice from product j_start on (sc.i0 = the packed entry holding j_start) through
+// f, four batches in flight (fetch(j + 96) is issued before batch j is consumed). f is called by every
+// lane (c < 0: no product) so it may use warp collectives. V: fetch values too.
+template <bool V, int NT, bool VAL, class VT, class BEG, class F>
+__device__ __forceinline__ void warp_slice_from(SliceCursor<NT, VAL, VT, BEG>& sc, int j_start, const Mat& B, F&& f) {
+    const int j_hi = sc.j_hi;
+    if (j_start >= j_hi) return;
+    int c0, c1, c2, c3;
+    double v0, v1, v2, v3;
+    sc.template fetchv<V>(B, j_start, c0, v0);
+    sc.template fetchv<V>(B, j_start + 32, c1, v1);
+    sc.template fetchv<V>(B, j_start + 64, c2, v2);
+    for (int j0 = j_start; j0 < j_hi; j0 += 128) {
+        sc.template fetchv<V>(B, j0 + 96, c3, v3);
+        f(c0, v0);
+        if (j0 + 128 >= j_hi) { f(c1, v1); f(c2, v2); f(c3, v3); break; }
+        sc.template fetchv<V>(B, j0 + 128, c0, v0);
+        f(c1, v1);
+        sc.template fetchv<V>(B, j0 + 160, c1, v1);
+        f(c2, v2);
+        sc.template fetchv<V>(B, j0 + 192, c2, v2);
+        f(c3, v3);
+    }
+}
 template <int NT, bool VAL, class VT, class BEG, class F>
 __device__ __forceinline__ void warp_slice(const BEG* s_beg, const int* s_off, const double* s_a, int nk, int tot,
                                            const Mat& B, F&& f) {
     SliceCursor<NT, VAL, VT, BEG> sc(s_beg, s_off, s_a, nk, tot);
-    const int j_lo = sc.j_lo, j_hi = sc.j_hi;
-    if (j_lo >= j_hi) return;
-    int c0, c1, c2, c3;
-    double v0, v1, v2, v3;
-    sc.fetch(B, j_lo, c0, v0);
-    sc.fetch(B, j_lo + 32, c1, v1);
-    sc.fetch(B, j_lo + 64, c2, v2);
-    for (int j0 = j_lo; j0 < j_hi; j0 += 128) {
-        sc.fetch(B, j0 + 96, c3, v3);
-        f(c0, v0);
-        if (j0 + 128 >= j_hi) { f(c1, v1); f(c2, v2); f(c3, v3); break; }
-        sc.fetch(B, j0 + 128, c0, v0);
-        f(c1, v1);
-        sc.fetch(B, j0 + 160, c1, v1);
-        f(c2, v2);
-        sc.fetch(B, j0 + 192, c2, v2);
-        f(c3, v3);
-    }
+    warp_slice_from<VAL>(sc, sc.j_lo, B, f);
 }
 
-// Small chunks (every warp slice <= 128 products, i.e. tot <= 4*NT): the warp's whole slice is
-// fetched once into registers (columns AND values), so a two-pass consumer (bitmap, then rank
-// accumulation) reads B once. Returns false (nothing fetched) when the chunk is too large.
+// The first four batches of the warp's slice fetched into registers (columns AND values) — a two-pass
+// consumer (bitmap, then rank accumulation) then re-reads B only for the rest of its slice, from the
+// returned cursor entry on (see warp_slice_rest).
 template <int NT, class VT, class BEG>
-__device__ __forceinline__ bool warp_slice_regs(const BEG* s_beg, const int* s_off, const double* s_a, int nk, int tot,
-                                                const Mat& B, int (&c)[4], double (&v)[4]) {
-    if (tot > 4 * NT) return false;
+__device__ __forceinline__ int warp_slice_head(const BEG* s_beg, const int* s_off, const double* s_a, int nk, int tot,
+                                               const Mat& B, int (&c)[4], double (&v)[4]) {
     SliceCursor<NT, true, VT, BEG> sc(s_beg, s_off, s_a, nk, tot);
     #pragma unroll
     for (int r = 0; r < 4; ++r) {
@@ -599,7 +605,15 @@ __device__ __forceinline__ bool warp_slice_regs(const BEG* s_beg, const int* s_o
         v[r] = 0.0;
         if (sc.j_lo + 32 * r < sc.j_hi) sc.fetch(B, sc.j_lo + 32 * r, c[r], v[r]);
     }
-    return true;
+    return sc.i0;
+}
+// Products [j_lo + 128, j_hi) of the warp's slice (after warp_slice_head; i0 = its return value).
+template <bool V, int NT, class VT, class BEG, class F>
+__device__ __forceinline__ void warp_slice_rest(const BEG* s_beg, const int* s_off, const double* s_a, int nk, int tot,
+                                                int i0, const Mat& B, F&& f) {
+    SliceCursor<NT, V, VT, BEG> sc(s_beg, s_off, s_a, nk, tot);
+    sc.i0 = i0;
+    warp_slice_from<V>(sc, sc.j_lo + 128, B, f);
 }
 
 // Segment of one k entry for tiles [.., t1) starting at its cursor: long B rows read the tile

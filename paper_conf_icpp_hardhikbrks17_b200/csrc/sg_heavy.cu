@@ -465,6 +465,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
             const int64_t lo = (int64_t)R.t0 * TW, hi = min(p, (int64_t)R.t1 * TW);
             int tot1 = 0, nk1 = 0;
             bool inreg = false;
+            int i0_rest = 0;
             int rc[4];
             double rv[4];
             // ---- pass 1: segments (advance cursors) + bitmap of the range ----
@@ -499,11 +500,14 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 auto setbit = [&](int32_t c, double) {
                     if (c >= 0) red_or_s(bb + 4u * ((uint32_t)c >> 5), 1u << (c & 31));
                 };
-                // small ranges: the products stay in registers from pass 1 to pass 2 (B read once)
-                inreg = SG_INREG && single && warp_slice_regs<NUM_T, VT, int32_t>(S.s_beg, S.s_off, S.s_a, nk, ctot, B, rc, rv);
+                // single-chunk rows: each warp's first four batches stay in registers from pass 1 to pass 2
+                // (B read once for ranges of up to 4 * NUM_T products), only the rest is re-read in pass 2
+                inreg = SG_INREG && single;
                 if (inreg) {
+                    i0_rest = warp_slice_head<NUM_T, VT, int32_t>(S.s_beg, S.s_off, S.s_a, nk, ctot, B, rc, rv);
                     #pragma unroll
                     for (int r = 0; r < 4; ++r) setbit(rc[r], 0.0);
+                    warp_slice_rest<false, NUM_T, VT, int32_t>(S.s_beg, S.s_off, S.s_a, nk, ctot, i0_rest, B, setbit);
                 } else {
                     warp_slice<NUM_T, false, VT, int32_t>(S.s_beg, S.s_off, nullptr, nk, ctot, B, setbit);
                 }
@@ -572,6 +576,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
             if (inreg) {
                 #pragma unroll
                 for (int r = 0; r < 4; ++r) acc(rc[r], rv[r]);
+                warp_slice_rest<true, NUM_T, VT, int32_t>(S.s_beg, S.s_off, S.s_a, nk1, tot1, i0_rest, B, acc);
             } else if (single) {
                 warp_slice<NUM_T, true, VT, int32_t>(S.s_beg, S.s_off, S.s_a, nk1, tot1, B, acc);  // pass-1 packing kept
             } else {
