@@ -107,10 +107,16 @@ typedef struct sg_plan sg_plan;   /* opaque; owns only its workspace */
  *   SG_OPT_VARIANT     kernel variant bits for A/B measurements (0 = the default kernels; bit 0: the
  *                      previous dense-window kernel, sg_dense.cu; bit 1: the previous heavy symbolic
  *                      kernel, k_sym_heavy in sg_heavy.cu; bit 2: row-major dense-window work items
- *                      instead of window-major ones). Every variant computes the same C.
- * The environment seeds them once, at the library's first call (SG_VALIDATE=1, SG_DW_LOG2=m).
+ *                      instead of window-major ones; bit 3: the CTA rank kernel for every rank row instead of
+ *                      the warp-tile kernel for rows of <= 64 k entries). Every variant computes the same C.
+ *   SG_OPT_L2_PERSIST  bytes of B.col kept in the persisting L2 carve-out during sg_symbolic / sg_numeric
+ *                      (every heavy product gathers a column of B): -1 = all of B.col up to the device's
+ *                      maximum carve-out, 0 (default) = off (measured no gain on C3: 239.9 vs 235.1 ms). The calls set the stream's access-policy window
+ *                      for their own launches and clear it before returning; the device's persisting-L2 limit
+ *                      is raised once (a process-wide setting).
+ * The environment seeds them once, at the library's first call (SG_VALIDATE=1, SG_DW_LOG2=m, SG_L2_PERSIST=b).
  * Errors: INVALID_ARG (unknown key or value out of range). sg_get_option: INT64_MIN if unknown. */
-typedef enum { SG_OPT_VALIDATE = 0, SG_OPT_DENSE_LOG2 = 1, SG_OPT_VARIANT = 2, SG_OPT_COUNT = 3 } sg_option;
+typedef enum { SG_OPT_VALIDATE = 0, SG_OPT_DENSE_LOG2 = 1, SG_OPT_VARIANT = 2, SG_OPT_L2_PERSIST = 3, SG_OPT_COUNT = 4 } sg_option;
 sg_status sg_set_option(int key, int64_t value);
 int64_t sg_get_option(int key);
 

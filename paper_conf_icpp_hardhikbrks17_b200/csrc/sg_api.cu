@@ -114,8 +114,58 @@ void init_options() {
         if (e && e[0] == '1') g_opt[SG_OPT_VALIDATE] = 1;
         e = getenv("SG_DW_LOG2");
         if (e && *e) g_opt[SG_OPT_DENSE_LOG2] = atoll(e);
+        g_opt[SG_OPT_L2_PERSIST] = 0;
+        e = getenv("SG_L2_PERSIST");
+        if (e && *e) g_opt[SG_OPT_L2_PERSIST] = atoll(e);
     });
 }
+
+// B.col in the persisting L2 carve-out for the launches of one call (SG_OPT_L2_PERSIST): every heavy
+// product gathers a column index of B, and B (193 MB on C3: 64 MB of columns, 129 MB of values) exceeds
+// the 126 MB L2, so without it the C stream and the value gathers evict the columns. The window is set on
+// the caller's stream for this call's launches only and cleared on exit.
+struct L2Window {
+    cudaStream_t s;
+    bool on = false;
+    L2Window(cudaStream_t st, const void* ptr, size_t bytes) : s(st) {
+        init_options();
+        const int64_t opt = g_opt[SG_OPT_L2_PERSIST].load();
+        if (opt == 0 || bytes == 0 || !ptr) return;
+        static size_t maxp = 0, maxwin = 0;
+        static std::once_flag once;
+        std::call_once(once, [] {
+            int dev = 0, a = 0, b = 0;
+            if (cudaGetDevice(&dev) != cudaSuccess) return;
+            if (cudaDeviceGetAttribute(&a, cudaDevAttrMaxPersistingL2CacheSize, dev) != cudaSuccess) a = 0;
+            if (cudaDeviceGetAttribute(&b, cudaDevAttrMaxAccessPolicyWindowSize, dev) != cudaSuccess) b = 0;
+            maxp = (size_t)a;
+            maxwin = (size_t)b;
+            cudaGetLastError();
+        });
+        if (maxp == 0 || maxwin == 0) return;
+        size_t want = opt > 0 && (size_t)opt < bytes ? (size_t)opt : bytes;
+        if (want > maxp) want = maxp;
+        size_t cur = 0;
+        if (cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize) == cudaSuccess && cur < want)
+            cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want);
+        cudaStreamAttrValue v = {};
+        v.accessPolicyWindow.base_ptr = const_cast<void*>(ptr);
+        v.accessPolicyWindow.num_bytes = bytes < maxwin ? bytes : maxwin;
+        const double hr = (double)want / (double)v.accessPolicyWindow.num_bytes;
+        v.accessPolicyWindow.hitRatio = (float)(hr < 1.0 ? hr : 1.0);
+        v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        on = cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &v) == cudaSuccess;
+        cudaGetLastError();
+    }
+    ~L2Window() {
+        if (!on) return;
+        cudaStreamAttrValue v = {};
+        v.accessPolicyWindow.num_bytes = 0;
+        cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &v);
+        cudaGetLastError();
+    }
+};
 
 int variant_bits() {
     init_options();
@@ -351,7 +401,8 @@ sg_status sg_set_option(int key, int64_t value) {
     if (key < 0 || key >= SG_OPT_COUNT) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_VALIDATE && value != 0 && value != 1) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_DENSE_LOG2 && (value < -1 || value > 62)) return SG_ERR_INVALID_ARG;
-    if (key == SG_OPT_VARIANT && (value < 0 || value > 7)) return SG_ERR_INVALID_ARG;
+    if (key == SG_OPT_VARIANT && (value < 0 || value > 15)) return SG_ERR_INVALID_ARG;
+    if (key == SG_OPT_L2_PERSIST && value < -1) return SG_ERR_INVALID_ARG;
     g_opt[key] = value;
     return SG_OK;
 }
@@ -646,6 +697,7 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
     pl->C_rp = C_row_ptr;
     const int64_t nr = pl->nr;
     Mat a = mat_of(A), b = mat_of(B);
+    L2Window l2w(s, b.col, 4 * (size_t)b.nnz);
     auto fail = [&](sg_status e) { pl->poisoned = true; sg_plan_destroy(pl); return e; };
     size_t nrb = (size_t)(nr > 0 ? nr : 1);
     pl->w = (int64_t*)palloc(pl, 8 * nrb);
@@ -725,6 +777,8 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
         pl->ranges = (RangeRec*)palloc(pl, sizeof(RangeRec) * (size_t)(pl->nslots > 0 ? pl->nslots : 1));
         pl->tp = (uint32_t*)palloc(pl, 4 * (size_t)(pl->nlong > 0 ? pl->nlong : 1) * (size_t)(pl->T + 1));
         if (!pl->ranges || !pl->tp) return fail(SG_ERR_OOM);
+        // unused range slots read as row -1 (the tile kernel walks every slot)
+        CKF(cudaMemsetAsync(pl->ranges, 0xff, sizeof(RangeRec) * (size_t)(pl->nslots > 0 ? pl->nslots : 1), s));
         if (pl->ndw > 0 && pl->amax + 32 > dense2_pcap()) {
             pl->pscr_cap = pl->amax + 32;
             pl->pscr = palloc(pl, dense2_part_bytes() * (size_t)pl->pscr_cap * 148);
@@ -774,6 +828,7 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
     if (((uintptr_t)C_col & 3u) || ((uintptr_t)C_val & (pl->dt == 0 ? 7u : 3u))) return SG_ERR_INVALID_ARG;
     if (pl->nnz_c == 0) return SG_OK;
     Mat a = mat_of(A), b = mat_of(B);
+    L2Window l2w(s, b.col, 4 * (size_t)b.nnz);
     for (int k = 0; k < NBIN_LIGHT; ++k)
         CKP(pl, launch_num_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], pl->rb, pl->span, pl->C_rp,
                                  C_col, C_val, s));
@@ -785,8 +840,15 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
             CKP(pl, launch_num_dense2(a, b, pl->heavy, pl->ndw, pl->rb, pl->w, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
                                       C_val, pl->counter, pl->pscr, pl->pscr_cap, pl->dtc, pl->ditems,
                                       pl->ditem_off + pl->ndw, s));
+        // rank rows: the CTA rank kernel takes the rows with more than tile_kreg() k entries, the warp-tile
+        // kernel the rest (SG_OPT_VARIANT bit 3: the CTA kernel takes all of them)
+        const bool tile = !(pl->variant & 8);
         CKP(pl, launch_num_heavy(a, b, pl->heavy, pl->ndw, pl->nheavy, pl->rb, pl->range_off, pl->nranges, pl->ranges,
-                                 pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter, pl->gscr, pl->amax, s));
+                                 pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter, pl->gscr, pl->amax,
+                                 tile ? (int)tile_kreg() : 0, s));
+        if (tile && pl->nheavy > pl->ndw)
+            CKP(pl, launch_num_tile(a, b, pl->ranges, pl->nslots, pl->rb, pl->long_id, pl->nlong > 0 ? pl->tp : nullptr,
+                                    pl->T, pl->C_rp, C_col, C_val, pl->counter, s));
     }
     if (s != pl->s) {  // the plan's workspace frees (on pl->s) wait for this call's kernels
         cudaEvent_t ev;

@@ -397,7 +397,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
     Mat A, Mat B, const int32_t* __restrict__ heavy, int64_t h0, int64_t nheavy, int64_t rb, const int64_t* __restrict__ range_off,
     const int32_t* __restrict__ nranges, const RangeRec* __restrict__ ranges, const int32_t* __restrict__ long_id,
     const uint32_t* __restrict__ tp, int T, const int64_t* __restrict__ C_rp, int32_t* __restrict__ C_col,
-    VT* __restrict__ C_val, unsigned long long* counter, int4* __restrict__ gscr, int64_t amax) {
+    VT* __restrict__ C_val, unsigned long long* counter, int4* __restrict__ gscr, int64_t amax, int amin) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     HeavySmem& S = *reinterpret_cast<HeavySmem*>(smem_raw);
     __shared__ long long s_j;
@@ -429,6 +429,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
         const int64_t row = rb + li;
         const int64_t s0 = __ldg(A.rp + row), s1 = __ldg(A.rp + row + 1);
         const int na = (int)(s1 - s0);
+        if (na <= amin) continue;  // a sparse rank row: the warp-tile kernel's (sg_tile.cu)
         const bool single = na <= KC;
         const int nr = nranges[h];
         const RangeRec* rr = ranges + range_off[h];
@@ -646,7 +647,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
 cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, int64_t h0, int64_t nheavy, int64_t rb,
                              const int64_t* range_off, const int32_t* nranges, const RangeRec* ranges,
                              const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
-                             void* C_val, unsigned long long* counter, int4* gscr, int64_t amax, cudaStream_t s) {
+                             void* C_val, unsigned long long* counter, int4* gscr, int64_t amax, int amin, cudaStream_t s) {
     if (nheavy - h0 <= 0) return cudaSuccess;
     const int smem = (int)sizeof(HeavySmem);
     cudaError_t e = cudaMemsetAsync(counter, 0, sizeof(unsigned long long), s);
@@ -657,12 +658,12 @@ cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, i
         if ((e = cudaFuncSetAttribute(k_num_heavy<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
         SG_LAUNCH("k_num_heavy", s, (k_num_heavy<double><<<grid, NUM_T, smem, s>>>(
                                         A, B, heavy, h0, nheavy, rb, range_off, nranges, ranges, long_id, tp, T, C_rp, C_col,
-                                        (double*)C_val, counter, gscr, amax)));
+                                        (double*)C_val, counter, gscr, amax, amin)));
     } else {
         if ((e = cudaFuncSetAttribute(k_num_heavy<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
         SG_LAUNCH("k_num_heavy", s, (k_num_heavy<float><<<grid, NUM_T, smem, s>>>(
                                         A, B, heavy, h0, nheavy, rb, range_off, nranges, ranges, long_id, tp, T, C_rp, C_col,
-                                        (float*)C_val, counter, gscr, amax)));
+                                        (float*)C_val, counter, gscr, amax, amin)));
     }
 #if defined(SG_HV_EXP) && SG_HV_EXP == 8
     {

@@ -122,7 +122,7 @@ size_t part_bytes();
 cudaError_t launch_num_heavy(const Mat& A, const Mat& B, const int32_t* heavy, int64_t h0, int64_t nheavy, int64_t rb,
                              const int64_t* range_off, const int32_t* nranges, const RangeRec* ranges,
                              const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
-                             void* C_val, unsigned long long* counter, int4* gscr, int64_t amax, cudaStream_t s);
+                             void* C_val, unsigned long long* counter, int4* gscr, int64_t amax, int amin /*skip rows with <= amin k entries*/, cudaStream_t s);
 cudaError_t launch_max_i64(const int64_t* x, int64_t n, unsigned long long* out /*zeroed here*/, cudaStream_t s);
 cudaError_t launch_max_a(const Mat& A, const int32_t* list, int64_t cnt, int64_t rb, unsigned long long* out,
                          cudaStream_t s);
@@ -148,6 +148,12 @@ cudaError_t launch_dense_items(const int32_t* heavy, int64_t ndw, const int64_t*
 int dense_window_cols();
 int dense_window_log2(int64_t p, int64_t opt);  // opt >= 0 overrides (sg_set_option; 62 disables the path)
 int heavy_kc();
+// warp-owned tile numeric for the rank rows (sg_tile.cu): range slots [0, nslots) (row < 0 = unused);
+// only rows with at most tile_kreg() k entries (the rest: launch_num_heavy with amin = tile_kreg())
+cudaError_t launch_num_tile(const Mat& A, const Mat& B, const RangeRec* ranges, int64_t nslots, int64_t rb,
+                            const int32_t* long_id, const uint32_t* tp, int T, const int64_t* C_rp, int32_t* C_col,
+                            void* C_val, unsigned long long* counter, cudaStream_t s);
+int64_t tile_kreg();
 int heavy_grid();
 int dense_grid();
 int dense_kc();
