@@ -294,7 +294,16 @@ def main():
     nnzA_dense = int(a_rows[dmask].sum().item())
     W_heavy = int(wrow[cls == 2].sum().item())
     W_dense = int(wrow[dmask].sum().item())
-    del cls, u, a_rows, wrow, dmask
+    # rank rows (heavy, below the dense cut): <= 64 k entries on the warp-tile kernel (k_num_tile), the rest
+    # on the CTA rank kernel (k_num_heavy); SG_OPT_VARIANT bit 3 puts them all on k_num_heavy
+    tmask = (cls == 2) & ~dmask & (a_rows <= 64)
+    if sg.get_option(sg.SG_OPT_VARIANT) & 8:
+        tmask = torch.zeros_like(tmask)
+    ntile = int(tmask.sum().item())
+    nnzC_tile = int(u[tmask].sum().item())
+    nnzA_tile = int(a_rows[tmask].sum().item())
+    W_tile = int(wrow[tmask].sum().item())
+    del cls, u, a_rows, wrow, dmask, tmask
     nnzC_total = nnz_local
     if world > 1:
         t = torch.tensor([nnz_local], device=dev, dtype=torch.int64)
@@ -352,8 +361,9 @@ def main():
     Bbytes = csr_bytes(H.nrows, H.nnz, vbytes)
     alg = {
         # compulsory bytes of one launch: its A rows, B once, its C entries
-        "k_num_heavy": 12 * (nnzA_heavy - nnzA_dense) + 8 * (nheavy - ndense) + Bbytes
-                       + (4 + vbytes) * (nnzC_heavy - nnzC_dense),
+        "k_num_heavy": 12 * (nnzA_heavy - nnzA_dense - nnzA_tile) + 8 * (nheavy - ndense - ntile) + Bbytes
+                       + (4 + vbytes) * (nnzC_heavy - nnzC_dense - nnzC_tile),
+        "k_num_tile": 12 * nnzA_tile + 8 * ntile + Bbytes + (4 + vbytes) * nnzC_tile,
         "k_num_dense": 12 * nnzA_dense + 8 * ndense + Bbytes + (4 + vbytes) * nnzC_dense,
         "k_sym_heavy": 4 * nnzA_heavy + 8 * nheavy + 8 * (H.nrows + 1) + 4 * H.nnz,
     }
@@ -380,7 +390,8 @@ def main():
     roof_smem = None
     mb = smem_peaks()
     if mb and bk:
-        ops = {"k_num_dense": (W_dense, "smem_cas_f64_16K"), "k_num_heavy": (W_heavy - W_dense, "smem_cas_f64_16K"),
+        ops = {"k_num_dense": (W_dense, "smem_cas_f64_16K"), "k_num_heavy": (W_heavy - W_dense - W_tile, "smem_cas_f64_16K"),
+               "k_num_tile": (W_tile, "smem_cas_f64_16K"),
                "k_sym_heavy": (W_heavy, "smem_or32_16K")}
         roof_smem = {}
         for k, (nprod, prim) in ops.items():

@@ -401,7 +401,7 @@ sg_status sg_set_option(int key, int64_t value) {
     if (key < 0 || key >= SG_OPT_COUNT) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_VALIDATE && value != 0 && value != 1) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_DENSE_LOG2 && (value < -1 || value > 62)) return SG_ERR_INVALID_ARG;
-    if (key == SG_OPT_VARIANT && (value < 0 || value > 15)) return SG_ERR_INVALID_ARG;
+    if (key == SG_OPT_VARIANT && (value < 0 || value > 31)) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_L2_PERSIST && value < -1) return SG_ERR_INVALID_ARG;
     g_opt[key] = value;
     return SG_OK;
@@ -792,7 +792,8 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
     }
     // a6 symbolic
     for (int k = 0; k < NBIN_LIGHT; ++k)
-        CKF(launch_sym_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], nullptr, row_begin, pl->u, pl->span,
+        CKF(launch_sym_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], nullptr, row_begin, pl->u,
+                             light_sorted(k, pl->p, pl->variant) ? nullptr : pl->span,
                              (unsigned long long*)(pl->dbin + 2 * NBINS + 1), s));
     if (pl->variant & 2) {
         CKF(launch_sym_heavy(a, b, pl->heavy, pl->nheavy, nullptr, row_begin, pl->u, pl->range_off, pl->ranges,
@@ -831,7 +832,7 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
     L2Window l2w(s, b.col, 4 * (size_t)b.nnz);
     for (int k = 0; k < NBIN_LIGHT; ++k)
         CKP(pl, launch_num_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], pl->rb, pl->span, pl->C_rp,
-                                 C_col, C_val, s));
+                                 C_col, C_val, light_sorted(k, pl->p, pl->variant), s));
     if (pl->nheavy > 0) {
         if (pl->variant & 1)
             CKP(pl, launch_num_dense(a, b, pl->heavy, pl->ndw, pl->rb, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,

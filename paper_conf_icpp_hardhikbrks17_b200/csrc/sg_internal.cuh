@@ -97,8 +97,11 @@ cudaError_t launch_bin_scatter(const int64_t* w, int64_t nr, int64_t thr, int64_
 cudaError_t launch_sym_light(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt,
                              const int64_t* rowmap, int64_t rb, int64_t* u, int2* span /*nullable*/,
                              unsigned long long* nskew /*nullable: count of column-skewed rows*/, cudaStream_t s);
+// light bin b takes the sorted warp path of the numeric pass for B with p columns (no span / skew
+// information needed from the symbolic pass then); SG_OPT_VARIANT bit 4 keeps the order-preserving hash
+bool light_sorted(int b, int64_t p, int variant);
 cudaError_t launch_num_light(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, int64_t rb,
-                             const int2* span, const int64_t* C_rp, int32_t* C_col, void* C_val, cudaStream_t s);
+                             const int2* span, const int64_t* C_rp, int32_t* C_col, void* C_val, bool sorted, cudaStream_t s);
 // heavy path (sg_heavy.cu)
 cudaError_t launch_long_rows(const Mat& B, int32_t* long_id, int64_t* d_nlong, cudaStream_t s);
 cudaError_t launch_build_tp(const Mat& B, const int32_t* long_id, int T, uint32_t* tp, cudaStream_t s);

@@ -66,6 +66,10 @@ template <int U> __device__ __forceinline__ uint64_t light_mult(int64_t width) {
     return (((uint64_t)(2 * U)) << 32) / (uint64_t)width;
 }
 constexpr int SKEW_MIN_U = 64;
+#ifndef SG_SYM_UNR
+#define SG_SYM_UNR 4
+#endif
+constexpr int SYM_UNR = SG_SYM_UNR;  // warp symbolic: gather batches in flight
 constexpr int SKEW_BUCKET = 40;
 
 // ------------------------------------------------------------------------------------------------
@@ -93,7 +97,7 @@ __global__ void __launch_bounds__(32 * R) k_sym_light(Mat A, Mat B, const int32_
         const int64_t s0 = __ldg(A.rp + row), s1 = __ldg(A.rp + row + 1);
         int ins = 0, cmn = INT_MAX, cmx = -1;
         for (int64_t pb = s0; pb < s1; pb += 32) {
-            chunk_products<false, double, 2>(A, B, pb, min(pb + 32, s1), [](int, int64_t&, int&) {},
+            chunk_products<false, double, SYM_UNR>(A, B, pb, min(pb + 32, s1), [](int, int64_t&, int&) {},
                                              [&](int32_t c, double) {
                                                  cmn = min(cmn, c);
                                                  cmx = max(cmx, c);
@@ -462,6 +466,179 @@ __global__ void __launch_bounds__(NT) k_num_light_blk(Mat A, Mat B, const int32_
     }
 }
 
+// ---- numeric, SORTED warp path (rows with w <= 512 when the column fits in 32 - log2 U bits) -----------
+// One warp per row: the row's w <= U products are gathered (flattened over its k entries) as 32-bit keys
+// (c << log2 U) | j, j = the product's index in the row, with a_ik * b_kj staged in shared memory at j;
+// the U keys (padded with all-ones) are bitonic-sorted in registers (U/32 per lane, blocked layout: lane
+// exchanges by shuffle, in-lane ones by min/max); then, in striped order, the first key of every column
+// run emits the column and the sum of its run's values (summed in product order) at the position given
+// by a ballot prefix of the run heads. No hashing and no shared-memory atomics: the light rows of ER or
+// permuted R-MAT have almost no duplicate columns (C2: nnz(C) / W = 0.9995), so a probe-and-CAS table
+// spends its atomics on entries that never meet.
+#ifndef SG_SORT_UNR
+#define SG_SORT_UNR 4
+#endif
+constexpr int SORT_UNR = SG_SORT_UNR;  // gather batches in flight per round
+
+template <int N>
+__device__ __forceinline__ void bitonic_warp_blocked(uint32_t (&x)[N / 32]) {
+    constexpr int E = N / 32;
+    const int lane = threadIdx.x & 31;
+    #pragma unroll
+    for (int k = 2; k <= N; k <<= 1) {
+        #pragma unroll
+        for (int j = k >> 1; j > 0; j >>= 1) {
+            if (j >= E) {  // partner in lane ^ (j / E), same register
+                const int lx = j / E;
+                const bool lower = (lane & lx) == 0;
+                #pragma unroll
+                for (int r = 0; r < E; ++r) {
+                    const bool asc = (((lane * E + r) & k) == 0);
+                    const uint32_t y = __shfl_xor_sync(FULL, x[r], lx);
+                    x[r] = (lower == asc) ? min(x[r], y) : max(x[r], y);
+                }
+            } else {  // partner in the same lane, register r ^ j
+                #pragma unroll
+                for (int r = 0; r < E; ++r) {
+                    if (r & j) continue;
+                    const bool asc = (((lane * E + r) & k) == 0);
+                    const uint32_t a = x[r], b = x[r | j];
+                    const uint32_t lo = min(a, b), hi = max(a, b);
+                    x[r] = asc ? lo : hi;
+                    x[r | j] = asc ? hi : lo;
+                }
+            }
+        }
+    }
+}
+
+template <int U, int R, class VT>
+__global__ void __launch_bounds__(32 * R, 1024 / (32 * R)) k_num_light_sort(Mat A, Mat B, const int32_t* __restrict__ list, int64_t cnt,
+                                                          int64_t rb, const int64_t* __restrict__ C_rp,
+                                                          int32_t* __restrict__ C_col, VT* __restrict__ C_val) {
+    static_assert(U >= 32 && (U & (U - 1)) == 0, "U: a power of two >= 32");
+    constexpr int E = U / 32, LOGU = __builtin_ctz(U);
+    __shared__ __align__(16) uint32_t skeys[R][U];
+    __shared__ double svals[R][U];
+    const int g = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    uint32_t* sk = skeys[g];
+    double* sv = svals[g];
+    for (int64_t jr = (int64_t)blockIdx.x * R + g; jr < cnt; jr += (int64_t)gridDim.x * R) {
+        const int64_t li = list[jr];
+        const int64_t row = rb + li;
+        const int64_t s0 = __ldg(A.rp + row), s1 = __ldg(A.rp + row + 1);
+        // ---- gather: product j -> key (c << LOGU) | j, value at sv[j] ----
+        int jb = 0;
+        for (int64_t pb = s0; pb < s1; pb += 32) {
+            const int64_t pa = pb + lane;
+            int len = 0;
+            int64_t q0 = 0;
+            double a = 0.0;
+            if (pa < s1) {
+                const int k = __ldg(A.col + pa);
+                q0 = __ldg(B.rp + k);
+                len = (int)(__ldg(B.rp + k + 1) - q0);
+                a = ldv<VT>(A.val, pa);
+            }
+            const int inc = warp_incl_scan(len);
+            const int off = inc - len;
+            const int tot = __shfl_sync(FULL, inc, 31);
+            for (int j0 = 0; j0 < tot; j0 += 32 * SORT_UNR) {
+                int c[SORT_UNR], jj[SORT_UNR];
+                double v[SORT_UNR];
+                #pragma unroll
+                for (int r = 0; r < SORT_UNR; ++r) {
+                    const int j = j0 + 32 * r + lane;
+                    int sl = 0;
+                    #pragma unroll
+                    for (int bb = 16; bb; bb >>= 1) {
+                        const int o = __shfl_sync(FULL, off, sl + bb);
+                        if (o <= j) sl += bb;
+                    }
+                    const int64_t q = __shfl_sync(FULL, q0, sl) + (j - __shfl_sync(FULL, off, sl));
+                    const double as = __shfl_sync(FULL, a, sl);
+                    c[r] = -1;
+                    jj[r] = jb + j;
+                    if (j < tot) {
+                        c[r] = __ldg(B.col + q);
+                        v[r] = as * ldv<VT>(B.val, q);
+                    }
+                }
+                #pragma unroll
+                for (int r = 0; r < SORT_UNR; ++r)
+                    if (c[r] >= 0) {
+                        sk[jj[r]] = ((uint32_t)c[r] << LOGU) | (uint32_t)jj[r];
+                        sv[jj[r]] = v[r];
+                    }
+            }
+            jb += tot;
+        }
+        const int w = jb;  // <= U (the bin bound)
+        for (int j = w + lane; j < U; j += 32) sk[j] = 0xFFFFFFFFu;
+        __syncwarp();
+        // ---- sort (blocked: lane holds keys [lane E, lane E + E)) ----
+        uint32_t x[E];
+        #pragma unroll
+        for (int r = 0; r < E; ++r) x[r] = sk[lane * E + r];
+        bitonic_warp_blocked<U>(x);
+        __syncwarp();
+        #pragma unroll
+        for (int r = 0; r < E; ++r) sk[lane * E + r] = x[r];
+        __syncwarp();
+        // ---- runs of equal columns -> one entry each, in order ----
+        const int64_t base = C_rp[li];
+        int pos0 = 0;
+        for (int e0 = 0; e0 < w; e0 += 32) {
+            const int e = e0 + lane;
+            const uint32_t key = e < w ? sk[e] : 0xFFFFFFFFu;
+            const uint32_t col = key >> LOGU;
+            const bool head = e < w && (e == 0 || (sk[e - 1] >> LOGU) != col);
+            const unsigned m = __ballot_sync(FULL, head);
+            if (head) {
+                double sum = sv[key & (U - 1)];
+                for (int t = e + 1; t < w; ++t) {
+                    const uint32_t kt = sk[t];
+                    if ((kt >> LOGU) != col) break;
+                    sum += sv[kt & (U - 1)];
+                }
+                const int64_t o = base + pos0 + __popc(m & lanemask_lt());
+                st_out(C_col + o, (int32_t)col);
+                st_out(C_val + o, (VT)sum);
+            }
+            pos0 += __popc(m);
+        }
+        __syncwarp();  // sk / sv reused by the next row
+    }
+}
+
+// the sorted warp path applies to bin b (U = 2^b) when its keys fit: c < 2^(32 - log2 max(U, 32))
+#ifndef SG_LIGHT_SORT
+#define SG_LIGHT_SORT 1
+#endif
+bool light_sorted(int b, int64_t p, int variant) {
+    const int lu = b < 5 ? 5 : b;
+    return SG_LIGHT_SORT && !(variant & 16) && b <= 9 && p <= ((int64_t)1 << (32 - lu));
+}
+
+template <class VT>
+static cudaError_t num_light_sort_V(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, int64_t rb,
+                                    const int64_t* C_rp, int32_t* C_col, void* C_val, cudaStream_t s) {
+#define SG_SORT_CASE(U_, R_)                                                                              \
+    SG_LAUNCH("k_num_light_sort", s, (k_num_light_sort<U_, R_, VT><<<grid_for(cnt, R_, 148 * 32), 32 * R_, 0, s>>>( \
+                                         A, B, list, cnt, rb, C_rp, C_col, (VT*)C_val)));                  \
+    break;
+    switch (b) {
+        case 0: case 1: case 2: case 3: case 4: case 5: SG_SORT_CASE(32, 8)
+        case 6: SG_SORT_CASE(64, 8)
+        case 7: SG_SORT_CASE(128, 8)
+        case 8: SG_SORT_CASE(256, 8)
+        case 9: SG_SORT_CASE(512, 4)
+        default: return cudaErrorInvalidValue;
+    }
+#undef SG_SORT_CASE
+    return cudaGetLastError();
+}
+
 template <class VT>
 static cudaError_t num_light_V(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, int64_t rb,
                                const int2* span, const int64_t* C_rp, int32_t* C_col, void* C_val, cudaStream_t s) {
@@ -500,8 +677,12 @@ static cudaError_t num_light_V(int b, const Mat& A, const Mat& B, const int32_t*
 }
 
 cudaError_t launch_num_light(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, int64_t rb,
-                             const int2* span, const int64_t* C_rp, int32_t* C_col, void* C_val, cudaStream_t s) {
+                             const int2* span, const int64_t* C_rp, int32_t* C_col, void* C_val, bool sorted,
+                             cudaStream_t s) {
     if (cnt <= 0) return cudaSuccess;
+    if (sorted)
+        return A.dt == 0 ? num_light_sort_V<double>(b, A, B, list, cnt, rb, C_rp, C_col, C_val, s)
+                         : num_light_sort_V<float>(b, A, B, list, cnt, rb, C_rp, C_col, C_val, s);
     return A.dt == 0 ? num_light_V<double>(b, A, B, list, cnt, rb, span, C_rp, C_col, C_val, s)
                      : num_light_V<float>(b, A, B, list, cnt, rb, span, C_rp, C_col, C_val, s);
 }

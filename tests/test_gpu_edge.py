@@ -20,9 +20,13 @@ pytestmark = pytest.mark.gpu
 
 sg = pytest.importorskip("paper_conf_icpp_hardhikbrks17_b200")
 
-# path -> (thr, dense_log2): light = every row with w <= cap_L on the light kernels; rank = every
-# non-empty row heavy on the rank kernel; dense = every non-empty row heavy on the dense-window kernel
-PATHS = {"light": (4096, 62), "rank": (0, 62), "dense": (0, 0), "mixed": (256, 10)}
+# path -> (thr, dense_log2, variant): light = every row with w <= cap_L on the light kernels (the sorted
+# warp path for w <= 512, the order-preserving hash above; light_hash: the hash for every bin); rank =
+# every non-empty row heavy on the rank kernels (rows of <= 64 k entries on the warp-tile kernel, the rest
+# on the CTA kernel; rank_cta: the CTA kernel for all); dense = every non-empty row heavy on the
+# dense-window kernel
+PATHS = {"light": (4096, 62, 0), "light_hash": (4096, 62, 16), "rank": (0, 62, 0), "rank_cta": (0, 62, 8),
+         "dense": (0, 0, 0), "mixed": (256, 10, 0)}
 
 
 @pytest.fixture
@@ -48,8 +52,9 @@ def _run(A, thr):
 @pytest.mark.parametrize("mode", ["signed", "zeros"])
 @pytest.mark.parametrize("dtype", ["f64", "f32"])
 def test_cancellation_and_stored_zeros_every_path(options, path, mode, dtype):
-    thr, dl = PATHS[path]
+    thr, dl, var = PATHS[path]
     sg.set_option(sg.SG_OPT_DENSE_LOG2, dl)
+    sg.set_option(sg.SG_OPT_VARIANT, var)
     A = gen.config("rmat13", mode=mode, dtype=dtype)
     (rp, col, val), info = _run(A, thr)
     R = oracle.spgemm(A, A)
@@ -78,8 +83,10 @@ def test_cancellation_dense_kernel_variants(options, variant):
 
 
 @pytest.mark.parametrize("mode", ["signed", "zeros"])
-def test_sorted_light_path_with_cancellation(mode):
-    """Un-permuted R-MAT (column-skewed light rows take the uniform-hash + bitonic-sort path)."""
+def test_sorted_light_path_with_cancellation(options, mode):
+    """Un-permuted R-MAT (column-skewed light rows take the uniform-hash + bitonic-sort path; variant bit 4
+    keeps every light bin on the hash path, whose skew detection routes them there)."""
+    sg.set_option(sg.SG_OPT_VARIANT, 16)
     A = gen.rmat(14, permute=False, mode=mode)
     (rp, col, val), info = _run(A, 4096)
     R = oracle.spgemm(A, A)
@@ -91,8 +98,9 @@ def test_all_zero_values_keep_full_structure(options):
     """Every stored value 0: C's values are all 0 and its structure is the full boolean product."""
     A = gen.config("rmat12")
     Z = gen.CSR(A.nrows, A.ncols, A.row_ptr, A.col, np.zeros_like(A.val), "zeros")
-    for thr, dl in PATHS.values():
+    for thr, dl, var in PATHS.values():
         sg.set_option(sg.SG_OPT_DENSE_LOG2, dl)
+        sg.set_option(sg.SG_OPT_VARIANT, var)
         (rp, col, val), _ = _run(Z, thr)
         R = oracle.spgemm(A, A)
         assert np.array_equal(rp, R.row_ptr) and np.array_equal(col, R.col)
@@ -103,9 +111,30 @@ def test_negative_zero_products_are_structural(options):
     """-0.0 inputs: products are +-0.0, every entry exists and compares equal to 0."""
     A = gen.config("C1")
     N = gen.CSR(A.nrows, A.ncols, A.row_ptr, A.col, np.full_like(A.val, -0.0), "negzero")
-    for thr, dl in PATHS.values():
+    for thr, dl, var in PATHS.values():
         sg.set_option(sg.SG_OPT_DENSE_LOG2, dl)
+        sg.set_option(sg.SG_OPT_VARIANT, var)
         (rp, col, val), _ = _run(N, thr)
         R = oracle.spgemm(A, A)
         assert np.array_equal(rp, R.row_ptr) and np.array_equal(col, R.col)
         assert np.all(val == 0)
+
+
+@pytest.mark.parametrize("name", ["C1", "rmat14"])
+def test_kernel_variants_same_c(options, name):
+    """Every SG_OPT_VARIANT computes the same C (integer values: bit-exact), equal to the oracle: the
+    warp-tile vs CTA rank kernels (bit 3) and the sorted warp light path vs the order-preserving hash
+    (bit 4), at a threshold that puts rows on both light and heavy paths."""
+    A = gen.config(name, mode="int")
+    R = oracle.spgemm(A, A)
+    dA = sg.DeviceCSR.from_host(A)
+    thr = sg.sg_sample_threshold(dA, dA, 0.05, 1)[0]
+    outs = []
+    for var in (0, 8, 16, 24):
+        sg.set_option(sg.SG_OPT_VARIANT, var)
+        (rp, col, val), info = _run(A, thr)
+        assert np.array_equal(rp, R.row_ptr)
+        compare_rows(rp, col, val, R, "f64", exact_values=True)
+        outs.append((col, val))
+    for col, val in outs[1:]:
+        assert np.array_equal(col, outs[0][0]) and np.array_equal(val, outs[0][1])

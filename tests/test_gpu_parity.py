@@ -484,10 +484,19 @@ def test_dense_window_integer_values_exact(dense_log2, dtype):
     assert info["n_dense"] == info["n_heavy"] > 0
 
 
+@pytest.fixture
+def hash_light():
+    old = sg.get_option(sg.SG_OPT_VARIANT)
+    sg.set_option(sg.SG_OPT_VARIANT, old | 16)
+    yield
+    sg.set_option(sg.SG_OPT_VARIANT, old)
+
+
 @pytest.mark.parametrize("scale,thr", [(14, 4096), (16, 1024)])
-def test_light_skewed_rows_sorted_path(scale, thr):
+def test_light_skewed_rows_sorted_path(scale, thr, hash_light):
     """Un-permuted R-MAT (hubs at low ids): light rows whose columns crowd the order-preserving
-    hash's homes take the uniform-hash + bitonic-sort path; C is unchanged (structure bit-exact)."""
+    hash's homes take the uniform-hash + bitonic-sort path; C is unchanged (structure bit-exact).
+    (SG_OPT_VARIANT bit 4: every light bin on the hash path, so the skew detection runs for all.)"""
     A = gen.rmat(scale, permute=False)
     (rp, col, val), info, _ = _full_product(A, A, thr)
     R = oracle.spgemm(A, A, with_absmag=True)
@@ -496,7 +505,7 @@ def test_light_skewed_rows_sorted_path(scale, thr):
     assert info["n_light_sorted"] > 0
 
 
-def test_light_sorted_path_integer_values_exact():
+def test_light_sorted_path_integer_values_exact(hash_light):
     A = gen.rmat(14, permute=False, mode="int")
     (rp, col, val), info, _ = _full_product(A, A, 4096)
     R = oracle.spgemm(A, A, with_absmag=True)
@@ -505,7 +514,7 @@ def test_light_sorted_path_integer_values_exact():
 
 
 @pytest.mark.parametrize("name", ["C2", "rmat16"])
-def test_uniform_rows_keep_the_order_preserving_path(name):
+def test_uniform_rows_keep_the_order_preserving_path(name, hash_light):
     """Permuted / uniform inputs: (almost) no light row is flagged as column-skewed."""
     A = gen.config(name)
     _, info, _ = _full_product(A, A, 4096)
