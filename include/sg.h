@@ -116,9 +116,13 @@ typedef struct sg_plan sg_plan;   /* opaque; owns only its workspace */
  *                      maximum carve-out, 0 (default) = off (measured no gain on C3: 239.9 vs 235.1 ms). The calls set the stream's access-policy window
  *                      for their own launches and clear it before returning; the device's persisting-L2 limit
  *                      is raised once (a process-wide setting).
+ *   SG_OPT_TP_MAX_BYTES  memory budget of the plan's B tile-pointer table (4 bytes x (long B rows) x (p/8192 + 1);
+ *                      it grows with rows x columns, not nnz): -1 (default) = 8 GiB; above the budget the
+ *                      heavy kernels locate B-row segments by binary search instead (same C, slower).
  * The environment seeds them once, at the library's first call (SG_VALIDATE=1, SG_DW_LOG2=m, SG_L2_PERSIST=b).
  * Errors: INVALID_ARG (unknown key or value out of range). sg_get_option: INT64_MIN if unknown. */
-typedef enum { SG_OPT_VALIDATE = 0, SG_OPT_DENSE_LOG2 = 1, SG_OPT_VARIANT = 2, SG_OPT_L2_PERSIST = 3, SG_OPT_COUNT = 4 } sg_option;
+typedef enum { SG_OPT_VALIDATE = 0, SG_OPT_DENSE_LOG2 = 1, SG_OPT_VARIANT = 2, SG_OPT_L2_PERSIST = 3, SG_OPT_TP_MAX_BYTES = 4,
+               SG_OPT_COUNT = 5 } sg_option;
 sg_status sg_set_option(int key, int64_t value);
 int64_t sg_get_option(int key);
 

@@ -42,7 +42,7 @@ EXPORTS = ["sg_status_string", "sg_version", "sg_default_cost_model", "sg_row_wo
            "sg_sym_c_create", "sg_sym_c_buffers", "sg_sym_c_layout", "sg_sym_c_assemble", "sg_sym_c_destroy",
            "sg_copy_device", "sg_default_cost_model_for", "sg_hh_filter", "sg_hh_hstack", "sg_hh_identity2", "sg_hh_sample"]
 
-SG_OPT_VALIDATE, SG_OPT_DENSE_LOG2, SG_OPT_VARIANT, SG_OPT_L2_PERSIST = 0, 1, 2, 3
+SG_OPT_VALIDATE, SG_OPT_DENSE_LOG2, SG_OPT_VARIANT, SG_OPT_L2_PERSIST, SG_OPT_TP_MAX_BYTES = 0, 1, 2, 3, 4
 
 
 class SgError(RuntimeError):

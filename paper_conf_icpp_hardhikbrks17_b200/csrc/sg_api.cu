@@ -44,6 +44,7 @@ struct sg_plan {
     int32_t* long_id = nullptr;
     uint32_t* tp = nullptr;
     int64_t nlong = 0;
+    int64_t nlong_tp = 0;           // nlong if the tile-pointer table is built, else 0 (over SG_OPT_TP_MAX_BYTES)
     int T = 0;
     unsigned long long* counter = nullptr;
     const int64_t* C_rp = nullptr;
@@ -115,6 +116,7 @@ void init_options() {
         e = getenv("SG_DW_LOG2");
         if (e && *e) g_opt[SG_OPT_DENSE_LOG2] = atoll(e);
         g_opt[SG_OPT_L2_PERSIST] = 0;
+        g_opt[SG_OPT_TP_MAX_BYTES] = -1;
         e = getenv("SG_L2_PERSIST");
         if (e && *e) g_opt[SG_OPT_L2_PERSIST] = atoll(e);
     });
@@ -403,6 +405,7 @@ sg_status sg_set_option(int key, int64_t value) {
     if (key == SG_OPT_DENSE_LOG2 && (value < -1 || value > 62)) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_VARIANT && (value < 0 || value > 31)) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_L2_PERSIST && value < -1) return SG_ERR_INVALID_ARG;
+    if (key == SG_OPT_TP_MAX_BYTES && value < -1) return SG_ERR_INVALID_ARG;
     g_opt[key] = value;
     return SG_OK;
 }
@@ -775,7 +778,16 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
         pl->nslots = hb[0];
         pl->amax = hb[1];
         pl->ranges = (RangeRec*)palloc(pl, sizeof(RangeRec) * (size_t)(pl->nslots > 0 ? pl->nslots : 1));
-        pl->tp = (uint32_t*)palloc(pl, 4 * (size_t)(pl->nlong > 0 ? pl->nlong : 1) * (size_t)(pl->T + 1));
+        // the tile-pointer table grows with (long B rows) x (tiles): over its budget the heavy kernels binary-search
+        // (the round-1 dense / symbolic kernels of SG_OPT_VARIANT bits 0-1 need the table: built regardless)
+        {
+            const int64_t opt = g_opt[SG_OPT_TP_MAX_BYTES].load();
+            const double budget = opt < 0 ? 8.0 * (1 << 30) : (double)opt;
+            const double need = 4.0 * (double)pl->nlong * (double)(pl->T + 1);
+            if (need > budget && !(pl->variant & 3)) pl->nlong_tp = 0;
+            else pl->nlong_tp = pl->nlong;
+        }
+        pl->tp = (uint32_t*)palloc(pl, 4 * (size_t)(pl->nlong_tp > 0 ? pl->nlong_tp : 1) * (size_t)(pl->T + 1));
         if (!pl->ranges || !pl->tp) return fail(SG_ERR_OOM);
         // unused range slots read as row -1 (the tile kernel walks every slot)
         CKF(cudaMemsetAsync(pl->ranges, 0xff, sizeof(RangeRec) * (size_t)(pl->nslots > 0 ? pl->nslots : 1), s));
@@ -788,7 +800,7 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
             pl->gscr = (int4*)palloc(pl, sizeof(int4) * (size_t)(heavy_grid() > dense_grid() ? heavy_grid() : dense_grid()) * (size_t)pl->amax);
             if (!pl->gscr) return fail(SG_ERR_OOM);
         }
-        if (pl->nlong > 0) CKF(launch_build_tp(b, pl->long_id, pl->T, pl->tp, s));
+        if (pl->nlong_tp > 0) CKF(launch_build_tp(b, pl->long_id, pl->T, pl->tp, s));
     }
     // a6 symbolic
     for (int k = 0; k < NBIN_LIGHT; ++k)
@@ -797,14 +809,14 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
                              (unsigned long long*)(pl->dbin + 2 * NBINS + 1), s));
     if (pl->variant & 2) {
         CKF(launch_sym_heavy(a, b, pl->heavy, pl->nheavy, nullptr, row_begin, pl->u, pl->range_off, pl->ranges,
-                             pl->nranges, pl->ndw, pl->dtc, pl->long_id, pl->nlong > 0 ? pl->tp : nullptr, pl->T,
+                             pl->nranges, pl->ndw, pl->dtc, pl->long_id, pl->nlong_tp > 0 ? pl->tp : nullptr, pl->T,
                              pl->counter, s, pl->nbig));
     } else if (pl->nheavy > 0) {
         const int64_t np = sym2_scratch_parts(pl->amax);
         void* pscr = np > 0 ? palloc(pl, part_bytes() * (size_t)np) : nullptr;
         if (np > 0 && !pscr) return fail(SG_ERR_OOM);
         CKF(launch_sym_heavy2(a, b, pl->heavy, pl->nheavy, nullptr, row_begin, pl->w, pl->u, pl->range_off, pl->ranges,
-                              pl->nranges, pl->ndw, pl->dtc, pl->long_id, pl->nlong > 0 ? pl->tp : nullptr, pl->T,
+                              pl->nranges, pl->ndw, pl->dtc, pl->long_id, pl->nlong_tp > 0 ? pl->tp : nullptr, pl->T,
                               pl->counter, s, pl->nbig, pscr, pl->amax));
     }
     CKF(scan_exclusive(pl->u, C_row_ptr, nr, stmp, s));
@@ -835,20 +847,21 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
                                  C_col, C_val, light_sorted(k, pl->p, pl->variant), s));
     if (pl->nheavy > 0) {
         if (pl->variant & 1)
-            CKP(pl, launch_num_dense(a, b, pl->heavy, pl->ndw, pl->rb, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
+            CKP(pl, launch_num_dense(a, b, pl->heavy, pl->ndw, pl->rb, pl->long_id, pl->nlong_tp > 0 ? pl->tp : nullptr, pl->T, pl->C_rp, C_col,
                                      C_val, pl->counter, pl->gscr, pl->amax, pl->dtc, pl->ditems, pl->ditem_off + pl->ndw, s));
         else
-            CKP(pl, launch_num_dense2(a, b, pl->heavy, pl->ndw, pl->rb, pl->w, pl->long_id, pl->tp, pl->T, pl->C_rp, C_col,
+            CKP(pl, launch_num_dense2(a, b, pl->heavy, pl->ndw, pl->rb, pl->w, pl->long_id, pl->nlong_tp > 0 ? pl->tp : nullptr, pl->T, pl->C_rp, C_col,
                                       C_val, pl->counter, pl->pscr, pl->pscr_cap, pl->dtc, pl->ditems,
                                       pl->ditem_off + pl->ndw, s));
         // rank rows: the CTA rank kernel takes the rows with more than tile_kreg() k entries, the warp-tile
         // kernel the rest (SG_OPT_VARIANT bit 3: the CTA kernel takes all of them)
         const bool tile = !(pl->variant & 8);
         CKP(pl, launch_num_heavy(a, b, pl->heavy, pl->ndw, pl->nheavy, pl->rb, pl->range_off, pl->nranges, pl->ranges,
-                                 pl->long_id, pl->tp, pl->T, pl->C_rp, C_col, C_val, pl->counter, pl->gscr, pl->amax,
+                                 pl->long_id, pl->nlong_tp > 0 ? pl->tp : nullptr, pl->T, pl->C_rp, C_col, C_val,
+                                 pl->counter, pl->gscr, pl->amax,
                                  tile ? (int)tile_kreg() : 0, s));
         if (tile && pl->nheavy > pl->ndw)
-            CKP(pl, launch_num_tile(a, b, pl->ranges, pl->nslots, pl->rb, pl->long_id, pl->nlong > 0 ? pl->tp : nullptr,
+            CKP(pl, launch_num_tile(a, b, pl->ranges, pl->nslots, pl->rb, pl->long_id, pl->nlong_tp > 0 ? pl->tp : nullptr,
                                     pl->T, pl->C_rp, C_col, C_val, pl->counter, s));
     }
     if (s != pl->s) {  // the plan's workspace frees (on pl->s) wait for this call's kernels

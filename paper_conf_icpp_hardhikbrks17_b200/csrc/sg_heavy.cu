@@ -392,6 +392,13 @@ __device__ unsigned long long g_hv_rng[24][4];
 __device__ unsigned long long g_hv_ph[24][5];
 #endif
 
+// seg_end that also serves long B rows when the plan has no tile pointers (table over its memory budget,
+// SG_OPT_TP_MAX_BYTES): a binary search of the row's remaining entries
+__device__ __forceinline__ int seg_end_any(const Mat& B, int cur, int e1, int q0, bool is_long, uint32_t tpv, int64_t hi) {
+    if (!is_long && e1 - cur > LONG_ROW) return (int)lower_bound_col(B.col, cur, e1, hi);
+    return seg_end(B, cur, e1, q0, is_long, tpv, hi);
+}
+
 template <class VT>
 __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
     Mat A, Mat B, const int32_t* __restrict__ heavy, int64_t h0, int64_t nheavy, int64_t rb, const int64_t* __restrict__ range_off,
@@ -440,7 +447,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
             const int k = __ldg(A.col + s0 + i);
             const int32_t q0 = (int32_t)__ldg(B.rp + k), q1 = (int32_t)__ldg(B.rp + k + 1);
             if (single) {
-                const int lid = q1 - q0 > LONG_ROW ? __ldg(long_id + k) : -1;
+                const int lid = tp && q1 - q0 > LONG_ROW ? __ldg(long_id + k) : -1;
                 S.c_cur[i] = q0; S.c_end[i] = q1; S.c_q0[i] = q0; S.c_lid[i] = lid;
                 S.c_a[i] = ldv<VT>(A.val, s0 + i);
                 if (lid >= 0 && nr > 0) tpv = __ldg(tp + (int64_t)lid * (T + 1) + rr[0].t1);
@@ -477,16 +484,16 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 if (i < na) {
                     if (single) {
                         const int cur = S.c_cur[i], lid = S.c_lid[i];
-                        const int end = seg_end(B, cur, S.c_end[i], S.c_q0[i], lid >= 0, tpv, hi);
+                        const int end = seg_end_any(B, cur, S.c_end[i], S.c_q0[i], lid >= 0, tpv, hi);
                         beg = cur; len = end - cur; a = S.c_a[i];
                         S.c_cur[i] = end;
                     } else {
                         const int4 g = gs[i];
                         const int k = __ldg(A.col + s0 + i);
                         const int32_t q0 = (int32_t)__ldg(B.rp + k), e1 = (int32_t)__ldg(B.rp + k + 1);
-                        const bool lng = e1 - q0 > LONG_ROW;
+                        const bool lng = tp && e1 - q0 > LONG_ROW;
                         const uint32_t tv = lng ? __ldg(tp + (int64_t)__ldg(long_id + k) * (T + 1) + R.t1) : 0u;
-                        const int end = seg_end(B, g.x, e1, q0, lng, tv, hi);
+                        const int end = seg_end_any(B, g.x, e1, q0, lng, tv, hi);
                         beg = g.x; len = end - g.x;
                         gs[i] = make_int4(end, 0, beg, len);
                     }

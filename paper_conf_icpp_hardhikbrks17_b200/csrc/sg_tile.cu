@@ -293,20 +293,15 @@ __global__ void __launch_bounds__(TT_T, TT_OCC) k_num_tile(
                 }
                 __syncwarp();
                 TT_MARK(3);
-                // ---- rank prefix: lane owns words [8 lane, 8 lane + 8) ----
+                // ---- rank prefix: lane owns words [4 lane, 4 lane + 4) and [128 + 4 lane, 128 + 4 lane + 4) (unit-stride
+                // 16-byte accesses: no bank conflicts); one warp scan per half ----
                 int ut;
-                {
 #if SG_TT_DUP
+                {
                     const uint4* b4 = reinterpret_cast<const uint4*>(S.bm) + 4 * lane;
                     const uint4 x0 = b4[0], x1 = b4[1], x2 = b4[2], x3 = b4[3];
                     const int c0 = __popc(x0.x), c1 = __popc(x0.z), c2 = __popc(x1.x), c3 = __popc(x1.z);
                     const int c4 = __popc(x2.x), c5 = __popc(x2.z), c6 = __popc(x3.x), c7 = __popc(x3.z);
-#else
-                    const uint4 w0 = reinterpret_cast<const uint4*>(S.bm)[2 * lane];
-                    const uint4 w1 = reinterpret_cast<const uint4*>(S.bm)[2 * lane + 1];
-                    const int c0 = __popc(w0.x), c1 = __popc(w0.y), c2 = __popc(w0.z), c3 = __popc(w0.w);
-                    const int c4 = __popc(w1.x), c5 = __popc(w1.y), c6 = __popc(w1.z), c7 = __popc(w1.w);
-#endif
                     const int sum = c0 + c1 + c2 + c3 + c4 + c5 + c6 + c7;
                     const int pinc = warp_incl_scan(sum);
                     ut = __shfl_sync(FULL, pinc, 31);
@@ -319,6 +314,23 @@ __global__ void __launch_bounds__(TT_T, TT_OCC) k_num_tile(
                     o.w = (uint32_t)p6 | ((uint32_t)p7 << 16);
                     reinterpret_cast<uint4*>(S.pref)[lane] = o;
                 }
+#else
+                {
+                    const uint4 w0 = reinterpret_cast<const uint4*>(S.bm)[lane];
+                    const uint4 w1 = reinterpret_cast<const uint4*>(S.bm)[32 + lane];
+                    const int c0 = __popc(w0.x), c1 = __popc(w0.y), c2 = __popc(w0.z), c3 = __popc(w0.w);
+                    const int c4 = __popc(w1.x), c5 = __popc(w1.y), c6 = __popc(w1.z), c7 = __popc(w1.w);
+                    const int s1 = c0 + c1 + c2 + c3, s2 = c4 + c5 + c6 + c7;
+                    const int i1 = warp_incl_scan(s1), i2 = warp_incl_scan(s2);
+                    const int t1 = __shfl_sync(FULL, i1, 31);
+                    ut = t1 + __shfl_sync(FULL, i2, 31);
+                    const int p0 = i1 - s1, p1 = p0 + c0, p2 = p1 + c1, p3 = p2 + c2;
+                    const int p4 = t1 + i2 - s2, p5 = p4 + c4, p6 = p5 + c5, p7 = p6 + c6;
+                    uint2* pr = reinterpret_cast<uint2*>(S.pref);
+                    pr[lane] = make_uint2((uint32_t)p0 | ((uint32_t)p1 << 16), (uint32_t)p2 | ((uint32_t)p3 << 16));
+                    pr[32 + lane] = make_uint2((uint32_t)p4 | ((uint32_t)p5 << 16), (uint32_t)p6 | ((uint32_t)p7 << 16));
+                }
+#endif
                 __syncwarp();
                 TT_MARK(4);
                 // ---- pass 2 (per rank window of CAPW): accumulate at rank(c); values out; clear ----
@@ -375,8 +387,8 @@ __global__ void __launch_bounds__(TT_T, TT_OCC) k_num_tile(
                     bm4[4 * lane + 2] = make_uint4(0, 0, 0, 0);
                     bm4[4 * lane + 3] = make_uint4(0, 0, 0, 0);
 #else
-                    bm4[2 * lane] = make_uint4(0, 0, 0, 0);
-                    bm4[2 * lane + 1] = make_uint4(0, 0, 0, 0);
+                    bm4[lane] = make_uint4(0, 0, 0, 0);
+                    bm4[32 + lane] = make_uint4(0, 0, 0, 0);
 #endif
                 }
                 out += ut;

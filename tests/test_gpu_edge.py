@@ -31,10 +31,11 @@ PATHS = {"light": (4096, 62, 0), "light_hash": (4096, 62, 16), "rank": (0, 62, 0
 
 @pytest.fixture
 def options():
-    old = (sg.get_option(sg.SG_OPT_DENSE_LOG2), sg.get_option(sg.SG_OPT_VARIANT))
+    old = (sg.get_option(sg.SG_OPT_DENSE_LOG2), sg.get_option(sg.SG_OPT_VARIANT), sg.get_option(sg.SG_OPT_TP_MAX_BYTES))
     yield
     sg.set_option(sg.SG_OPT_DENSE_LOG2, old[0])
     sg.set_option(sg.SG_OPT_VARIANT, old[1])
+    sg.set_option(sg.SG_OPT_TP_MAX_BYTES, old[2])
 
 
 def _run(A, thr):
@@ -138,3 +139,18 @@ def test_kernel_variants_same_c(options, name):
         outs.append((col, val))
     for col, val in outs[1:]:
         assert np.array_equal(col, outs[0][0]) and np.array_equal(val, outs[0][1])
+
+
+@pytest.mark.parametrize("path", ["rank", "rank_cta", "dense", "mixed"])
+def test_heavy_paths_without_tile_pointers(options, path):
+    """SG_OPT_TP_MAX_BYTES = 0: no B tile-pointer table (the table grows with rows x columns); every
+    heavy kernel finds its B-row segments by binary search and C is unchanged (integer values: bit-exact)."""
+    thr, dl, var = PATHS[path]
+    sg.set_option(sg.SG_OPT_DENSE_LOG2, dl)
+    sg.set_option(sg.SG_OPT_VARIANT, var)
+    sg.set_option(sg.SG_OPT_TP_MAX_BYTES, 0)
+    A = gen.config("rmat13", mode="int")
+    (rp, col, val), info = _run(A, thr)
+    R = oracle.spgemm(A, A)
+    assert np.array_equal(rp, R.row_ptr)
+    compare_rows(rp, col, val, R, "f64", exact_values=True)
