@@ -96,8 +96,10 @@ def main():
             light = (w > 0) & (w <= t)
             heavy = w > t
             arow = np.diff(H.row_ptr)
-            kl = sum(v[1] for k, v in bk.items() if k in ("k_sym_light", "k_num_light"))
-            kh = sum(v[1] for k, v in bk.items() if k in ("k_sym_heavy", "k_num_heavy", "k_num_dense"))
+            # light path: k_sym_light, k_num_light (hash) and k_num_light_sort (sorted warp path);
+            # heavy path: k_sym_heavy, the rank kernels k_num_heavy / k_num_tile and k_num_dense
+            kl = sum(v[1] for k, v in bk.items() if k.startswith(("k_sym_light", "k_num_light")))
+            kh = sum(v[1] for k, v in bk.items() if k in ("k_sym_heavy", "k_num_heavy", "k_num_tile", "k_num_dense"))
             rows.append({"t": t, "ms": ms, "ms_light": kl, "ms_heavy": kh, "r": r(t),
                          "L": [int(light.sum()), int(w[light].sum()), int(u[light].sum())],
                          "H": [int(heavy.sum()), int(w[heavy].sum()), int(u[heavy].sum()),
