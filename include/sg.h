@@ -109,8 +109,8 @@ typedef struct sg_plan sg_plan;   /* opaque; owns only its workspace */
  *                      kernel, k_sym_heavy in sg_heavy.cu; bit 2: row-major dense-window work items
  *                      instead of window-major ones; bit 3: the CTA rank kernel for every rank row instead of
  *                      the warp-tile kernel for rows of <= 64 k entries; bit 4: the order-preserving hash for
- *                      every light bin instead of the sorted warp path for w <= 512). Every variant computes
- *                      the same C.
+ *                      every light bin instead of the sorted warp path for w <= 512; bit 5: the warp-tile
+ *                      kernel even when a plan has fewer than 4096 rank rows). Every variant computes the same C.
  *   SG_OPT_L2_PERSIST  bytes of B.col kept in the persisting L2 carve-out during sg_symbolic / sg_numeric
  *                      (every heavy product gathers a column of B): -1 = all of B.col up to the device's
  *                      maximum carve-out, 0 (default) = off (measured no gain on C3: 239.9 vs 235.1 ms). The calls set the stream's access-policy window

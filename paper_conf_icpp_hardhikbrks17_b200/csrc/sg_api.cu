@@ -231,15 +231,18 @@ CostModelD cm_of(const sg_cost_model* c) {
 }
 
 // Default model: calibrated from the measured kernels (profiles/).
-// Refitted in round 2 on the round-2 kernels (sg_sym2.cu, sg_dense2.cu) by tools/sweep.py: non-negative
-// least squares of the per-class kernel times over the threshold grids of ER 2^18, R-MAT 18, un-permuted
-// R-MAT 18 and R-MAT 20 (C3) together, with R(u)'s floor tiles_fixed = ceil(p / 131072) per matrix
-// (profiles/r02_sweep_fitall.json "fit"), in ps of SM time. tiles_fixed here is the p <= 131072 value;
-// calls with cm == NULL use default_range_floor(B.ncols). (Round 1's constants, fitted before the heavy
-// kernels changed: 33399, 7915, 0, 0, 17907513, 1102, 68338, 209 with R(u) = max(1, ceil(u/12288)).)
+// Refitted for the round-2 final kernels (warp-tile rank kernel, sorted light path) by tools/sweep.py:
+// non-negative least squares of the per-class kernel times over the threshold grids of ER 2^18, R-MAT 18,
+// un-permuted R-MAT 18 and R-MAT 20 (C3) together, with R(u)'s floor tiles_fixed = ceil(p / 131072) per
+// matrix (profiles/r02g_sweep_precal2.json + r02g_sweep_precal_c3.json, joint fit in
+// profiles/r02g_costmodel_fit.txt), in ps of SM time. tiles_fixed here is the p <= 131072 value; calls with
+// cm == NULL use default_range_floor(B.ncols). (Earlier fits: round-2 mid 0, 9315, 0, 0, 5016705, 0, 74786,
+// 1854; round 1: 33399, 7915, 0, 0, 17907513, 1102, 68338, 209 with R(u) = max(1, ceil(u/12288)).)
+constexpr int64_t kTileMinRows = 4096;  // rank rows below which the warp-tile kernel is not used
+
 const sg_cost_model kDefaultModel = {
-    /*kappa_L*/ 0, /*lambda_L*/ 9315, /*sigma_L*/ 0, /*rho_L*/ 0,
-    /*kappa_H*/ 5016705, /*lambda_H*/ 0, /*tau_H*/ 74786, /*mu_H*/ 1854,
+    /*kappa_L*/ 0, /*lambda_L*/ 7079, /*sigma_L*/ 0, /*rho_L*/ 0,
+    /*kappa_H*/ 3723548, /*lambda_H*/ 0, /*tau_H*/ 46855, /*mu_H*/ 2169,
     /*tiles_fixed*/ 1, /*capu*/ 12288, /*cap_L*/ SG_CAP_L_MAX};
 
 // The heavy path's minimum number of column ranges per row: a row whose columns span [0, p) needs at
@@ -403,7 +406,7 @@ sg_status sg_set_option(int key, int64_t value) {
     if (key < 0 || key >= SG_OPT_COUNT) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_VALIDATE && value != 0 && value != 1) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_DENSE_LOG2 && (value < -1 || value > 62)) return SG_ERR_INVALID_ARG;
-    if (key == SG_OPT_VARIANT && (value < 0 || value > 31)) return SG_ERR_INVALID_ARG;
+    if (key == SG_OPT_VARIANT && (value < 0 || value > 63)) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_L2_PERSIST && value < -1) return SG_ERR_INVALID_ARG;
     if (key == SG_OPT_TP_MAX_BYTES && value < -1) return SG_ERR_INVALID_ARG;
     g_opt[key] = value;
@@ -784,7 +787,11 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
             const int64_t opt = g_opt[SG_OPT_TP_MAX_BYTES].load();
             const double budget = opt < 0 ? 8.0 * (1 << 30) : (double)opt;
             const double need = 4.0 * (double)pl->nlong * (double)(pl->T + 1);
-            if (need > budget && !(pl->variant & 3)) pl->nlong_tp = 0;
+            // ... and a table for a handful of heavy rows costs more than their binary searches (C2 at t = 512:
+            // 97 heavy rows, 262 K long B rows): build it when the heavy rows' tile lookups (~ nheavy x T)
+            // are at least a quarter of the long rows it covers
+            const bool few = (double)pl->nheavy * (double)pl->T < 0.25 * (double)pl->nlong;
+            if ((need > budget || few) && !(pl->variant & 3)) pl->nlong_tp = 0;
             else pl->nlong_tp = pl->nlong;
         }
         pl->tp = (uint32_t*)palloc(pl, 4 * (size_t)(pl->nlong_tp > 0 ? pl->nlong_tp : 1) * (size_t)(pl->T + 1));
@@ -855,7 +862,9 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
                                       pl->ditem_off + pl->ndw, s));
         // rank rows: the CTA rank kernel takes the rows with more than tile_kreg() k entries, the warp-tile
         // kernel the rest (SG_OPT_VARIANT bit 3: the CTA kernel takes all of them)
-        const bool tile = !(pl->variant & 8);
+        // (a few rank rows: the CTA kernel for all of them, its 16 warps per range shorten the latency tail
+        // of a warp walking a range's tiles alone)
+        const bool tile = !(pl->variant & 8) && (pl->nheavy - pl->ndw >= kTileMinRows || (pl->variant & 32));
         CKP(pl, launch_num_heavy(a, b, pl->heavy, pl->ndw, pl->nheavy, pl->rb, pl->range_off, pl->nranges, pl->ranges,
                                  pl->long_id, pl->nlong_tp > 0 ? pl->tp : nullptr, pl->T, pl->C_rp, C_col, C_val,
                                  pl->counter, pl->gscr, pl->amax,

@@ -22,11 +22,11 @@ sg = pytest.importorskip("paper_conf_icpp_hardhikbrks17_b200")
 
 # path -> (thr, dense_log2, variant): light = every row with w <= cap_L on the light kernels (the sorted
 # warp path for w <= 512, the order-preserving hash above; light_hash: the hash for every bin); rank =
-# every non-empty row heavy on the rank kernels (rows of <= 64 k entries on the warp-tile kernel, the rest
-# on the CTA kernel; rank_cta: the CTA kernel for all); dense = every non-empty row heavy on the
+# every non-empty row heavy on the rank kernels (rows of <= 64 k entries on the warp-tile kernel, forced by
+# variant bit 5 at these sizes, the rest on the CTA kernel; rank_cta: the CTA kernel for all); dense = every non-empty row heavy on the
 # dense-window kernel
-PATHS = {"light": (4096, 62, 0), "light_hash": (4096, 62, 16), "rank": (0, 62, 0), "rank_cta": (0, 62, 8),
-         "dense": (0, 0, 0), "mixed": (256, 10, 0)}
+PATHS = {"light": (4096, 62, 0), "light_hash": (4096, 62, 16), "rank": (0, 62, 32), "rank_cta": (0, 62, 8),
+         "dense": (0, 0, 0), "mixed": (256, 10, 32)}
 
 
 @pytest.fixture
@@ -124,14 +124,14 @@ def test_negative_zero_products_are_structural(options):
 @pytest.mark.parametrize("name", ["C1", "rmat14"])
 def test_kernel_variants_same_c(options, name):
     """Every SG_OPT_VARIANT computes the same C (integer values: bit-exact), equal to the oracle: the
-    warp-tile vs CTA rank kernels (bit 3) and the sorted warp light path vs the order-preserving hash
+    warp-tile vs CTA rank kernels (bits 3 and 5) and the sorted warp light path vs the order-preserving hash
     (bit 4), at a threshold that puts rows on both light and heavy paths."""
     A = gen.config(name, mode="int")
     R = oracle.spgemm(A, A)
     dA = sg.DeviceCSR.from_host(A)
     thr = sg.sg_sample_threshold(dA, dA, 0.05, 1)[0]
     outs = []
-    for var in (0, 8, 16, 24):
+    for var in (0, 8, 16, 24, 32, 48):
         sg.set_option(sg.SG_OPT_VARIANT, var)
         (rp, col, val), info = _run(A, thr)
         assert np.array_equal(rp, R.row_ptr)
