@@ -3,7 +3,7 @@
 # DRAM traffic of the bench command (-> profiles/ncu_traffic.json, read by bench.py for roofline.traffic),
 # the default bench line (C3 fp64, e2e + CPU oracle baseline), the fp32 line, C2 and R-MAT 18 lines.
 #   bash tools/final_measure.sh <tag>
-T=${1:-r02}
+T=${1:-r02g}
 O=gpurun_out
 export PYTORCH_CUDA_ALLOC_CONF=expandable_segments:True
 timeout 1800 python -m pytest tests -m gpu -q -p no:cacheprovider > $O/${T}_gpu_tests.log 2>&1; tail -2 $O/${T}_gpu_tests.log
@@ -17,3 +17,4 @@ timeout 1500 python bench.py > $O/${T}_bench_c3.log 2>&1; tail -1 $O/${T}_bench_
 timeout 600 python bench.py --dtype f32 --no-e2e > $O/${T}_bench_c3_f32.log 2>&1; tail -1 $O/${T}_bench_c3_f32.log | cut -c1-200
 timeout 300 python bench.py --config C2 --steps 20 --warmup 5 --no-e2e --no-cpu --no-profile > $O/${T}_bench_c2.log 2>&1; tail -1 $O/${T}_bench_c2.log | cut -c1-200
 timeout 300 python bench.py --config R18 --steps 10 --warmup 3 --no-e2e --no-cpu > $O/${T}_bench_r18.log 2>&1; tail -1 $O/${T}_bench_r18.log | cut -c1-200
+python tools/step_breakdown.py --config C2 > $O/${T}_c2_breakdown.txt 2>&1; tail -2 $O/${T}_c2_breakdown.txt
