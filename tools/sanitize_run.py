@@ -25,17 +25,22 @@ def main():
     from _util import compare_rows
     cases = [  # (label, matrix, thr, dense_log2, variant)
         ("light+rank", gen.rmat(a.scale), 256, 62, 0),
+        ("light (sorted warp path) + rank (warp-tile)", gen.rmat(a.scale), 256, 62, 32),
+        ("light (hash path) + rank (CTA)", gen.rmat(a.scale), 256, 62, 8 | 16),
         ("rank only", gen.rmat(a.scale), 0, 62, 0),
+        ("rank only, warp-tile forced", gen.rmat(a.scale, mode="signed"), 0, 62, 32),
         ("dense2 only", gen.rmat(a.scale, mode="signed"), 0, 0, 0),
         ("dense (round-1) only", gen.rmat(a.scale, mode="signed"), 0, 0, 1),
         ("mixed default", gen.rmat(a.scale + 2), -1, -1, 0),
         ("sorted light (unpermuted)", gen.rmat(a.scale + 1, permute=False, mode="zeros"), 4096, -1, 0),
         ("fp32", gen.rmat(a.scale, dtype="f32"), 64, 8, 0),
     ]
+    cases.append(("no tile pointers, warp-tile + CTA rank + dense2", gen.rmat(a.scale, mode="signed"), 0, 10, 32 | 128))
     ok = True
     for label, A, thr, dl, var in cases:
         sg.set_option(sg.SG_OPT_DENSE_LOG2, dl)
-        sg.set_option(sg.SG_OPT_VARIANT, var)
+        sg.set_option(sg.SG_OPT_VARIANT, var & 127)
+        sg.set_option(sg.SG_OPT_TP_MAX_BYTES, 0 if var & 128 else -1)
         dA = sg.DeviceCSR.from_host(A)
         t = thr if thr >= 0 else sg.sg_sample_threshold(dA, dA, 0.05, 3)[0]
         plan = sg.sg_symbolic(dA, dA, t)
@@ -45,7 +50,8 @@ def main():
         rp = plan.row_ptr.cpu().numpy()
         try:
             assert np.array_equal(rp, R.row_ptr)
-            compare_rows(rp, col.cpu().numpy(), val.cpu().numpy(), R, A.dtype, exact_values=A.val.dtype != np.float32 and label != "light+rank" and label != "rank only" and label != "mixed default")
+            exact = bool(np.all(A.val == np.round(A.val)))  # integer-valued inputs: sums exact, values bit-exact
+            compare_rows(rp, col.cpu().numpy(), val.cpu().numpy(), R, A.dtype, exact_values=exact)
             print(f"{label}: OK (nnz {plan.nnz}, info {plan.info()['n_heavy']} heavy / {plan.info()['n_dense']} dense)", flush=True)
         except AssertionError as e:
             ok = False
@@ -53,6 +59,7 @@ def main():
         plan.destroy()
     sg.set_option(sg.SG_OPT_DENSE_LOG2, -1)
     sg.set_option(sg.SG_OPT_VARIANT, 0)
+    sg.set_option(sg.SG_OPT_TP_MAX_BYTES, -1)
     print("ALL OK" if ok else "SOME FAILED")
 
 
