@@ -4,6 +4,16 @@
 #include "sg_internal.cuh"
 #include <climits>
 
+// Bounds assertions of a debug build (-DSG_DEBUG_BOUNDS, tools/ab_builds / the GPU tests with SG_LIB_PATH):
+// every kernel's output count per row / range against the symbolic plan, cursor and rank ranges. A failed
+// assert traps the kernel, so the call returns SG_ERR_CUDA and the test fails. Compiled out by default.
+#if defined(SG_DEBUG_BOUNDS)
+#include <cassert>
+#define SG_BOUND(cond) assert(cond)
+#else
+#define SG_BOUND(cond) do { } while (0)
+#endif
+
 namespace sg {
 
 constexpr unsigned FULL = 0xffffffffu;

@@ -542,6 +542,7 @@ __global__ void __launch_bounds__(NUM_T, NUM_OCC) k_num_heavy(
                 int t2;
                 if (kBulk && tid == 0) bulk_wait_read();  // previous range's values have left shared memory
                 const int p0 = block_scan<NUM_T>(c0 + c1 + c2 + c3 + c4 + c5 + c6 + c7, &t2, S.ws);
+                SG_BOUND(t2 == R.cnt);  // the range's bitmap holds exactly the plan's entries
                 if (kBulk) {
                     for (int e = tid; e < clear_n; e += NUM_T) S.vals[e] = 0.0;
                     clear_n = 0;

@@ -574,6 +574,7 @@ __global__ void __launch_bounds__(32 * R, 1024 / (32 * R)) k_num_light_sort(Mat 
             jb += tot;
         }
         const int w = jb;  // <= U (the bin bound)
+        SG_BOUND(w <= U);
         for (int j = w + lane; j < U; j += 32) sk[j] = 0xFFFFFFFFu;
         __syncwarp();
         // ---- sort (blocked: lane holds keys [lane E, lane E + E)) ----
@@ -607,6 +608,7 @@ __global__ void __launch_bounds__(32 * R, 1024 / (32 * R)) k_num_light_sort(Mat 
             }
             pos0 += __popc(m);
         }
+        SG_BOUND(base + pos0 == C_rp[li + 1]);  // exactly the symbolic pass's u_i entries
         __syncwarp();  // sk / sv reused by the next row
     }
 }

@@ -239,6 +239,7 @@ __global__ void __launch_bounds__(TT_T, TT_OCC) k_num_tile(
                     L.l1 = e1 - k1.cur;
                     k1.cur = e1;
                 }
+                SG_BOUND(L.l0 >= 0 && L.l1 >= 0 && k0.cur <= k0.q1 && k1.cur <= k1.q1);
                 const int len = L.l0 + L.l1;
                 const int inc = warp_incl_scan(len);
                 L.tot = __shfl_sync(FULL, inc, 31);
@@ -331,6 +332,7 @@ __global__ void __launch_bounds__(TT_T, TT_OCC) k_num_tile(
                     pr[32 + lane] = make_uint2((uint32_t)p4 | ((uint32_t)p5 << 16), (uint32_t)p6 | ((uint32_t)p7 << 16));
                 }
 #endif
+                SG_BOUND(out + ut <= C_rp[R.row + 1]);
                 __syncwarp();
                 TT_MARK(4);
                 // ---- pass 2 (per rank window of CAPW): accumulate at rank(c); values out; clear ----
@@ -398,6 +400,7 @@ __global__ void __launch_bounds__(TT_T, TT_OCC) k_num_tile(
                 if (lane == 0) { tph[8] += ut; tph[9] += 1; }
 #endif
             }
+            SG_BOUND(out == C_rp[R.row] + R.off + R.cnt);  // the range holds exactly the plan's entries
 #if defined(SG_TT_EXP)
             if (lane == 0) tph[7] += 1;
 #endif
