@@ -28,13 +28,13 @@ namespace sg {
 #define SG_TT_WARPS 4
 #endif
 #ifndef SG_TT_OCC
-#define SG_TT_OCC 6
+#define SG_TT_OCC 7
 #endif
 #ifndef SG_CAPW
-#define SG_CAPW 768
+#define SG_CAPW 640
 #endif
 #ifndef SG_TT_CHUNK
-#define SG_TT_CHUNK 4
+#define SG_TT_CHUNK 1
 #endif
 #ifndef SG_TT_NB
 #define SG_TT_NB 4
@@ -45,7 +45,11 @@ constexpr int TT_OCC = SG_TT_OCC;      // CTAs per SM (shared-memory bound)
 constexpr int CAPW = SG_CAPW;          // accumulator entries per warp
 constexpr int TT_CHUNK = SG_TT_CHUNK;  // range slots taken per counter increment
 constexpr int NB = SG_TT_NB;           // batches of 32 products per round (the first round stays in registers)
-constexpr int KREG = 64;               // rows with at most KREG k entries (two per lane)
+#ifndef SG_KREG
+#define SG_KREG 64
+#endif
+constexpr int KREG = SG_KREG;          // rows with at most KREG (<= 64) k entries (up to two per lane)
+static_assert(KREG <= 64, "two k entries per lane at most");
 constexpr int TWW = TW / 32;           // bitmap words per tile
 static_assert(TWW == 8 * 32, "prefix layout: 8 words per lane");
 
