@@ -37,6 +37,8 @@ struct sg_plan {
     int64_t nskew = 0;              // light rows on the sorted path (column-skewed; sg_light.cu)
     int dw_log2 = 0;
     int2* span = nullptr;           // light rows: [cmin, cmax] of the output columns
+    uint32_t* lkeys = nullptr;      // sorted light bins: each row's sorted column keys (symbolic -> numeric)
+    int64_t lkey_off[NBIN_LIGHT] = {0};
     int4* gscr = nullptr;           // heavy rows with more than KC entries: per-k cursor scratch
     void* pscr = nullptr;           // dense2: per-CTA part scratch for rows with many k entries
     int64_t pscr_cap = 0;
@@ -809,11 +811,27 @@ sg_status sg_symbolic(const sg_csr_view* A, const sg_csr_view* B, int64_t thr, i
         }
         if (pl->nlong_tp > 0) CKF(launch_build_tp(b, pl->long_id, pl->T, pl->tp, s));
     }
-    // a6 symbolic
-    for (int k = 0; k < NBIN_LIGHT; ++k)
-        CKF(launch_sym_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], nullptr, row_begin, pl->u,
-                             light_sorted(k, pl->p, pl->variant) ? nullptr : pl->span,
-                             (unsigned long long*)(pl->dbin + 2 * NBINS + 1), s));
+    // a6 symbolic. Light bins on the sorted path sort their rows' column keys here and keep them for the
+    // numeric pass (one slot of light_sort_width(b) keys per row, bin by bin); the others count with a hash set.
+    {
+        int64_t nkeys = 0;
+        for (int k = 0; k < NBIN_LIGHT; ++k) {
+            pl->lkey_off[k] = nkeys;
+            if (light_sorted(k, pl->p, pl->variant)) nkeys += pl->bin_cnt[k] * (int64_t)light_sort_width(k);
+        }
+        if (nkeys > 0) {
+            pl->lkeys = (uint32_t*)palloc(pl, 4 * (size_t)nkeys);
+            if (!pl->lkeys) return fail(SG_ERR_OOM);
+        }
+    }
+    for (int k = 0; k < NBIN_LIGHT; ++k) {
+        if (light_sorted(k, pl->p, pl->variant))
+            CKF(launch_sym_light_sort(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], row_begin,
+                                      pl->lkeys + pl->lkey_off[k], pl->u, s));
+        else
+            CKF(launch_sym_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], nullptr, row_begin, pl->u, pl->span,
+                                 (unsigned long long*)(pl->dbin + 2 * NBINS + 1), s));
+    }
     if (pl->variant & 2) {
         CKF(launch_sym_heavy(a, b, pl->heavy, pl->nheavy, nullptr, row_begin, pl->u, pl->range_off, pl->ranges,
                              pl->nranges, pl->ndw, pl->dtc, pl->long_id, pl->nlong_tp > 0 ? pl->tp : nullptr, pl->T,
@@ -849,9 +867,14 @@ sg_status sg_numeric(sg_plan* pl, const sg_csr_view* A, const sg_csr_view* B, in
     if (pl->nnz_c == 0) return SG_OK;
     Mat a = mat_of(A), b = mat_of(B);
     L2Window l2w(s, b.col, 4 * (size_t)b.nnz);
-    for (int k = 0; k < NBIN_LIGHT; ++k)
-        CKP(pl, launch_num_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], pl->rb, pl->span, pl->C_rp,
-                                 C_col, C_val, light_sorted(k, pl->p, pl->variant), s));
+    for (int k = 0; k < NBIN_LIGHT; ++k) {
+        if (light_sorted(k, pl->p, pl->variant))
+            CKP(pl, launch_num_light_keys(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], pl->rb,
+                                          pl->lkeys + pl->lkey_off[k], pl->C_rp, C_col, C_val, s));
+        else
+            CKP(pl, launch_num_light(k, a, b, pl->lists + pl->bin_off[k], pl->bin_cnt[k], pl->rb, pl->span, pl->C_rp,
+                                     C_col, C_val, s));
+    }
     if (pl->nheavy > 0) {
         if (pl->variant & 1)
             CKP(pl, launch_num_dense(a, b, pl->heavy, pl->ndw, pl->rb, pl->long_id, pl->nlong_tp > 0 ? pl->tp : nullptr, pl->T, pl->C_rp, C_col,

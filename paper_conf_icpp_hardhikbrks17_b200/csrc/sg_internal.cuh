@@ -100,8 +100,16 @@ cudaError_t launch_sym_light(int b, const Mat& A, const Mat& B, const int32_t* l
 // light bin b takes the sorted warp path of the numeric pass for B with p columns (no span / skew
 // information needed from the symbolic pass then); SG_OPT_VARIANT bit 4 keeps the order-preserving hash
 bool light_sorted(int b, int64_t p, int variant);
+// the sorted light path, split over the passes: the symbolic pass sorts each row's column keys into the row's
+// slot of light_sort_width(b) keys (keys + list position x width) and writes u_i; the numeric pass gathers
+// the values and emits C from the stored keys
+int light_sort_width(int b);
+cudaError_t launch_sym_light_sort(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, int64_t rb,
+                                  uint32_t* keys, int64_t* u, cudaStream_t s);
+cudaError_t launch_num_light_keys(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, int64_t rb,
+                                  const uint32_t* keys, const int64_t* C_rp, int32_t* C_col, void* C_val, cudaStream_t s);
 cudaError_t launch_num_light(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, int64_t rb,
-                             const int2* span, const int64_t* C_rp, int32_t* C_col, void* C_val, bool sorted, cudaStream_t s);
+                             const int2* span, const int64_t* C_rp, int32_t* C_col, void* C_val, cudaStream_t s);
 // heavy path (sg_heavy.cu)
 cudaError_t launch_long_rows(const Mat& B, int32_t* long_id, int64_t* d_nlong, cudaStream_t s);
 cudaError_t launch_build_tp(const Mat& B, const int32_t* long_id, int T, uint32_t* tp, cudaStream_t s);

@@ -512,14 +512,20 @@ __device__ __forceinline__ void bitonic_warp_blocked(uint32_t (&x)[N / 32]) {
     }
 }
 
-template <int U, int R, class VT>
-__global__ void __launch_bounds__(32 * R, 1024 / (32 * R)) k_num_light_sort(Mat A, Mat B, const int32_t* __restrict__ list, int64_t cnt,
-                                                          int64_t rb, const int64_t* __restrict__ C_rp,
-                                                          int32_t* __restrict__ C_col, VT* __restrict__ C_val) {
+// The sorted path is split between the two passes: the SYMBOLIC pass gathers the row's columns, sorts the
+// keys and keeps them (the row's slot of U keys in a plan buffer; u_i = the number of column runs); the
+// NUMERIC pass gathers only the values, in the same product order j, and emits from the stored keys.
+// MODE 1: symbolic (columns -> sorted keys, u_i); MODE 2: numeric (values + stored keys -> C).
+template <int U, int R, class VT, int MODE>
+__global__ void __launch_bounds__(32 * R, 1024 / (32 * R)) k_light_sort(Mat A, Mat B, const int32_t* __restrict__ list,
+                                                                     int64_t cnt, int64_t rb, uint32_t* __restrict__ keys,
+                                                                     int64_t* __restrict__ u, const int64_t* __restrict__ C_rp,
+                                                                     int32_t* __restrict__ C_col, VT* __restrict__ C_val) {
     static_assert(U >= 32 && (U & (U - 1)) == 0, "U: a power of two >= 32");
     constexpr int E = U / 32, LOGU = __builtin_ctz(U);
+    constexpr bool VALS = MODE == 2;
     __shared__ __align__(16) uint32_t skeys[R][U];
-    __shared__ double svals[R][U];
+    __shared__ double svals[R][VALS ? U : 1];
     const int g = threadIdx.x >> 5, lane = threadIdx.x & 31;
     uint32_t* sk = skeys[g];
     double* sv = svals[g];
@@ -527,7 +533,8 @@ __global__ void __launch_bounds__(32 * R, 1024 / (32 * R)) k_num_light_sort(Mat 
         const int64_t li = list[jr];
         const int64_t row = rb + li;
         const int64_t s0 = __ldg(A.rp + row), s1 = __ldg(A.rp + row + 1);
-        // ---- gather: product j -> key (c << LOGU) | j, value at sv[j] ----
+        uint32_t* rk = keys + jr * U;  // the row's key slot
+        // ---- gather: product j -> key (c << LOGU) | j (symbolic) or value a_ik b_kj at sv[j] (numeric) ----
         int jb = 0;
         for (int64_t pb = s0; pb < s1; pb += 32) {
             const int64_t pa = pb + lane;
@@ -538,13 +545,13 @@ __global__ void __launch_bounds__(32 * R, 1024 / (32 * R)) k_num_light_sort(Mat 
                 const int k = __ldg(A.col + pa);
                 q0 = __ldg(B.rp + k);
                 len = (int)(__ldg(B.rp + k + 1) - q0);
-                a = ldv<VT>(A.val, pa);
+                if (VALS) a = ldv<VT>(A.val, pa);
             }
             const int inc = warp_incl_scan(len);
             const int off = inc - len;
             const int tot = __shfl_sync(FULL, inc, 31);
             for (int j0 = 0; j0 < tot; j0 += 32 * SORT_UNR) {
-                int c[SORT_UNR], jj[SORT_UNR];
+                int c[SORT_UNR];
                 double v[SORT_UNR];
                 #pragma unroll
                 for (int r = 0; r < SORT_UNR; ++r) {
@@ -556,78 +563,94 @@ __global__ void __launch_bounds__(32 * R, 1024 / (32 * R)) k_num_light_sort(Mat 
                         if (o <= j) sl += bb;
                     }
                     const int64_t q = __shfl_sync(FULL, q0, sl) + (j - __shfl_sync(FULL, off, sl));
-                    const double as = __shfl_sync(FULL, a, sl);
+                    const double as = VALS ? __shfl_sync(FULL, a, sl) : 0.0;
                     c[r] = -1;
-                    jj[r] = jb + j;
                     if (j < tot) {
-                        c[r] = __ldg(B.col + q);
-                        v[r] = as * ldv<VT>(B.val, q);
+                        if (VALS) { c[r] = 0; v[r] = as * ldv<VT>(B.val, q); }
+                        else c[r] = __ldg(B.col + q);
                     }
                 }
                 #pragma unroll
                 for (int r = 0; r < SORT_UNR; ++r)
                     if (c[r] >= 0) {
-                        sk[jj[r]] = ((uint32_t)c[r] << LOGU) | (uint32_t)jj[r];
-                        sv[jj[r]] = v[r];
+                        const int jj = jb + j0 + 32 * r + lane;
+                        if (VALS) sv[jj] = v[r];
+                        else sk[jj] = ((uint32_t)c[r] << LOGU) | (uint32_t)jj;
                     }
             }
             jb += tot;
         }
         const int w = jb;  // <= U (the bin bound)
         SG_BOUND(w <= U);
-        for (int j = w + lane; j < U; j += 32) sk[j] = 0xFFFFFFFFu;
-        __syncwarp();
-        // ---- sort (blocked: lane holds keys [lane E, lane E + E)) ----
-        uint32_t x[E];
-        #pragma unroll
-        for (int r = 0; r < E; ++r) x[r] = sk[lane * E + r];
-        bitonic_warp_blocked<U>(x);
-        __syncwarp();
-        #pragma unroll
-        for (int r = 0; r < E; ++r) sk[lane * E + r] = x[r];
-        __syncwarp();
-        // ---- runs of equal columns -> one entry each, in order ----
-        const int64_t base = C_rp[li];
-        int pos0 = 0;
-        for (int e0 = 0; e0 < w; e0 += 32) {
-            const int e = e0 + lane;
-            const uint32_t key = e < w ? sk[e] : 0xFFFFFFFFu;
-            const uint32_t col = key >> LOGU;
-            const bool head = e < w && (e == 0 || (sk[e - 1] >> LOGU) != col);
-            const unsigned m = __ballot_sync(FULL, head);
-            if (head) {
-                double sum = sv[key & (U - 1)];
-                for (int t = e + 1; t < w; ++t) {
-                    const uint32_t kt = sk[t];
-                    if ((kt >> LOGU) != col) break;
-                    sum += sv[kt & (U - 1)];
-                }
-                const int64_t o = base + pos0 + __popc(m & lanemask_lt());
-                st_out(C_col + o, (int32_t)col);
-                st_out(C_val + o, (VT)sum);
+        if constexpr (MODE == 1) {
+            for (int j = w + lane; j < U; j += 32) sk[j] = 0xFFFFFFFFu;
+            __syncwarp();
+            // ---- sort (blocked: lane holds keys [lane E, lane E + E)); keep; count the column runs ----
+            uint32_t x[E];
+            #pragma unroll
+            for (int r = 0; r < E; ++r) x[r] = sk[lane * E + r];
+            bitonic_warp_blocked<U>(x);
+            if constexpr (E % 4 == 0) {
+                #pragma unroll
+                for (int r = 0; r < E; r += 4)
+                    *reinterpret_cast<uint4*>(rk + lane * E + r) = make_uint4(x[r], x[r + 1], x[r + 2], x[r + 3]);
+            } else {
+                #pragma unroll
+                for (int r = 0; r < E; ++r) rk[lane * E + r] = x[r];
             }
-            pos0 += __popc(m);
+            const uint32_t prev_last = __shfl_up_sync(FULL, x[E - 1], 1);
+            int heads = 0;
+            #pragma unroll
+            for (int r = 0; r < E; ++r) {
+                const int i = lane * E + r;
+                const uint32_t prev = r > 0 ? x[r - 1] : prev_last;
+                heads += (i < w && (i == 0 || (prev >> LOGU) != (x[r] >> LOGU))) ? 1 : 0;
+            }
+            heads = warp_sum(heads);
+            if (lane == 0) u[li] = heads;
+            __syncwarp();  // sk reused by the next row
+        } else {
+            // ---- the stored keys; runs of equal columns -> one entry each, in order ----
+            for (int e = lane; e < w; e += 32) sk[e] = rk[e];
+            __syncwarp();
+            const int64_t base = C_rp[li];
+            int pos0 = 0;
+            for (int e0 = 0; e0 < w; e0 += 32) {
+                const int e = e0 + lane;
+                const uint32_t key = e < w ? sk[e] : 0xFFFFFFFFu;
+                const uint32_t col = key >> LOGU;
+                const bool head = e < w && (e == 0 || (sk[e - 1] >> LOGU) != col);
+                const unsigned m = __ballot_sync(FULL, head);
+                if (head) {
+                    double sum = sv[key & (U - 1)];
+                    for (int t = e + 1; t < w; ++t) {
+                        const uint32_t kt = sk[t];
+                        if ((kt >> LOGU) != col) break;
+                        sum += sv[kt & (U - 1)];
+                    }
+                    const int64_t o = base + pos0 + __popc(m & lanemask_lt());
+                    st_out(C_col + o, (int32_t)col);
+                    st_out(C_val + o, (VT)sum);
+                }
+                pos0 += __popc(m);
+            }
+            SG_BOUND(base + pos0 == C_rp[li + 1]);  // exactly the symbolic pass's u_i entries
+            __syncwarp();  // sk / sv reused by the next row
         }
-        SG_BOUND(base + pos0 == C_rp[li + 1]);  // exactly the symbolic pass's u_i entries
-        __syncwarp();  // sk / sv reused by the next row
     }
 }
 
-// the sorted warp path applies to bin b (U = 2^b) when its keys fit: c < 2^(32 - log2 max(U, 32))
-#ifndef SG_LIGHT_SORT
-#define SG_LIGHT_SORT 1
-#endif
-bool light_sorted(int b, int64_t p, int variant) {
-    const int lu = b < 5 ? 5 : b;
-    return SG_LIGHT_SORT && !(variant & 16) && b <= 9 && p <= ((int64_t)1 << (32 - lu));
-}
+// key-slot width of bin b on the sorted path (keys per row)
+int light_sort_width(int b) { return b < 5 ? 32 : (1 << b); }
 
-template <class VT>
-static cudaError_t num_light_sort_V(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, int64_t rb,
-                                    const int64_t* C_rp, int32_t* C_col, void* C_val, cudaStream_t s) {
-#define SG_SORT_CASE(U_, R_)                                                                              \
-    SG_LAUNCH("k_num_light_sort", s, (k_num_light_sort<U_, R_, VT><<<grid_for(cnt, R_, 148 * 32), 32 * R_, 0, s>>>( \
-                                         A, B, list, cnt, rb, C_rp, C_col, (VT*)C_val)));                  \
+template <class VT, int MODE>
+static cudaError_t light_sort_V(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, int64_t rb,
+                                uint32_t* keys, int64_t* u, const int64_t* C_rp, int32_t* C_col, void* C_val,
+                                cudaStream_t s) {
+    const char* nm = MODE == 1 ? "k_sym_light_sort" : "k_num_light_sort";
+#define SG_SORT_CASE(U_, R_)                                                                                   \
+    SG_LAUNCH(nm, s, (k_light_sort<U_, R_, VT, MODE><<<grid_for(cnt, R_, 148 * 32), 32 * R_, 0, s>>>(            \
+                         A, B, list, cnt, rb, keys, u, C_rp, C_col, (VT*)C_val)));                             \
     break;
     switch (b) {
         case 0: case 1: case 2: case 3: case 4: case 5: SG_SORT_CASE(32, 8)
@@ -639,6 +662,29 @@ static cudaError_t num_light_sort_V(int b, const Mat& A, const Mat& B, const int
     }
 #undef SG_SORT_CASE
     return cudaGetLastError();
+}
+
+cudaError_t launch_sym_light_sort(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, int64_t rb,
+                                  uint32_t* keys, int64_t* u, cudaStream_t s) {
+    if (cnt <= 0) return cudaSuccess;
+    return light_sort_V<double, 1>(b, A, B, list, cnt, rb, keys, u, nullptr, nullptr, nullptr, s);
+}
+
+cudaError_t launch_num_light_keys(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, int64_t rb,
+                                  const uint32_t* keys, const int64_t* C_rp, int32_t* C_col, void* C_val, cudaStream_t s) {
+    if (cnt <= 0) return cudaSuccess;
+    uint32_t* k = const_cast<uint32_t*>(keys);
+    return A.dt == 0 ? light_sort_V<double, 2>(b, A, B, list, cnt, rb, k, nullptr, C_rp, C_col, C_val, s)
+                     : light_sort_V<float, 2>(b, A, B, list, cnt, rb, k, nullptr, C_rp, C_col, C_val, s);
+}
+
+// the sorted warp path applies to bin b (U = 2^b) when its keys fit: c < 2^(32 - log2 max(U, 32))
+#ifndef SG_LIGHT_SORT
+#define SG_LIGHT_SORT 1
+#endif
+bool light_sorted(int b, int64_t p, int variant) {
+    const int lu = b < 5 ? 5 : b;
+    return SG_LIGHT_SORT && !(variant & 16) && b <= 9 && p <= ((int64_t)1 << (32 - lu));
 }
 
 template <class VT>
@@ -679,12 +725,8 @@ static cudaError_t num_light_V(int b, const Mat& A, const Mat& B, const int32_t*
 }
 
 cudaError_t launch_num_light(int b, const Mat& A, const Mat& B, const int32_t* list, int64_t cnt, int64_t rb,
-                             const int2* span, const int64_t* C_rp, int32_t* C_col, void* C_val, bool sorted,
-                             cudaStream_t s) {
+                             const int2* span, const int64_t* C_rp, int32_t* C_col, void* C_val, cudaStream_t s) {
     if (cnt <= 0) return cudaSuccess;
-    if (sorted)
-        return A.dt == 0 ? num_light_sort_V<double>(b, A, B, list, cnt, rb, C_rp, C_col, C_val, s)
-                         : num_light_sort_V<float>(b, A, B, list, cnt, rb, C_rp, C_col, C_val, s);
     return A.dt == 0 ? num_light_V<double>(b, A, B, list, cnt, rb, span, C_rp, C_col, C_val, s)
                      : num_light_V<float>(b, A, B, list, cnt, rb, span, C_rp, C_col, C_val, s);
 }
