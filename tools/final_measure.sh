@@ -3,7 +3,7 @@
 # DRAM traffic of the bench command (-> profiles/ncu_traffic.json, read by bench.py for roofline.traffic),
 # the default bench line (C3 fp64, e2e + CPU oracle baseline), the fp32 line, C2 and R-MAT 18 lines.
 #   bash tools/final_measure.sh <tag>
-T=${1:-r02g}
+T=${1:-r02h}
 O=gpurun_out
 export PYTORCH_CUDA_ALLOC_CONF=expandable_segments:True
 timeout 1800 python -m pytest tests -m gpu -q -p no:cacheprovider > $O/${T}_gpu_tests.log 2>&1; tail -2 $O/${T}_gpu_tests.log
