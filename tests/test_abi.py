@@ -62,6 +62,17 @@ def test_options_roundtrip_and_validation():
         with pytest.raises(sg.SgError, match="INVALID_ARG"):
             sg.set_option(99, 0)
         assert sg.load().sg_get_option(99) == -(2**63)
+        # defaults: fixed-size tile-pointer budget (-1 = 8 GiB), no L2 persisting window, kernel variant 0
+        assert sg.get_option(sg.SG_OPT_TP_MAX_BYTES) == -1
+        assert sg.get_option(sg.SG_OPT_L2_PERSIST) == 0
+        assert sg.get_option(sg.SG_OPT_VARIANT) == 0
+        for key, good, bad in ((sg.SG_OPT_VARIANT, 63, 64), (sg.SG_OPT_TP_MAX_BYTES, 0, -2), (sg.SG_OPT_L2_PERSIST, -1, -2)):
+            o = sg.get_option(key)
+            sg.set_option(key, good)
+            assert sg.get_option(key) == good
+            with pytest.raises(sg.SgError, match="INVALID_ARG"):
+                sg.set_option(key, bad)
+            sg.set_option(key, o)
     finally:
         sg.set_option(sg.SG_OPT_DENSE_LOG2, old)
 
