@@ -60,36 +60,12 @@ __device__ unsigned long long g_tt[10];
 #define TT_MARK(k) do { } while (0)
 #endif
 
-// SG_TT_DUP=1 (timing experiment, slower): pass 1 marks columns with >= 2 products (atom.or with return)
-// and pass 2 stores the single product of the other columns with a plain store instead of the fp64
-// atomic: tile kernel 87.5 vs 61.6 ms on C3 (the returning atomic OR costs more than the CAS it saves)
-#ifndef SG_TT_DUP
-#define SG_TT_DUP 0
-#endif
 struct __align__(16) TileWarp {
     double acc[CAPW];
     double av[KREG];      // a_ik of the range's row
-#if SG_TT_DUP
-    uint2 bm[TWW];        // (occupancy word, duplicate word): bit c of .y = column c has >= 2 products
-#else
     uint32_t bm[TWW];
-#endif
     uint16_t pref[TWW];
 };
-
-__device__ __forceinline__ uint32_t atom_or_s(uint32_t a, uint32_t v) {
-    uint32_t old;
-    asm volatile("atom.shared.or.b32 %0, [%1], %2;" : "=r"(old) : "r"(a), "r"(v) : "memory");
-    return old;
-}
-__device__ __forceinline__ uint2 ld_u32x2_s(uint32_t a) {
-    uint2 v;
-    asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a) : "memory");
-    return v;
-}
-__device__ __forceinline__ void st_f64_s(uint32_t a, double v) {
-    asm volatile("st.shared.f64 [%0], %1;" ::"r"(a), "d"(v) : "memory");
-}
 
 // one k entry's cursor: B positions [cur, q1) still to come; q0 = start of the B row; lid = tile-pointer id
 // (-1: short row); nx = the prefetched end information for the NEXT tile (long: tp[lid][t+1] of that tile;
@@ -191,11 +167,7 @@ __global__ void __launch_bounds__(TT_T, TT_OCC) k_num_tile(
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     TileWarp& S = reinterpret_cast<TileWarp*>(smem_raw)[wid];
     for (int q = lane; q < CAPW; q += 32) S.acc[q] = 0.0;
-#if SG_TT_DUP
-    for (int q = lane; q < TWW; q += 32) S.bm[q] = make_uint2(0u, 0u);
-#else
     for (int q = lane; q < TWW; q += 32) S.bm[q] = 0u;
-#endif
     __syncwarp();
     const uint32_t a_acc = smem_addr(S.acc), a_bm = smem_addr(S.bm), a_pref = smem_addr(S.pref);
     const int64_t p = B.ncols;
@@ -266,23 +238,9 @@ __global__ void __launch_bounds__(TT_T, TT_OCC) k_num_tile(
                 round(L, 0, true, rc, rv, rk);
                 const int64_t tlo = (int64_t)t * TW;
                 // tlo is a multiple of 32: word (c - tlo) >> 5 = (c >> 5) - (tlo >> 5)
-#if SG_TT_DUP
-                constexpr uint32_t BMS = 8u;  // bytes per bitmap entry
-#else
-                constexpr uint32_t BMS = 4u;
-#endif
-                const uint32_t bw = opaque_u32(a_bm - BMS * ((uint32_t)tlo >> 5));
+                const uint32_t bw = opaque_u32(a_bm - 4u * ((uint32_t)tlo >> 5));
                 const uint32_t pw = opaque_u32(a_pref - 2u * ((uint32_t)tlo >> 5));
-                // the first product of a column sets its occupancy bit; a later one (the OR returns the bit
-                // already set) marks the column as a duplicate
-                auto setbit = [&](int32_t c) {
-                    const uint32_t a = bw + BMS * ((uint32_t)c >> 5), bit = 1u << (c & 31);
-#if SG_TT_DUP
-                    if (atom_or_s(a, bit) & bit) red_or_s(a + 4u, bit);
-#else
-                    red_or_s(a, bit);
-#endif
-                };
+                auto setbit = [&](int32_t c) { red_or_s(bw + 4u * ((uint32_t)c >> 5), 1u << (c & 31)); };
                 TT_MARK(2);
                 // ---- pass 1: bitmap (the first round is in registers, later rounds gather columns only) ----
                 #pragma unroll
@@ -301,25 +259,6 @@ __global__ void __launch_bounds__(TT_T, TT_OCC) k_num_tile(
                 // ---- rank prefix: lane owns words [4 lane, 4 lane + 4) and [128 + 4 lane, 128 + 4 lane + 4) (unit-stride
                 // 16-byte accesses: no bank conflicts); one warp scan per half ----
                 int ut;
-#if SG_TT_DUP
-                {
-                    const uint4* b4 = reinterpret_cast<const uint4*>(S.bm) + 4 * lane;
-                    const uint4 x0 = b4[0], x1 = b4[1], x2 = b4[2], x3 = b4[3];
-                    const int c0 = __popc(x0.x), c1 = __popc(x0.z), c2 = __popc(x1.x), c3 = __popc(x1.z);
-                    const int c4 = __popc(x2.x), c5 = __popc(x2.z), c6 = __popc(x3.x), c7 = __popc(x3.z);
-                    const int sum = c0 + c1 + c2 + c3 + c4 + c5 + c6 + c7;
-                    const int pinc = warp_incl_scan(sum);
-                    ut = __shfl_sync(FULL, pinc, 31);
-                    const int p0 = pinc - sum, p1 = p0 + c0, p2 = p1 + c1, p3 = p2 + c2, p4 = p3 + c3, p5 = p4 + c4,
-                              p6 = p5 + c5, p7 = p6 + c6;
-                    uint4 o;
-                    o.x = (uint32_t)p0 | ((uint32_t)p1 << 16);
-                    o.y = (uint32_t)p2 | ((uint32_t)p3 << 16);
-                    o.z = (uint32_t)p4 | ((uint32_t)p5 << 16);
-                    o.w = (uint32_t)p6 | ((uint32_t)p7 << 16);
-                    reinterpret_cast<uint4*>(S.pref)[lane] = o;
-                }
-#else
                 {
                     const uint4 w0 = reinterpret_cast<const uint4*>(S.bm)[lane];
                     const uint4 w1 = reinterpret_cast<const uint4*>(S.bm)[32 + lane];
@@ -335,7 +274,6 @@ __global__ void __launch_bounds__(TT_T, TT_OCC) k_num_tile(
                     pr[lane] = make_uint2((uint32_t)p0 | ((uint32_t)p1 << 16), (uint32_t)p2 | ((uint32_t)p3 << 16));
                     pr[32 + lane] = make_uint2((uint32_t)p4 | ((uint32_t)p5 << 16), (uint32_t)p6 | ((uint32_t)p7 << 16));
                 }
-#endif
                 SG_BOUND(out + ut <= C_rp[R.row + 1]);
                 __syncwarp();
                 TT_MARK(4);
@@ -345,21 +283,9 @@ __global__ void __launch_bounds__(TT_T, TT_OCC) k_num_tile(
                     auto acc = [&](int32_t c, double b, int ki) {
                         const double v = S.av[ki] * b;
                         const uint32_t cw = (uint32_t)c >> 5, bit = 1u << (c & 31);
-#if SG_TT_DUP
-                        const uint2 wd = ld_u32x2_s(bw + BMS * cw);
-                        const uint32_t wv = wd.x;
-#else
-                        const uint32_t wv = ld_u32_s(bw + BMS * cw);
-#endif
+                        const uint32_t wv = ld_u32_s(bw + 4u * cw);
                         const int rk = (int)ld_u16_s(pw + 2u * cw) + __popc(wv & (bit - 1u)) - r0;
                         if ((unsigned)rk < (unsigned)CAPW) {
-#if SG_TT_DUP
-                            if (!(wd.y & bit)) {  // the column's only product: a plain store, no read
-                                st_f64_s(a_acc + 8u * (uint32_t)rk, v);
-                                st_out(C_col + ob + rk, c);
-                                return;
-                            }
-#endif
                             // the first product of a column finds 0.0 and writes the column (a later one
                             // only if the partial sum is exactly 0.0: the same column again)
                             if (atom_add_f64_s(a_acc + 8u * (uint32_t)rk, v) == 0.0) st_out(C_col + ob + rk, c);
@@ -387,15 +313,8 @@ __global__ void __launch_bounds__(TT_T, TT_OCC) k_num_tile(
                 }
                 {
                     uint4* bm4 = reinterpret_cast<uint4*>(S.bm);
-#if SG_TT_DUP
-                    bm4[4 * lane] = make_uint4(0, 0, 0, 0);
-                    bm4[4 * lane + 1] = make_uint4(0, 0, 0, 0);
-                    bm4[4 * lane + 2] = make_uint4(0, 0, 0, 0);
-                    bm4[4 * lane + 3] = make_uint4(0, 0, 0, 0);
-#else
                     bm4[lane] = make_uint4(0, 0, 0, 0);
                     bm4[32 + lane] = make_uint4(0, 0, 0, 0);
-#endif
                 }
                 out += ut;
                 __syncwarp();
