@@ -283,6 +283,15 @@ sg_status sg_hh_sample(const sg_csr_view* A, uint64_t seed, double f, int64_t* r
                        int32_t* col_out, int64_t* pos_out, void* val_out /*nullable*/, int64_t* s_out /*host*/,
                        int64_t* nnz_out /*host*/, void* stream);
 
+/* Sample ("a smaller instance"; R3): A_S = the rows `rows` (device int64[nrows], any
+ * order, each in [0, A.nrows)) of A as a CSR with all of A's columns (B stays whole). Outputs (device):
+ * rp_out int64[nrows+1], col_out / val_out of capacity `cap` entries; *nnz_out (host) = nnz(A_S), written
+ * even when it exceeds cap. Synchronises (the row-id check and nnz read back). Errors: INVALID_ARG (a row id
+ * out of range, null pointers), SHAPE (nnz(A_S) > cap: nothing copied; call again with the returned size).
+ * The measured-mode Identify of the Python binding (measured_threshold) times the hot path on A_S B. */
+sg_status sg_gather_rows(const sg_csr_view* A, const int64_t* rows, int64_t nrows, int64_t* rp_out, int32_t* col_out,
+                         void* val_out, int64_t cap, int64_t* nnz_out /*host*/, void* stream);
+
 /* The host-only arithmetic of sg_gather (no device work, usable without a GPU): lay holds the
  * per-rank (row_begin, row_end, nnz) triples in rank order. Checks that the blocks are contiguous
  * from row 0 (SHAPE otherwise) and writes begin[r] (first row of rank r, nranks entries), off[r]

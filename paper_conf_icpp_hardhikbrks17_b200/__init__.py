@@ -26,6 +26,7 @@ __all__ = [
     "sg_row_work", "sg_sample_rows", "sg_sample_threshold", "sg_threshold_on_rows", "sg_exhaustive_threshold",
     "sg_cost_curve",
     "sg_partition", "sg_symbolic", "sg_numeric", "sg_gather", "sg_default_cost_model", "spgemm",
+    "sg_gather_rows", "measured_threshold",
     "SG_CAP_L_MAX",
 ]
 
@@ -40,7 +41,8 @@ EXPORTS = ["sg_status_string", "sg_version", "sg_default_cost_model", "sg_row_wo
            "sg_profile_enable", "sg_launch_count", "sg_profile_count", "sg_profile_read", "sg_profile_reset",
            "sg_gather_layout", "sg_threshold_on_rows", "sg_set_option", "sg_get_option",
            "sg_sym_c_create", "sg_sym_c_buffers", "sg_sym_c_layout", "sg_sym_c_assemble", "sg_sym_c_destroy",
-           "sg_copy_device", "sg_default_cost_model_for", "sg_hh_filter", "sg_hh_hstack", "sg_hh_identity2", "sg_hh_sample"]
+           "sg_copy_device", "sg_default_cost_model_for", "sg_hh_filter", "sg_hh_hstack", "sg_hh_identity2", "sg_hh_sample",
+           "sg_gather_rows"]
 
 SG_OPT_VALIDATE, SG_OPT_DENSE_LOG2, SG_OPT_VARIANT, SG_OPT_L2_PERSIST, SG_OPT_TP_MAX_BYTES = 0, 1, 2, 3, 4
 
@@ -138,6 +140,7 @@ def load(build_if_missing: bool = True):
         "sg_hh_hstack": (st, [P, P, P, P, P, P]),
         "sg_hh_identity2": (st, [i64, ctypes.c_int, P, P, P, P]),
         "sg_hh_sample": (st, [P, ctypes.c_uint64, ctypes.c_double, P, P, P, P, P, pi64, pi64, P]),
+        "sg_gather_rows": (st, [V, P, i64, P, P, P, i64, pi64, P]),
         "sg_get_option": (i64, [ctypes.c_int]),
         "sg_plan_get_info": (st, [P, ctypes.POINTER(PlanInfo)]),
         "sg_plan_get_classes": (st, [P, P, P]),
@@ -256,6 +259,75 @@ def sg_sample_rows(n: int, sample_frac: float, seed: int, row_begin: int = 0, ro
     _check(lib().sg_sample_rows(row_begin, row_end, sample_frac, seed, _ptr(out), out.numel(), ctypes.byref(c),
                                 _stream()), "sg_sample_rows")
     return out[: c.value]
+
+
+def sg_gather_rows(A: DeviceCSR, rows: torch.Tensor) -> DeviceCSR:
+    """A_S = the rows `rows` of A (all of A's columns), built on the device (sg_gather_rows)."""
+    _require_cuda()
+    rows = rows.to(device=A.row_ptr.device, dtype=torch.int64).contiguous()
+    nr = rows.numel()
+    rp = torch.empty(nr + 1, dtype=torch.int64, device=A.row_ptr.device)
+    nz = ctypes.c_int64(0)
+    cap = 0
+    while True:
+        col = torch.empty(max(cap, 1), dtype=torch.int32, device=A.row_ptr.device)
+        val = torch.empty(max(cap, 1), dtype=A.val.dtype, device=A.row_ptr.device)
+        code = lib().sg_gather_rows(ctypes.byref(A.view()), _ptr(rows), nr, _ptr(rp), _ptr(col), _ptr(val), cap,
+                                    ctypes.byref(nz), _stream())
+        if code == _STATUS.index("SG_ERR_SHAPE") and nz.value > cap:
+            cap = int(nz.value)  # second call with the size the first one returned
+            continue
+        _check(code, "sg_gather_rows")
+        break
+    m = int(nz.value)
+    return DeviceCSR(nr, A.ncols, rp, col[:m], val[:m])
+
+
+def _threshold_grid(cap: int = SG_CAP_L_MAX) -> list[int]:
+    ts, k = {0, cap}, 0
+    while round(16 * 2 ** (k / 4)) <= cap:
+        ts.add(int(round(16 * 2 ** (k / 4))))
+        k += 1
+    return sorted(ts)
+
+
+def measured_threshold(A: DeviceCSR, B: DeviceCSR, sample_frac: float = 0.01, seed: int = 1, reps: int = 1,
+                       grid: list[int] | None = None):
+    """The paper's measured Identify ("identify the best threshold for the sample by running
+    the algorithm"; L141): Sample the rows S (sg_sample_rows, R3/R4), build A_S = A[S, :] with B
+    whole (sg_gather_rows), time sg_symbolic + sg_numeric of A_S B on the device at the candidate thresholds
+    of a geometric grid — every 8th point first, then the 17 points around the fastest — and Extrapolate the
+    fastest t unchanged (L236). The default Identify of sg_sample_threshold evaluates the calibrated cost
+    model instead (deterministic, the parity-tested one). Returns (thr, {"T_ms": {t: ms}, "sample_rows": |S|})."""
+    _require_cuda()
+    S = sg_sample_rows(A.nrows, sample_frac, seed, device=A.row_ptr.device)
+    if S.numel() == 0:
+        raise SgError(_STATUS.index("SG_ERR_EMPTY_SAMPLE"), "measured_threshold")
+    AS = sg_gather_rows(A, S)
+    G = grid or _threshold_grid()
+    timed: dict[int, float] = {}
+
+    def T(t: int) -> float:
+        if t not in timed:
+            best = None
+            for _ in range(max(1, reps)):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(torch.cuda.current_stream())
+                plan = sg_symbolic(AS, B, t)
+                col, val = sg_numeric(plan, AS, B)
+                e1.record(torch.cuda.current_stream())
+                torch.cuda.synchronize()
+                plan.destroy()
+                del col, val
+                ms = e0.elapsed_time(e1)
+                best = ms if best is None else min(best, ms)
+            timed[t] = best
+        return timed[t]
+
+    coarse = G[::8] + ([G[-1]] if (len(G) - 1) % 8 else [])
+    k = G.index(min(coarse, key=T))
+    thr = min(G[max(0, k - 8): k + 9], key=T)
+    return thr, {"T_ms": dict(sorted(timed.items())), "sample_rows": int(S.numel())}
 
 
 def sg_sample_threshold(A: DeviceCSR, B: DeviceCSR, sample_frac: float, seed: int, cm: CostModel | None = None):

@@ -1040,6 +1040,41 @@ sg_status sg_hh_sample(const sg_csr_view* A, uint64_t seed, double f, int64_t* r
     return SG_OK;
 }
 
+sg_status sg_gather_rows(const sg_csr_view* A, const int64_t* rows, int64_t nrows, int64_t* rp_out, int32_t* col_out,
+                         void* val_out, int64_t cap, int64_t* nnz_out, void* stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    init_pool();
+    sg_status st = validate_one(A, s);
+    if (st != SG_OK) return st;
+    if (nrows < 0 || cap < 0 || !rp_out || !nnz_out || (nrows > 0 && !rows)) return SG_ERR_INVALID_ARG;
+    Mat m = mat_of(A);
+    {
+        Scratch sc(s);  // row ids in range (one flag read back)
+        unsigned long long* bad = (unsigned long long*)sc.get(sizeof(unsigned long long));
+        if (!bad) return SG_ERR_OOM;
+        unsigned long long hb = 0;
+        CK(cudaMemsetAsync(bad, 0, sizeof(unsigned long long), s));
+        CK(launch_check_rows(rows, nrows, A->nrows, bad, s));
+        CK(cudaMemcpyAsync(&hb, bad, sizeof(hb), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (hb) return SG_ERR_INVALID_ARG;
+    }
+    Scratch sc(s);
+    int64_t* len = (int64_t*)sc.get(sizeof(int64_t) * (size_t)(nrows > 0 ? nrows : 1));
+    void* tmp = sc.get(scan_tmp_bytes(nrows));
+    if (!len || !tmp) return SG_ERR_OOM;
+    CK(launch_rows_len(m, rows, nrows, len, s));
+    CK(scan_exclusive(len, rp_out, nrows, tmp, s));
+    int64_t nz = 0;
+    CK(cudaMemcpyAsync(&nz, rp_out + nrows, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    *nnz_out = nz;
+    if (nz > cap) return SG_ERR_SHAPE;
+    if (nz > 0 && (!col_out || !val_out)) return SG_ERR_INVALID_ARG;
+    CK(launch_rows_copy(m, rows, nrows, rp_out, col_out, val_out, s));
+    return SG_OK;
+}
+
 sg_status sg_copy_device(void* dst, const void* src, int64_t bytes, void* stream) {
     if (bytes < 0 || (bytes > 0 && (!dst || !src))) return SG_ERR_INVALID_ARG;
     if (bytes == 0) return SG_OK;

@@ -124,7 +124,44 @@ __global__ void k_hh_rows_of_rank(int64_t n, const int64_t* __restrict__ keep, c
         if (keep[i]) rows_of_rank[rank[i]] = i;
 }
 
+// A[S, :] (the row sample of the measured Identify): lengths of the listed rows, then a warp-per-row copy
+__global__ void k_rows_len(Mat M, const int64_t* __restrict__ rows, int64_t nr, int64_t* __restrict__ len) {
+    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < nr; j += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t i = rows[j];
+        len[j] = M.rp[i + 1] - M.rp[i];
+    }
+}
+
+template <class VT>
+__global__ void k_rows_copy(Mat M, const int64_t* __restrict__ rows, int64_t nr, const int64_t* __restrict__ out_rp,
+                            int32_t* __restrict__ col, VT* __restrict__ val) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t j = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; j < nr;
+         j += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+        const int64_t o = out_rp[j], n = out_rp[j + 1] - o, s = M.rp[rows[j]];
+        for (int64_t q = lane; q < n; q += 32) {
+            col[o + q] = __ldg(M.col + s + q);
+            val[o + q] = __ldg(reinterpret_cast<const VT*>(M.val) + s + q);
+        }
+    }
+}
+
 }  // namespace
+
+cudaError_t launch_rows_len(const Mat& M, const int64_t* rows, int64_t nr, int64_t* len, cudaStream_t s) {
+    if (nr <= 0) return cudaSuccess;
+    SG_LAUNCH("k_rows_len", s, (k_rows_len<<<grid_for(nr, 256, 148 * 8), 256, 0, s>>>(M, rows, nr, len)));
+    return cudaGetLastError();
+}
+
+cudaError_t launch_rows_copy(const Mat& M, const int64_t* rows, int64_t nr, const int64_t* out_rp, int32_t* col, void* val,
+                             cudaStream_t s) {
+    if (nr <= 0) return cudaSuccess;
+    const int g = grid_for(nr, 8, 148 * 16);
+    if (M.dt == 0) SG_LAUNCH("k_rows_copy", s, (k_rows_copy<double><<<g, 256, 0, s>>>(M, rows, nr, out_rp, col, (double*)val)));
+    else SG_LAUNCH("k_rows_copy", s, (k_rows_copy<float><<<g, 256, 0, s>>>(M, rows, nr, out_rp, col, (float*)val)));
+    return cudaGetLastError();
+}
 
 cudaError_t launch_hh_len(const Mat& M, int64_t t, int high, int64_t* len, cudaStream_t s) {
     if (M.nrows <= 0) return cudaSuccess;

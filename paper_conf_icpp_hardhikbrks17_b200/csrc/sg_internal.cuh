@@ -191,6 +191,9 @@ cudaError_t launch_class_usum_dev(const int64_t* w, const int64_t* u, int64_t nr
                                   unsigned long long* out, cudaStream_t s);
 // HH four-block variant (sg_hh.cu)
 cudaError_t launch_hh_len(const Mat& M, int64_t t, int high, int64_t* len, cudaStream_t s);
+cudaError_t launch_rows_len(const Mat& M, const int64_t* rows, int64_t nr, int64_t* len, cudaStream_t s);
+cudaError_t launch_rows_copy(const Mat& M, const int64_t* rows, int64_t nr, const int64_t* out_rp, int32_t* col, void* val,
+                             cudaStream_t s);
 cudaError_t launch_hh_copy(const Mat& M, const int64_t* out_rp, int32_t* col, void* val, cudaStream_t s);
 cudaError_t launch_hh_hstack(const Mat& P, const Mat& Q, int64_t* rp, int32_t* col, void* val, int pass, cudaStream_t s);
 cudaError_t launch_hh_identity2(int64_t p, int dt, int64_t* rp, int32_t* col, void* val, cudaStream_t s);
