@@ -324,10 +324,16 @@ def measured_threshold(A: DeviceCSR, B: DeviceCSR, sample_frac: float = 0.01, se
             timed[t] = best
         return timed[t]
 
+    thr = _coarse_fine(G, T)
+    return thr, {"T_ms": dict(sorted(timed.items())), "sample_rows": int(S.numel())}
+
+
+def _coarse_fine(G: list[int], T) -> int:
+    """The measured Identify's search over the sorted grid G: every 8th point (and the last), then the 17
+    points around the fastest of those; returns the fastest point evaluated (host logic, CPU-tested)."""
     coarse = G[::8] + ([G[-1]] if (len(G) - 1) % 8 else [])
     k = G.index(min(coarse, key=T))
-    thr = min(G[max(0, k - 8): k + 9], key=T)
-    return thr, {"T_ms": dict(sorted(timed.items())), "sample_rows": int(S.numel())}
+    return min(G[max(0, k - 8): k + 9], key=T)
 
 
 def sg_sample_threshold(A: DeviceCSR, B: DeviceCSR, sample_frac: float, seed: int, cm: CostModel | None = None):

@@ -88,3 +88,23 @@ def test_negative_cost_coefficients_rejected_before_device_work():
     thr = ctypes.c_int64(0)
     st = L.sg_sample_threshold(ctypes.byref(v), ctypes.byref(v), 0.5, 1, ctypes.byref(cm), ctypes.byref(thr), None, None)
     assert st == 1  # SG_ERR_INVALID_ARG
+
+
+def test_measured_identify_search_logic():
+    """measured_threshold's grid and coarse -> fine search (host logic): the grid is 0, 16 * 2^(k/4) and
+    cap_L; on a unimodal time curve the search returns its minimum, and it only evaluates coarse points
+    plus the 17 around the coarse best."""
+    import paper_conf_icpp_hardhikbrks17_b200 as sg
+    G = sg._threshold_grid()
+    assert G[0] == 0 and G[1] == 16 and G[-1] == sg.SG_CAP_L_MAX and G == sorted(set(G))
+    assert all(1.0 < b / a <= 1.25 for a, b in zip(G[1:-1], G[2:-1]))  # 2^(1/4) steps, rounded
+    for best in (0, 16, 181, 1024, 3444, 4096):
+        seen = []
+
+        def T(t, best=best):
+            seen.append(t)
+            return abs(t - best) + 1.0
+        assert sg._coarse_fine(G, T) == best
+        coarse = set(G[::8]) | {G[-1]}
+        k = G.index(min(coarse, key=lambda t: abs(t - best)))
+        assert set(seen) <= coarse | set(G[max(0, k - 8): k + 9])
