@@ -28,16 +28,16 @@ namespace sg {
 #define SG_TT_WARPS 4
 #endif
 #ifndef SG_TT_OCC
-#define SG_TT_OCC 7
+#define SG_TT_OCC 8
 #endif
 #ifndef SG_CAPW
-#define SG_CAPW 640
+#define SG_CAPW 512
 #endif
 #ifndef SG_TT_CHUNK
 #define SG_TT_CHUNK 1
 #endif
 #ifndef SG_TT_NB
-#define SG_TT_NB 4
+#define SG_TT_NB 3
 #endif
 constexpr int TT_WARPS = SG_TT_WARPS;  // warps per CTA (independent; the CTA only shares the launch)
 constexpr int TT_T = 32 * TT_WARPS;
