@@ -188,3 +188,42 @@ def test_measured_threshold_is_the_fastest_evaluated_candidate():
     R = oracle.spgemm(A, A, with_absmag=True)
     assert np.array_equal(rp, R.row_ptr)
     compare_rows(rp, col, val, R, "f64")
+
+
+def test_tile_kernel_rank_windows_of_a_dense_tile(options):
+    """A tile with more outputs than the warp-tile kernel's accumulator (512 entries) is accumulated in
+    rank windows: rows of <= 64 k entries whose B rows fill most of tile 0 (8192 columns) — integer values,
+    bit-exact against the oracle, with the warp-tile kernel forced (variant bit 5) and no dense-window rows."""
+    rng = np.random.default_rng(11)
+    n, p = 256, 20000
+    rows, cols = [], []
+    for i in range(n):  # B = A: row i holds 40-64 columns, most of them in [0, 8192)
+        k = int(rng.integers(40, 65))
+        c = np.unique(np.concatenate([rng.choice(8192, k - 4, replace=False), rng.choice(np.arange(8192, p), 4)]))
+        rows.append(np.full(c.size, i)); cols.append(c)
+    r = np.concatenate(rows); c = np.concatenate(cols)
+    rp = np.zeros(n + 1, dtype=np.int64); np.add.at(rp, r + 1, 1); rp = np.cumsum(rp)
+    val = rng.integers(1, 5, size=c.size).astype(np.float64)
+    # B: p x p, rows [0, n) as generated, the rest empty; A: the same pattern with columns folded into
+    # [0, n) (every k of A hits a non-empty B row), so each row of C fills most of tile 0
+    Brp = np.concatenate([rp, np.full(p - n, rp[-1], dtype=np.int64)])
+    B = gen.CSR(p, p, Brp, c.astype(np.int32), val, "dense-tile-B")
+    Ac = (c % n).astype(np.int64)
+    order = np.lexsort((Ac, r))
+    r2, c2, v2 = r[order], Ac[order], val[order]
+    keep = np.ones(r2.size, bool); keep[1:] = (r2[1:] != r2[:-1]) | (c2[1:] != c2[:-1])
+    r2, c2, v2 = r2[keep], c2[keep], v2[keep]
+    rp2 = np.zeros(n + 1, dtype=np.int64); np.add.at(rp2, r2 + 1, 1); rp2 = np.cumsum(rp2)
+    A = gen.CSR(n, p, rp2, c2.astype(np.int32), v2, "dense-tile-A")
+    sg.set_option(sg.SG_OPT_DENSE_LOG2, 62)
+    sg.set_option(sg.SG_OPT_VARIANT, 32)
+    dA, dB = sg.DeviceCSR.from_host(A), sg.DeviceCSR.from_host(B)
+    plan = sg.sg_symbolic(dA, dB, 0)
+    col, cval = sg.sg_numeric(plan, dA, dB)
+    torch.cuda.synchronize()
+    R = oracle.spgemm(A, B)
+    crp = plan.row_ptr.cpu().numpy()
+    assert np.array_equal(crp, R.row_ptr)
+    assert int(np.diff(R.row_ptr).max()) > 512  # some tile holds more outputs than one accumulator window
+    compare_rows(crp, col.cpu().numpy(), cval.cpu().numpy(), R, "f64", exact_values=True)
+    plan.destroy()
