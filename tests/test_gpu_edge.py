@@ -227,3 +227,32 @@ def test_tile_kernel_rank_windows_of_a_dense_tile(options):
     assert int(np.diff(R.row_ptr).max()) > 512  # some tile holds more outputs than one accumulator window
     compare_rows(crp, col.cpu().numpy(), cval.cpu().numpy(), R, "f64", exact_values=True)
     plan.destroy()
+
+
+def _random_csr(rng, nrows, ncols, deg, name):
+    rows, cols = [], []
+    for i in range(nrows):
+        c = np.unique(rng.integers(0, ncols, size=int(rng.integers(1, 2 * deg))))
+        rows.append(np.full(c.size, i)); cols.append(c)
+    r = np.concatenate(rows); c = np.concatenate(cols)
+    rp = np.zeros(nrows + 1, dtype=np.int64); np.add.at(rp, r + 1, 1)
+    return gen.CSR(nrows, ncols, np.cumsum(rp), c.astype(np.int32), rng.integers(1, 5, size=c.size).astype(np.float64), name)
+
+
+def test_light_sorted_and_hash_bins_in_one_plan():
+    """The sorted light path needs c < 2^(32 - log2 U): with B.ncols = 2^24 bin 8 (U = 256) is sorted and
+    bin 9 (U = 512) falls back to the hash path in the same plan; C bit-exact against the oracle."""
+    rng = np.random.default_rng(4)
+    A = _random_csr(rng, 2048, 2048, 20, "A")
+    B = _random_csr(rng, 2048, 1 << 24, 20, "B")
+    dA, dB = sg.DeviceCSR.from_host(A), sg.DeviceCSR.from_host(B)
+    plan = sg.sg_symbolic(dA, dB, 4096)
+    col, val = sg.sg_numeric(plan, dA, dB)
+    torch.cuda.synchronize()
+    R = oracle.spgemm(A, B)
+    w = oracle.row_work(A, B)
+    assert ((w > 256) & (w <= 512)).any() and ((w > 128) & (w <= 256)).any()  # both bins populated
+    crp = plan.row_ptr.cpu().numpy()
+    assert np.array_equal(crp, R.row_ptr)
+    compare_rows(crp, col.cpu().numpy(), val.cpu().numpy(), R, "f64", exact_values=True)
+    plan.destroy()
